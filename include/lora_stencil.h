@@ -1,0 +1,156 @@
+/*
+ * lora_stencil.h — C-ABI of the B200-native LoRAStencil engine.
+ *
+ * What the library computes (PAPER.md = /root/reference/PAPER.md, "P:n" = its line n):
+ *   A time-iterated d-dimensional FP64 stencil (d = 2, 3): every interior point is replaced,
+ *   T times, by the weighted sum of its (2r+1)^d neighbourhood (§I; eq. 2).
+ *   The weights are factored on the host into rank-1 terms u_k v_k^T (eq. 8 P:149-153;
+ *   Pyramidal Matrix Adaptation, eq. 15) and each term is evaluated as the banded
+ *   Toeplitz chain U_k X V_k (eq. 5-7, eq. 9): Residual Dimension
+ *   Gathering (§III-B), on FP64 tensor cores with Butterfly Vector Swapping (§III-D, eq. 17)
+ *   or on the FP64 CUDA-core pipe, chosen per plan (see lora_engine).  3D stencils are
+ *   evaluated plane by plane (Alg. 2).
+ *
+ * Conventions:
+ *   * Arrays are PADDED: extent N_i + 2r along axis i, C order, slowest axis first.
+ *     The r-wide halo holds fixed Dirichlet boundary values and is never updated.
+ *   * weights[a0][a1]([a2]) multiplies in[x0+a0-r][x1+a1-r]([x2+a2-r])  (correlation).
+ *   * Jacobi: each step reads only the previous step.
+ *
+ * Errors: functions return LORA_OK (0) or a negative lora_status; lora_stencil_plan returns
+ * NULL on failure.  lora_stencil_last_error() returns a thread-local message for the last
+ * failure on the calling thread.  Kernel launch errors are reported synchronously;
+ * asynchronous device faults surface at the caller's next synchronisation (set the
+ * environment variable LORA_SYNC_CHECK=1 to synchronise and check inside every run call).
+ *
+ * Threading: a plan is not re-entrant (its device scratch is shared); distinct plans may be
+ * used concurrently from different threads.
+ */
+#ifndef LORA_STENCIL_H_
+#define LORA_STENCIL_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct lora_plan lora_plan; /* opaque; owns host factors, device scratch/pinned buffers */
+typedef struct lora_comm lora_comm; /* opaque; owns an ncclComm_t and two CUDA streams        */
+
+typedef enum {
+  LORA_OK = 0,
+  LORA_ERR_INVALID_ARG = -1, /* bad pointer, size, radius, ndim, timesteps < 0           */
+  LORA_ERR_UNSUPPORTED = -2, /* radius > 4, engine not available for this shape          */
+  LORA_ERR_ALIAS = -3,       /* in and out overlap                                        */
+  LORA_ERR_CUDA = -4,        /* a CUDA runtime call or kernel launch failed               */
+  LORA_ERR_NCCL = -5,        /* NCCL missing or a NCCL call failed                        */
+  LORA_ERR_OOM = -6,         /* device or pinned host allocation failed                   */
+  LORA_ERR_FACTOR = -7       /* the factorisation does not reconstruct W to 1e-14          */
+} lora_status;
+
+/* Engine used for the rank-1 terms (the scalar C_{h+1} term and single-weight 3D planes are
+ * always point-wise DFMA, P:275 and Alg. 2 lines 3-5). */
+typedef enum {
+  LORA_ENGINE_AUTO = 0,     /* planner picks the engine with the lowest issued FP64 work    */
+  LORA_ENGINE_TC = 1,       /* RDG chains U X V on FP64 tensor cores (mma.m8n8k4.f64), BVS  */
+  LORA_ENGINE_RDG_CUDA = 2, /* RDG chains as two banded passes on the FP64 CUDA-core pipe   */
+  LORA_ENGINE_DIRECT = 3    /* no factorisation: the (2r+1)^d-point sum on CUDA cores (K11) */
+} lora_engine;
+
+typedef struct {
+  int engine;  /* lora_engine; 0 = AUTO                                                     */
+  int fuse_k;  /* time steps per HBM round trip; 0 = planner's choice, 1 = no fusion          */
+  int reserved[6];
+} lora_plan_opts;
+
+typedef struct {               /* filled by lora_stencil_plan_query                          */
+  int ndim, radius;
+  int64_t grid[3];             /* interior extents (slowest first); grid[2] = 1 in 2D         */
+  int engine;                  /* lora_engine actually used                                   */
+  int n_terms;                 /* rank-1 terms over all planes, incl. scalar / point-wise     */
+  int n_tc_chain;              /* terms evaluated as a two-stage chain U X V                  */
+  int n_tc_single;             /* star arms: one banded stage (a unit-vector factor)          */
+  int n_cuda;                  /* scalar / point-wise terms on the DFMA pipe                  */
+  int n_planes_pointwise;      /* 3D planes with exactly one nonzero weight (Alg. 2 line 3)   */
+  int z_symmetric;             /* 3D: W[r-k] == W[r+k] for all k (planes pre-added)          */
+  int fuse_k;                  /* time steps per HBM round trip                               */
+  int halo_depth;              /* fuse_k * radius                                             */
+  int tile_m, tile_n;          /* CTA output tile (rows, columns of the fastest axis)         */
+  double recon_err;            /* max|sum u v^T - W| / max|W|                                 */
+  double growth;               /* sum_k ||u_k||_1 ||v_k||_1 / ||W||_1                         */
+  double fma_per_point_issued; /* FP64 FMAs issued per point per step by the chosen engine    */
+  double fma_per_point_direct; /* (2r+1)^d, nonzero weights only                              */
+  double fma_per_point_separable; /* sum over terms of (len u + len v) + point-wise terms      */
+} lora_plan_info;
+
+/* Plans a stencil.  Host-only work (no CUDA call): validates, factors every 2D plane
+ * (star arms / PMA / complete-pivot elimination, Q6), checks the reconstruction
+ * (<= 1e-14 relative, else NULL with LORA_ERR_FACTOR), and picks engine, tile and fusion.
+ *   weights    host, (2*radius+1)^ndim doubles, row-major, copied (caller keeps ownership)
+ *   ndim       2 or 3
+ *   radius     1..4
+ *   grid_shape host, ndim interior extents (slowest first), each >= 1
+ * The plan binds to the CUDA device that is current at its first run call. */
+lora_plan* lora_stencil_plan(const double* weights, int ndim, int radius, const int64_t* grid_shape);
+/* As lora_stencil_plan with options (opts may be NULL = defaults). */
+lora_plan* lora_stencil_plan_ex(const double* weights, int ndim, int radius, const int64_t* grid_shape,
+                                const lora_plan_opts* opts);
+
+/* Runs `timesteps` Jacobi steps.  `in` and `out` are DEVICE pointers to padded arrays of
+ * prod(N_i + 2r) doubles, 8-byte aligned (16-byte alignment and an even padded last extent
+ * enable TMA staging).  `in` is never written; on return (stream-ordered) `out` holds step T
+ * in its interior and a copy of `in`'s halo.  timesteps = 0 copies.  in/out must not overlap
+ * (LORA_ERR_ALIAS).  `stream` is a cudaStream_t (NULL = legacy default stream).  The first
+ * call allocates the plan's device scratch (one padded buffer) on the current device. */
+int lora_stencil_run(lora_plan* p, const double* in, double* out, int64_t timesteps, void* stream);
+
+/* The same computation from HOST buffers: copies `in_host` to plan-owned device memory,
+ * runs, and copies the result to `out_host`, all ordered on `stream`, and synchronises the
+ * stream before returning.  Pinned (cudaHostAlloc / cudaHostRegister) buffers give full
+ * PCIe/C2C bandwidth; pageable buffers work but are staged by the driver. */
+int lora_stencil_run_host(lora_plan* p, const double* in_host, double* out_host, int64_t timesteps, void* stream);
+
+/* Fills *info from the plan (host-only). */
+int lora_stencil_plan_query(const lora_plan* p, lora_plan_info* info);
+
+/* Host-only access to the factorisation, for tests and tools.  For plane q (0 in 2D,
+ * 0..2r in 3D) the plan holds terms k = 0..n-1, each a pair of vectors of length 2r+1
+ * (centred, zero-padded) with  W_plane = sum_k u_k v_k^T.  Writes at most max_terms terms:
+ * term_plane[k], term_kind[k] (0 chain, 1 single-stage arm, 2 scalar/point-wise),
+ * term_radius[k] (support radius of the term), u[k*(2r+1) + i], v[k*(2r+1) + j].
+ * *n_terms receives the total count.  Buffers may be NULL when max_terms = 0. */
+int lora_stencil_plan_terms(const lora_plan* p, int max_terms, int* n_terms, int* term_plane, int* term_kind,
+                            int* term_radius, double* u, double* v);
+
+void lora_stencil_plan_destroy(lora_plan* p);
+
+/* ---- multi-GPU: slab decomposition along the slowest axis, halo exchange over NCCL ---- */
+
+/* Size of the opaque NCCL unique id (ncclUniqueId, 128 bytes). */
+size_t lora_stencil_comm_id_size(void);
+/* Rank 0 creates an id (host bytes, lora_stencil_comm_id_size() long) and broadcasts it,
+ * e.g. with torch.distributed.broadcast_object_list.  NCCL is loaded at run time from the
+ * libnccl.so.2 the process already has (torch's) or the system one. */
+int lora_stencil_comm_get_id(void* id_out);
+/* Collective over `nranks` processes, one GPU each (current device). */
+int lora_stencil_comm_init(lora_comm** c, int nranks, int rank, const void* nccl_unique_id);
+/* Collective: every rank calls with the same timesteps.  `p` is planned with this rank's
+ * LOCAL interior shape (n0_local, N1[, N2]) — uneven splits are allowed.  in_local/out_local
+ * are device padded arrays of that local shape.  Rank 0's low halo and rank n-1's high halo
+ * are the physical Dirichlet boundary; the other slab-edge halos are overwritten each step
+ * by the neighbours' edge rows/planes.  Ordered on `stream`. */
+int lora_stencil_run_dist(lora_plan* p, lora_comm* c, const double* in_local, double* out_local, int64_t timesteps,
+                          void* stream);
+void lora_stencil_comm_destroy(lora_comm* c);
+
+/* Thread-local message for the last failure on this thread ("" if none). */
+const char* lora_stencil_last_error(void);
+/* Library version string. */
+const char* lora_stencil_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LORA_STENCIL_H_ */

@@ -1,0 +1,196 @@
+// C-ABI layer (include/lora_stencil.h): validation, device state, the time loop.
+// The time loop (P:21 Jacobi iteration; eq. 18 counts T steps) ping-pongs between `out` and one
+// plan-owned scratch buffer so that the last step lands in `out`; `in` is never written.
+#include <cuda_runtime.h>
+
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "kernels.hpp"
+#include "plan.hpp"
+
+struct lora_plan : lora::Plan {};
+
+namespace lora {
+thread_local std::string g_err;
+int fail(int code, const std::string& msg) { g_err = msg; return code; }
+int cuda_fail(cudaError_t e, const char* what) {
+  g_err = std::string(what) + ": " + cudaGetErrorString(e);
+  return LORA_ERR_CUDA;
+}
+bool sync_check() {
+  static int v = [] { const char* e = std::getenv("LORA_SYNC_CHECK"); return e && e[0] == '1' ? 1 : 0; }();
+  return v != 0;
+}
+
+// Binds the plan to the current device at first use and allocates `want_scratch` buffers.
+int ensure_device(Plan& p, bool want_scratch) {
+  int dev = -1;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+  if (p.device < 0) p.device = dev;
+  if (p.device != dev) return fail(LORA_ERR_INVALID_ARG, "plan is bound to another CUDA device");
+  if (want_scratch && !p.scratch) {
+    e = cudaMalloc(&p.scratch, p.elems * sizeof(double));
+    if (e != cudaSuccess) { cudaGetLastError(); p.scratch = nullptr; return fail(LORA_ERR_OOM, "cudaMalloc(scratch) failed"); }
+  }
+  return LORA_OK;
+}
+
+cudaError_t step(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  switch (p.engine) {
+    case LORA_ENGINE_TC: return launch_tc2d(p, src, dst, s);
+    case LORA_ENGINE_RDG_CUDA: return launch_rdg2d(p, src, dst, s);
+    default: return launch_direct(p, src, dst, s);
+  }
+}
+
+int run_device(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s) {
+  const size_t bytes = p.elems * sizeof(double);
+  if (T == 0) {
+    cudaError_t e = cudaMemcpyAsync(out, in, bytes, cudaMemcpyDeviceToDevice, s);
+    return e == cudaSuccess ? LORA_OK : cuda_fail(e, "cudaMemcpyAsync");
+  }
+  int rc = ensure_device(p, T >= 2);
+  if (rc) return rc;
+  cudaError_t e = launch_copy_halo(p, in, out, s);
+  if (e != cudaSuccess) return cuda_fail(e, "copy_halo launch");
+  if (T >= 2) {
+    e = launch_copy_halo(p, in, p.scratch, s);
+    if (e != cudaSuccess) return cuda_fail(e, "copy_halo launch");
+  }
+  // step t (1..T) writes `out` when (T - t) is even, else the scratch buffer.
+  const double* src = in;
+  for (int64_t t = 1; t <= T; ++t) {
+    double* dst = ((T - t) % 2 == 0) ? out : p.scratch;
+    e = step(p, src, dst, s);
+    if (e != cudaSuccess) return cuda_fail(e, "stencil kernel launch");
+    src = dst;
+  }
+  if (sync_check()) {
+    e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return cuda_fail(e, "LORA_SYNC_CHECK stream sync");
+  }
+  return LORA_OK;
+}
+}  // namespace lora
+
+using namespace lora;
+
+extern "C" {
+
+const char* lora_stencil_last_error(void) { return g_err.c_str(); }
+const char* lora_stencil_version(void) { return "lora_stencil_b200 0.1 (sm_100a)"; }
+
+lora_plan* lora_stencil_plan_ex(const double* weights, int ndim, int radius, const int64_t* grid_shape,
+                                const lora_plan_opts* opts) {
+  lora_plan* p = new (std::nothrow) lora_plan();
+  if (!p) { g_err = "out of host memory"; return nullptr; }
+  std::string err;
+  int rc = plan_build(*p, weights, ndim, radius, grid_shape, opts, err);
+  if (rc != LORA_OK) { g_err = err; delete p; return nullptr; }
+  g_err.clear();
+  return p;
+}
+
+lora_plan* lora_stencil_plan(const double* weights, int ndim, int radius, const int64_t* grid_shape) {
+  return lora_stencil_plan_ex(weights, ndim, radius, grid_shape, nullptr);
+}
+
+void lora_stencil_plan_destroy(lora_plan* p) {
+  if (!p) return;
+  if (p->device >= 0) {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (cur != p->device) cudaSetDevice(p->device);
+    if (p->scratch) cudaFree(p->scratch);
+    if (p->dev_in) cudaFree(p->dev_in);
+    if (p->dev_out) cudaFree(p->dev_out);
+    if (cur >= 0 && cur != p->device) cudaSetDevice(cur);
+  }
+  delete p;
+}
+
+int lora_stencil_plan_query(const lora_plan* p, lora_plan_info* info) {
+  if (!p || !info) return fail(LORA_ERR_INVALID_ARG, "NULL plan or info");
+  std::memset(info, 0, sizeof(*info));
+  info->ndim = p->ndim; info->radius = p->R;
+  for (int i = 0; i < 3; ++i) info->grid[i] = i < p->ndim ? p->N[i] : 1;
+  info->engine = p->engine;
+  info->n_terms = (int)p->terms.size();
+  for (const Term& t : p->terms) {
+    if (t.kind == kChain) info->n_tc_chain++;
+    else if (t.kind == kArm) info->n_tc_single++;
+    else info->n_cuda++;
+  }
+  info->n_planes_pointwise = p->n_planes_point;
+  info->z_symmetric = p->z_symmetric;
+  info->fuse_k = p->fuse_k;
+  info->halo_depth = p->fuse_k * p->R;
+  info->tile_m = p->tile_m; info->tile_n = p->tile_n;
+  info->recon_err = p->recon_err;
+  info->growth = p->growth;
+  info->fma_per_point_issued = p->fma_issued;
+  info->fma_per_point_direct = p->fma_direct;
+  info->fma_per_point_separable = p->fma_separable;
+  return LORA_OK;
+}
+
+int lora_stencil_plan_terms(const lora_plan* p, int max_terms, int* n_terms, int* term_plane, int* term_kind,
+                            int* term_radius, double* u, double* v) {
+  if (!p || !n_terms) return fail(LORA_ERR_INVALID_ARG, "NULL plan or n_terms");
+  if (max_terms > 0 && (!term_plane || !term_kind || !term_radius || !u || !v))
+    return fail(LORA_ERR_INVALID_ARG, "NULL output buffer");
+  const int n = 2 * p->R + 1;
+  *n_terms = (int)p->terms.size();
+  for (int k = 0; k < max_terms && k < (int)p->terms.size(); ++k) {
+    const Term& t = p->terms[k];
+    term_plane[k] = t.plane; term_kind[k] = t.kind; term_radius[k] = t.r;
+    for (int i = 0; i < n; ++i) { u[k * n + i] = t.u[i]; v[k * n + i] = t.v[i]; }
+  }
+  return LORA_OK;
+}
+
+int lora_stencil_run(lora_plan* p, const double* in, double* out, int64_t timesteps, void* stream) {
+  if (!p || !in || !out) return fail(LORA_ERR_INVALID_ARG, "NULL plan, in or out");
+  if (timesteps < 0) return fail(LORA_ERR_INVALID_ARG, "timesteps must be >= 0");
+  if ((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(out)) & 7)
+    return fail(LORA_ERR_INVALID_ARG, "in/out must be 8-byte aligned");
+  const size_t bytes = p->elems * sizeof(double);
+  const char* a = reinterpret_cast<const char*>(in);
+  const char* b = reinterpret_cast<const char*>(out);
+  if (a < b + bytes && b < a + bytes) return fail(LORA_ERR_ALIAS, "in and out overlap");
+  int rc = run_device(*p, in, out, timesteps, static_cast<cudaStream_t>(stream));
+  if (rc == LORA_OK) g_err.clear();
+  return rc;
+}
+
+int lora_stencil_run_host(lora_plan* p, const double* in_host, double* out_host, int64_t timesteps, void* stream) {
+  if (!p || !in_host || !out_host) return fail(LORA_ERR_INVALID_ARG, "NULL plan, in or out");
+  if (timesteps < 0) return fail(LORA_ERR_INVALID_ARG, "timesteps must be >= 0");
+  int rc = ensure_device(*p, false);
+  if (rc) return rc;
+  const size_t bytes = p->elems * sizeof(double);
+  if (!p->dev_in) {
+    if (cudaMalloc(&p->dev_in, bytes) != cudaSuccess) { cudaGetLastError(); p->dev_in = nullptr; return fail(LORA_ERR_OOM, "cudaMalloc(dev_in)"); }
+  }
+  if (!p->dev_out) {
+    if (cudaMalloc(&p->dev_out, bytes) != cudaSuccess) { cudaGetLastError(); p->dev_out = nullptr; return fail(LORA_ERR_OOM, "cudaMalloc(dev_out)"); }
+  }
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaMemcpyAsync(p->dev_in, in_host, bytes, cudaMemcpyHostToDevice, s);
+  if (e != cudaSuccess) return cuda_fail(e, "H2D copy");
+  rc = run_device(*p, p->dev_in, p->dev_out, timesteps, s);
+  if (rc) return rc;
+  e = cudaMemcpyAsync(out_host, p->dev_out, bytes, cudaMemcpyDeviceToHost, s);
+  if (e != cudaSuccess) return cuda_fail(e, "D2H copy");
+  e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(e, "stream sync");
+  g_err.clear();
+  return LORA_OK;
+}
+
+}  // extern "C"

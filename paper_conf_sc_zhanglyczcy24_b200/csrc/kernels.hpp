@@ -1,0 +1,25 @@
+// Launchers for the device kernels (internal).  Every launcher enqueues on `s` and returns
+// cudaGetLastError() of the launch.
+#pragma once
+#include <cuda_runtime.h>
+
+#include "plan.hpp"
+
+namespace lora {
+
+// Copies the Dirichlet halo ring of `in` into `dst` (both padded arrays of the plan's shape).
+cudaError_t launch_copy_halo(const Plan& p, const double* in, double* dst, cudaStream_t s);
+
+// K11: CUDA-core direct (2R+1)^d-point stencil, one time step src -> dst (interior only).
+cudaError_t launch_direct(const Plan& p, const double* src, double* dst, cudaStream_t s);
+
+// K1 (2D): RDG chains U_k X V_k on FP64 tensor cores (DMMA m8n8k4) with BVS, one step.
+cudaError_t launch_tc2d(const Plan& p, const double* src, double* dst, cudaStream_t s);
+
+// K6 (2D): RDG chains as banded passes on the FP64 CUDA-core pipe, one step.
+cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s);
+
+bool tc2d_supported(const Plan& p);
+bool rdg2d_supported(const Plan& p);
+
+}  // namespace lora

@@ -1,0 +1,259 @@
+// K1 — LoRAStencil 2D on FP64 tensor cores (§III-B RDG, §III-C PMA, §III-D BVS).
+//
+// Per warp: an 8-row x 64-column output tile P (eight 8x8 accumulator fragments).  For every
+// rank-1 term u_k v_k^T of the plan (eq. 9: P = sum_k U_k X V_k):
+//   Stage 1 (vertical gather, eq. 10):  T = U_k X.  U_k is the 8 x K1 banded Toeplitz matrix
+//     U[g][k] = u[k - g] (K1 = ceil4(8 + 2h_k)), held as K1/4 A-fragment registers per lane;
+//     X is read from shared memory as B fragments (lane (g,t) reads X[4kk+t][8nb+g]).  T is
+//     8 x 72 (nine 8x8 C fragments) and stays in registers.
+//   Stage 2 (horizontal gather, eq. 11) with Butterfly Vector Swapping (eq. 17): the C
+//     fragment of T block nb is reused AS an A fragment without any shuffle — register R0
+//     holds the even columns 2t, R1 the odd columns 2t+1 — and the rows of V are permuted
+//     the same way: B'[t][n] = V[8j + 2t + i][n] = v[8j + 2t + i - n]  (i = 0 for R0, 1 for R1).
+//     Output block ob needs T blocks ob and ob+1: 4 DMMAs (P:219 counts 4 for the 7x7 case).
+//   Star arms (u or v a unit vector) are a single banded stage; the scalar C_{h+1}
+//   and any single-weight term are a DFMA on the staged tile.
+// On sm_100a every mma.sync.m8n8k4.f64 is one DMMA.8x8x4 (SASS); there is no tcgen05 f64 kind.
+//
+// Tile staging: the (64+2R+4) x 72 input tile (padded coordinates, zero fill outside the
+// array so that 0 * pad never makes NaN) goes to shared memory with a row pitch of 76 doubles
+// (== 12 mod 16), which makes both the B-fragment (4 rows x 8 cols) and the A-fragment
+// (8 rows x 4 cols) LDS.64 patterns bank-conflict free.
+#include <cuda_runtime.h>
+
+#include "kernels.hpp"
+
+namespace lora {
+namespace {
+
+constexpr int TC_MAXT = 16;
+struct TcTerm {
+  int kind, r, ic, jc;     // kind: 0 chain, 1 horizontal arm, 2 vertical arm, 3 point
+  double u[kMaxN], v[kMaxN];
+};
+struct TcParams {
+  int nterms;
+  TcTerm t[TC_MAXT];
+};
+
+constexpr int TC_BM = 64, TC_BN = 64, TC_PITCH = 76;
+
+__device__ __forceinline__ void dmma(double (&c)[2], double a, double b) {
+  asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+               : "+d"(c[0]), "+d"(c[1])
+               : "d"(a), "d"(b));
+}
+
+template <int R>
+__host__ __device__ constexpr int tc_rows() { return TC_BM + 2 * R + 4; }
+
+// u/v are centred length 2R+1; a term of radius HR lives in [R-HR, R+HR].
+template <int R, int HR>
+__device__ __forceinline__ void chain_term(const double* __restrict__ X, int w, int g, int t, const TcTerm& tm,
+                                           double (&P)[8][2]) {
+  constexpr int K1 = ((8 + 2 * HR + 3) / 4) * 4, KS = K1 / 4;
+  constexpr int o = R - HR;
+  double a[KS];
+#pragma unroll
+  for (int kk = 0; kk < KS; ++kk) {
+    const int j = 4 * kk + t - g;
+    a[kk] = (j >= 0 && j <= 2 * HR) ? tm.u[o + j] : 0.0;
+  }
+  double T[9][2];
+#pragma unroll
+  for (int nb = 0; nb < 9; ++nb) { T[nb][0] = 0.0; T[nb][1] = 0.0; }
+  const double* xr = X + (8 * w + o + t) * TC_PITCH + g;
+#pragma unroll
+  for (int kk = 0; kk < KS; ++kk) {
+#pragma unroll
+    for (int nb = 0; nb < 9; ++nb) dmma(T[nb], a[kk], xr[4 * kk * TC_PITCH + 8 * nb]);
+  }
+  double vb[2][2];
+#pragma unroll
+  for (int j = 0; j < 2; ++j)
+#pragma unroll
+    for (int i = 0; i < 2; ++i) {
+      const int c = 8 * j + 2 * t + i - g;
+      vb[j][i] = (c >= 0 && c <= 2 * R) ? tm.v[c] : 0.0;
+    }
+#pragma unroll
+  for (int ob = 0; ob < 8; ++ob) {
+    dmma(P[ob], T[ob][0], vb[0][0]);
+    dmma(P[ob], T[ob][1], vb[0][1]);
+    dmma(P[ob], T[ob + 1][0], vb[1][0]);
+    dmma(P[ob], T[ob + 1][1], vb[1][1]);
+  }
+}
+
+// Horizontal arm (u = e_R): P[g][n] += sum_c X[8w+g+R][8ob+c] v[c-n]; A from smem, B = band of v.
+template <int R, int HR>
+__device__ __forceinline__ void harm_term(const double* __restrict__ X, int w, int g, int t, const TcTerm& tm,
+                                          double (&P)[8][2]) {
+  constexpr int K = ((8 + 2 * HR + 3) / 4) * 4, KS = K / 4;
+  constexpr int o = R - HR;
+  double b[KS];
+#pragma unroll
+  for (int kk = 0; kk < KS; ++kk) {
+    const int j = 4 * kk + t - g;
+    b[kk] = (j >= 0 && j <= 2 * HR) ? tm.v[o + j] : 0.0;
+  }
+  const double* xr = X + (8 * w + g + R) * TC_PITCH + o + t;
+#pragma unroll
+  for (int ob = 0; ob < 8; ++ob)
+#pragma unroll
+    for (int kk = 0; kk < KS; ++kk) dmma(P[ob], xr[8 * ob + 4 * kk], b[kk]);
+}
+
+// Vertical arm (v = e_R): P[g][n] += sum_k U[g][k] X[8w+o+k][8ob+n+R].
+template <int R, int HR>
+__device__ __forceinline__ void varm_term(const double* __restrict__ X, int w, int g, int t, const TcTerm& tm,
+                                          double (&P)[8][2]) {
+  constexpr int K1 = ((8 + 2 * HR + 3) / 4) * 4, KS = K1 / 4;
+  constexpr int o = R - HR;
+  double a[KS];
+#pragma unroll
+  for (int kk = 0; kk < KS; ++kk) {
+    const int j = 4 * kk + t - g;
+    a[kk] = (j >= 0 && j <= 2 * HR) ? tm.u[o + j] : 0.0;
+  }
+  const double* xr = X + (8 * w + o + t) * TC_PITCH + g + R;
+#pragma unroll
+  for (int ob = 0; ob < 8; ++ob)
+#pragma unroll
+    for (int kk = 0; kk < KS; ++kk) dmma(P[ob], a[kk], xr[4 * kk * TC_PITCH + 8 * ob]);
+}
+
+template <int R>
+__device__ __forceinline__ void point_term(const double* __restrict__ X, int w, int g, int t, const TcTerm& tm,
+                                           double (&P)[8][2]) {
+  const double wgt = tm.v[tm.jc];
+  const double* xr = X + (8 * w + g + tm.ic) * TC_PITCH + 2 * t + tm.jc;
+#pragma unroll
+  for (int ob = 0; ob < 8; ++ob) {
+    P[ob][0] = fma(wgt, xr[8 * ob], P[ob][0]);
+    P[ob][1] = fma(wgt, xr[8 * ob + 1], P[ob][1]);
+  }
+}
+
+
+template <int R>
+__global__ void __launch_bounds__(256, 2) tc2d_kernel(const double* __restrict__ in, double* __restrict__ out,
+                                                      int64_t N0, int64_t N1, const __grid_constant__ TcParams prm) {
+  extern __shared__ double X[];
+  constexpr int SH = tc_rows<R>();
+  constexpr int SWL = 72;  // staged columns (T blocks 0..8)
+  const int64_t P1 = N1 + 2 * R, P0 = N0 + 2 * R;
+  const int64_t y0 = int64_t(blockIdx.y) * TC_BM, x0 = int64_t(blockIdx.x) * TC_BN;
+  for (int i = threadIdx.x; i < SH * SWL; i += blockDim.x) {
+    const int r = i / SWL, c = i - r * SWL;
+    const int64_t gy = y0 + r, gx = x0 + c;
+    X[r * TC_PITCH + c] = (gy < P0 && gx < P1) ? __ldg(in + gy * P1 + gx) : 0.0;
+  }
+  __syncthreads();
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int g = lane >> 2, t = lane & 3;
+  double P[8][2];
+#pragma unroll
+  for (int ob = 0; ob < 8; ++ob) { P[ob][0] = 0.0; P[ob][1] = 0.0; }
+  for (int k = 0; k < prm.nterms; ++k) {
+    const TcTerm& tm = prm.t[k];
+    switch (tm.kind) {
+      case 0:
+        if (tm.r == 1) chain_term<R, 1>(X, w, g, t, tm, P);
+        else if constexpr (R >= 2) {
+          if (tm.r == 2) chain_term<R, (R >= 2 ? 2 : 1)>(X, w, g, t, tm, P);
+          else if constexpr (R >= 3) {
+            if (tm.r == 3) chain_term<R, (R >= 3 ? 3 : 1)>(X, w, g, t, tm, P);
+            else if constexpr (R >= 4) chain_term<R, 4>(X, w, g, t, tm, P);
+          }
+        }
+        break;
+      case 1:
+        if (tm.r <= 1) harm_term<R, 1>(X, w, g, t, tm, P);
+        else if constexpr (R >= 2) {
+          if (tm.r == 2) harm_term<R, (R >= 2 ? 2 : 1)>(X, w, g, t, tm, P);
+          else if constexpr (R >= 3) {
+            if (tm.r == 3) harm_term<R, (R >= 3 ? 3 : 1)>(X, w, g, t, tm, P);
+            else if constexpr (R >= 4) harm_term<R, 4>(X, w, g, t, tm, P);
+          }
+        }
+        break;
+      case 2:
+        if (tm.r <= 1) varm_term<R, 1>(X, w, g, t, tm, P);
+        else if constexpr (R >= 2) {
+          if (tm.r == 2) varm_term<R, (R >= 2 ? 2 : 1)>(X, w, g, t, tm, P);
+          else if constexpr (R >= 3) {
+            if (tm.r == 3) varm_term<R, (R >= 3 ? 3 : 1)>(X, w, g, t, tm, P);
+            else if constexpr (R >= 4) varm_term<R, 4>(X, w, g, t, tm, P);
+          }
+        }
+        break;
+      default:
+        point_term<R>(X, w, g, t, tm, P);
+    }
+  }
+  const int64_t gy = y0 + 8 * w + g;
+  if (gy >= N0) return;
+  double* orow = out + (gy + R) * P1 + R;
+#pragma unroll
+  for (int ob = 0; ob < 8; ++ob) {
+    const int64_t gx = x0 + 8 * ob + 2 * t;
+    if (gx < N1) orow[gx] = P[ob][0];
+    if (gx + 1 < N1) orow[gx + 1] = P[ob][1];
+  }
+}
+
+TcParams make_params(const Plan& p) {
+  TcParams prm{};
+  const int R = p.R, n = 2 * R + 1;
+  prm.nterms = 0;
+  for (const Term& t : p.terms) {
+    TcTerm& d = prm.t[prm.nterms++];
+    d.r = t.r < 1 ? 1 : t.r;
+    for (int i = 0; i < n; ++i) { d.u[i] = t.u[i]; d.v[i] = t.v[i]; }
+    d.ic = R; d.jc = R;
+    if (t.kind == kChain) d.kind = 0;
+    else if (t.kind == kArm) {
+      bool u_unit = true;  // u == e_R  -> horizontal arm
+      for (int i = 0; i < n; ++i) if (t.u[i] != (i == R ? 1.0 : 0.0)) u_unit = false;
+      d.kind = u_unit ? 1 : 2;
+    } else {
+      d.kind = 3;
+      for (int i = 0; i < n; ++i) if (t.u[i] != 0.0) d.ic = i;
+      for (int j = 0; j < n; ++j) if (t.v[j] != 0.0) d.jc = j;
+    }
+  }
+  return prm;
+}
+
+template <int R>
+cudaError_t tc_r(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  static bool attr = false;
+  const size_t smem = size_t(tc_rows<R>()) * TC_PITCH * sizeof(double);
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(tc2d_kernel<R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  const TcParams prm = make_params(p);
+  dim3 grid((unsigned)((p.N[1] + TC_BN - 1) / TC_BN), (unsigned)((p.N[0] + TC_BM - 1) / TC_BM));
+  tc2d_kernel<R><<<grid, 256, smem, s>>>(src, dst, p.N[0], p.N[1], prm);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+bool tc2d_supported(const Plan& p) { return p.ndim == 2 && (int)p.terms.size() <= TC_MAXT; }
+
+cudaError_t launch_tc2d(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  if (!tc2d_supported(p)) return cudaErrorInvalidValue;
+  switch (p.R) {
+    case 1: return tc_r<1>(p, src, dst, s);
+    case 2: return tc_r<2>(p, src, dst, s);
+    case 3: return tc_r<3>(p, src, dst, s);
+    case 4: return tc_r<4>(p, src, dst, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+}  // namespace lora

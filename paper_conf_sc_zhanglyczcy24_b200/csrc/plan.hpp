@@ -1,0 +1,55 @@
+// Internal plan representation shared by the planner, the C-ABI layer and the launchers.
+// Not part of the public ABI (include/lora_stencil.h is).
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "lora_stencil.h"
+
+namespace lora {
+
+constexpr int kMaxRadius = 4;
+constexpr int kMaxN = 2 * kMaxRadius + 1;  // 9
+
+enum TermKind { kChain = 0, kArm = 1, kPoint = 2 };
+
+// One rank-1 term u v^T of a 2D plane (eq. 3), stored centred in length 2R+1
+// (R = plan radius).  `r` is the term's own support radius (PMA pyramid level: eq. 15).
+// kPoint terms carry the single weight in v[jc] with u = e_ic (offset (ic-R, jc-R)).
+struct Term {
+  int plane = 0;       // 3D: z-offset index a0 in 0..2R (2D: 0)
+  int kind = kChain;
+  int r = 0;
+  double u[kMaxN] = {0};
+  double v[kMaxN] = {0};
+};
+
+struct Plan {
+  int ndim = 2, R = 1;
+  int64_t N[3] = {1, 1, 1};
+  std::vector<double> W;  // (2R+1)^ndim, row-major copy
+  std::vector<Term> terms;
+  int engine = LORA_ENGINE_AUTO;
+  int fuse_k = 1;
+  int tile_m = 0, tile_n = 0;
+  int z_symmetric = 0;
+  int n_planes_point = 0;
+  double recon_err = 0, growth = 0;
+  double fma_issued = 0, fma_direct = 0, fma_separable = 0;
+  // device state (lazily created at first run)
+  int device = -1;
+  double* scratch = nullptr;      // one padded buffer for the ping-pong
+  double* dev_in = nullptr;       // run_host staging (device copies of host in/out)
+  double* dev_out = nullptr;
+  size_t elems = 0;               // padded element count
+  int64_t P[3] = {1, 1, 1};       // padded extents
+};
+
+// planner.cpp
+int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64_t* grid, const lora_plan_opts* o,
+               std::string& err);
+double tc_fma_per_point(const Plan& p);
+double cuda_fma_per_point(const Plan& p);
+
+}  // namespace lora

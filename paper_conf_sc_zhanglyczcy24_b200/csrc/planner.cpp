@@ -1,0 +1,264 @@
+// Host planner: factor the stencil weights into rank-1 terms and choose the engine.
+//
+// Paper: eq. 8 "W can be decomposed into r matrices each with rank = 1";
+// PMA (§III-C, eq. 15): peel the radially symmetric W ring by ring with the
+// corner pivot, C_i = (R[:,0]/R[0,0]) (x) R[0,:], leaving a (2h-1)^2 radially symmetric
+// remainder, down to the 1x1 scalar C_{h+1} ("no additional MM is required").
+// Where the paper is silent (zero/tiny pivots, star stencils, non-symmetric W) this follows
+// DESIGN.md reading Q6: star arms, rank-revealing stop, complete-pivot elimination.
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "kernels.hpp"
+#include "plan.hpp"
+
+namespace lora {
+namespace {
+
+struct Mat {  // n x n, row-major
+  int n;
+  std::vector<double> a;
+  explicit Mat(int n_) : n(n_), a(size_t(n_) * n_, 0.0) {}
+  double& operator()(int i, int j) { return a[size_t(i) * n + j]; }
+  double operator()(int i, int j) const { return a[size_t(i) * n + j]; }
+};
+
+double maxabs(const Mat& m) {
+  double s = 0;
+  for (double x : m.a) s = std::max(s, std::fabs(x));
+  return s;
+}
+
+int support_radius(const double* x, int n) {  // max |i - c| over nonzeros, c = (n-1)/2
+  int c = (n - 1) / 2, r = 0;
+  for (int i = 0; i < n; ++i)
+    if (x[i] != 0.0) r = std::max(r, std::abs(i - c));
+  return r;
+}
+
+// Factor one (2R+1)^2 plane into terms appended to `out`.
+void factor_plane(const Mat& P, int R, int plane, double tol, std::vector<Term>& out) {
+  const int n = 2 * R + 1;
+  int nnz = 0, zi = 0, zj = 0;
+  bool star = true;
+  for (int i = 0; i < n; ++i)
+    for (int j = 0; j < n; ++j)
+      if (P(i, j) != 0.0) {
+        ++nnz; zi = i; zj = j;
+        if (i != R && j != R) star = false;
+      }
+  if (nnz == 0) return;                       // (0) W == 0: no terms
+  if (nnz == 1) {                             // single weight: point-wise (Alg. 2 lines 3-5)
+    Term t; t.plane = plane; t.kind = kPoint;
+    t.u[zi] = 1.0; t.v[zj] = P(zi, zj);
+    t.r = std::max(std::abs(zi - R), std::abs(zj - R));
+    out.push_back(t);
+    return;
+  }
+  if (star) {                                 // (i) arms: one unit-vector factor each
+    bool has_h = false, has_v = false;
+    for (int j = 0; j < n; ++j) if (j != R && P(R, j) != 0.0) has_h = true;
+    for (int i = 0; i < n; ++i) if (i != R && P(i, R) != 0.0) has_v = true;
+    if (has_h) {  // horizontal arm incl. the centre: u = e_R, v = P[R,:]
+      Term t; t.plane = plane; t.kind = kArm; t.u[R] = 1.0;
+      for (int j = 0; j < n; ++j) t.v[j] = P(R, j);
+      t.r = support_radius(t.v, n);
+      out.push_back(t);
+    }
+    if (has_v) {  // vertical arm: u = P[:,R] (centre only if no horizontal arm), v = e_R
+      Term t; t.plane = plane; t.kind = kArm; t.v[R] = 1.0;
+      for (int i = 0; i < n; ++i) t.u[i] = (i == R && has_h) ? 0.0 : P(i, R);
+      t.r = support_radius(t.u, n);
+      out.push_back(t);
+    }
+    return;
+  }
+  // (ii) PMA ring by ring while the remainder is radially (reflection) symmetric.
+  Mat Rm = P;
+  const double normW1 = [&] { double s = 0; for (double x : P.a) s += std::fabs(x); return s; }();
+  double growth = 0;
+  int k = 0;
+  for (; k <= R; ++k) {
+    if (maxabs(Rm) <= tol) break;             // rank revealed: stop (no 0/0 on separable W)
+    const int m = n - 2 * k;                  // current ring size 2(R-k)+1
+    if (m == 1) {                             // the scalar C_{h+1}
+      Term t; t.plane = plane; t.kind = kPoint; t.r = 0;
+      t.u[R] = 1.0; t.v[R] = Rm(R, R);
+      out.push_back(t);
+      Rm(R, R) = 0.0;
+      break;
+    }
+    bool border_zero = true, sym = true;
+    for (int i = k; i < n - k; ++i)
+      for (int j = k; j < n - k; ++j) {
+        bool on_border = (i == k || i == n - 1 - k || j == k || j == n - 1 - k);
+        if (on_border && std::fabs(Rm(i, j)) > tol) border_zero = false;
+        if (std::fabs(Rm(i, j) - Rm(n - 1 - i, j)) > tol || std::fabs(Rm(i, j) - Rm(i, n - 1 - j)) > tol) sym = false;
+      }
+    if (border_zero) continue;               // ring already empty: skip it
+    const double piv = Rm(k, k);
+    if (!sym || std::fabs(piv) <= tol) break; // hand the remainder to elimination
+    Term t; t.plane = plane; t.kind = kChain; t.r = R - k;
+    for (int i = k; i < n - k; ++i) t.u[i] = Rm(i, k) / piv;   // u = R[:,0] / R[0,0]
+    for (int j = k; j < n - k; ++j) t.v[j] = Rm(k, j);         // v = R[0,:]
+    double g = 0, nu = 0, nv = 0;
+    for (int i = 0; i < n; ++i) { nu += std::fabs(t.u[i]); nv += std::fabs(t.v[i]); }
+    g = nu * nv / normW1;
+    if (growth + g > 1e3) break;               // unbounded growth: use elimination instead
+    growth += g;
+    for (int i = k; i < n - k; ++i)
+      for (int j = k; j < n - k; ++j) Rm(i, j) -= t.u[i] * t.v[j];
+    for (int i = k; i < n - k; ++i) { Rm(i, k) = 0.0; Rm(i, n - 1 - k) = 0.0; Rm(k, i) = 0.0; Rm(n - 1 - k, i) = 0.0; }
+    out.push_back(t);
+  }
+  // (iii) complete-pivot elimination on whatever remains (PMA is its corner-pivot case).
+  for (int it = 0; it < n && maxabs(Rm) > tol; ++it) {
+    int pi = 0, pj = 0;
+    double best = -1;
+    for (int i = 0; i < n; ++i)
+      for (int j = 0; j < n; ++j)
+        if (std::fabs(Rm(i, j)) > best) { best = std::fabs(Rm(i, j)); pi = i; pj = j; }
+    const double piv = Rm(pi, pj);
+    Term t; t.plane = plane;
+    for (int i = 0; i < n; ++i) t.u[i] = Rm(i, pj) / piv;
+    for (int j = 0; j < n; ++j) t.v[j] = Rm(pi, j);
+    t.u[pi] = 1.0;
+    int nzu = 0, nzv = 0;
+    for (int i = 0; i < n; ++i) { nzu += t.u[i] != 0.0; nzv += t.v[i] != 0.0; }
+    for (int i = 0; i < n; ++i)
+      for (int j = 0; j < n; ++j) Rm(i, j) -= t.u[i] * t.v[j];
+    for (int i = 0; i < n; ++i) { Rm(i, pj) = 0.0; Rm(pi, i) = 0.0; }
+    if (nzu == 1 && nzv == 1) { t.kind = kPoint; t.r = std::max(std::abs(pi - R), std::abs(pj - R)); }
+    else if (nzu == 1 && pi == R) { t.kind = kArm; t.r = support_radius(t.v, n); }
+    else if (nzv == 1 && pj == R) { t.kind = kArm; t.r = support_radius(t.u, n); }
+    else { t.kind = kChain; t.r = std::max(support_radius(t.u, n), support_radius(t.v, n)); }
+    out.push_back(t);
+  }
+}
+
+}  // namespace
+
+// Issued FP64 FMAs per output point per step for the tensor-core engine:
+// stage 1 computes 8 x ceil8(BN + 2r) T values with K1 = ceil4(8 + 2r) per element, stage 2
+// 8 x BN outputs with K2 = 16 (BVS fragments of two T blocks); arms are one stage with
+// K = ceil4(8 + 2r) (horizontal arms: per output; vertical arms: per output too);
+// point-wise terms are 1 DFMA.
+double tc_fma_per_point(const Plan& p) {
+  const double BN = 64.0;
+  double f = 0;
+  for (const Term& t : p.terms) {
+    const int r = t.r;
+    const double K = 4.0 * std::ceil((8.0 + 2 * r) / 4.0);
+    if (t.kind == kPoint) f += 1;
+    else if (t.kind == kArm) f += K;
+    else f += K * (8.0 * std::ceil((BN + 2 * r) / 8.0)) / BN + 16.0;
+  }
+  return f;
+}
+
+// Issued FMAs per point for the CUDA-core RDG engine: two banded passes per chain term.
+double cuda_fma_per_point(const Plan& p) {
+  double f = 0;
+  for (const Term& t : p.terms) {
+    if (t.kind == kPoint) f += 1;
+    else if (t.kind == kArm) f += 2 * t.r + 1;
+    else f += 2.0 * (2 * t.r + 1);
+  }
+  return f;
+}
+
+int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64_t* grid, const lora_plan_opts* o,
+               std::string& err) {
+  if (!weights || !grid) { err = "weights and grid_shape must be non-NULL"; return LORA_ERR_INVALID_ARG; }
+  if (ndim != 2 && ndim != 3) { err = "ndim must be 2 or 3"; return LORA_ERR_INVALID_ARG; }
+  if (radius < 1) { err = "radius must be >= 1"; return LORA_ERR_INVALID_ARG; }
+  if (radius > kMaxRadius) { err = "radius > 4 is not supported (DESIGN.md Q14)"; return LORA_ERR_UNSUPPORTED; }
+  for (int i = 0; i < ndim; ++i)
+    if (grid[i] < 1) { err = "grid extents must be >= 1"; return LORA_ERR_INVALID_ARG; }
+  const int n = 2 * radius + 1;
+  const size_t nw = ndim == 2 ? size_t(n) * n : size_t(n) * n * n;
+  for (size_t i = 0; i < nw; ++i)
+    if (!std::isfinite(weights[i])) { err = "weights must be finite"; return LORA_ERR_INVALID_ARG; }
+  p.ndim = ndim; p.R = radius;
+  p.N[0] = p.N[1] = p.N[2] = 1;
+  for (int i = 0; i < ndim; ++i) p.N[i] = grid[i];
+  p.W.assign(weights, weights + nw);
+  p.elems = 1;
+  for (int i = 0; i < 3; ++i) p.P[i] = 1;
+  for (int i = 0; i < ndim; ++i) { p.P[i] = p.N[i] + 2 * radius; p.elems *= size_t(p.P[i]); }
+
+  double wmax = 0, w1 = 0;
+  int nnz = 0;
+  for (size_t i = 0; i < nw; ++i) { wmax = std::max(wmax, std::fabs(weights[i])); w1 += std::fabs(weights[i]); nnz += weights[i] != 0.0; }
+  const double tol = 1e-15 * wmax;
+  p.terms.clear();
+  const int nplanes = ndim == 2 ? 1 : n;
+  p.z_symmetric = 0; p.n_planes_point = 0;
+  for (int q = 0; q < nplanes; ++q) {
+    Mat P(n);
+    for (int i = 0; i < n; ++i)
+      for (int j = 0; j < n; ++j) P(i, j) = weights[size_t(q) * n * n + size_t(i) * n + j];
+    int plane_nnz = 0;
+    for (double x : P.a) plane_nnz += x != 0.0;
+    if (ndim == 3 && plane_nnz == 1) ++p.n_planes_point;
+    factor_plane(P, radius, ndim == 2 ? 0 : q, tol, p.terms);
+  }
+  if (ndim == 3) {
+    bool zs = true;
+    for (int q = 0; q < radius && zs; ++q)
+      for (int e = 0; e < n * n; ++e)
+        if (weights[size_t(q) * n * n + e] != weights[size_t(n - 1 - q) * n * n + e]) { zs = false; break; }
+    p.z_symmetric = zs ? 1 : 0;
+  }
+  // reconstruction check and growth (Q6: reject if > 1e-14)
+  std::vector<double> Wr(nw, 0.0);
+  double g = 0;
+  for (const Term& t : p.terms) {
+    double nu = 0, nv = 0;
+    for (int i = 0; i < n; ++i) { nu += std::fabs(t.u[i]); nv += std::fabs(t.v[i]); }
+    g += nu * nv;
+    for (int i = 0; i < n; ++i)
+      for (int j = 0; j < n; ++j) Wr[size_t(t.plane) * n * n + size_t(i) * n + j] += t.u[i] * t.v[j];
+  }
+  double e = 0;
+  for (size_t i = 0; i < nw; ++i) e = std::max(e, std::fabs(Wr[i] - weights[i]));
+  p.recon_err = wmax > 0 ? e / wmax : 0.0;
+  p.growth = w1 > 0 ? g / w1 : 0.0;
+  if (p.recon_err > 1e-14) { err = "factorisation does not reconstruct W to 1e-14"; return LORA_ERR_FACTOR; }
+
+  p.fma_direct = nnz;
+  p.fma_separable = 0;
+  for (const Term& t : p.terms) {
+    int lu = 0, lv = 0;
+    for (int i = 0; i < n; ++i) { lu += t.u[i] != 0.0; lv += t.v[i] != 0.0; }
+    p.fma_separable += (t.kind == kPoint) ? 1 : (t.kind == kArm ? std::max(lu, lv) : lu + lv);
+  }
+  // engine choice: lowest issued FP64 work at the measured pipe rates (DESIGN.md §Step 0:
+  // DMMA 37 TF, DFMA 34 TF, one shared FP64 budget).
+  int eng = o ? o->engine : LORA_ENGINE_AUTO;
+  if (eng < 0 || eng > LORA_ENGINE_DIRECT) { err = "unknown engine"; return LORA_ERR_INVALID_ARG; }
+  const double c_tc = tc_fma_per_point(p) / 37.0, c_rdg = cuda_fma_per_point(p) / 34.0, c_dir = p.fma_direct / 34.0;
+  const bool ok_tc = tc2d_supported(p), ok_rdg = rdg2d_supported(p);
+  if (eng == LORA_ENGINE_AUTO) {
+    eng = LORA_ENGINE_DIRECT;
+    double best = c_dir;
+    if (ok_tc && c_tc < best) { best = c_tc; eng = LORA_ENGINE_TC; }
+    if (ok_rdg && c_rdg < best) { best = c_rdg; eng = LORA_ENGINE_RDG_CUDA; }
+  } else if ((eng == LORA_ENGINE_TC && !ok_tc) || (eng == LORA_ENGINE_RDG_CUDA && !ok_rdg)) {
+    err = "requested engine does not support this stencil (ndim / term count)";
+    return LORA_ERR_UNSUPPORTED;
+  }
+  p.engine = eng;
+  p.fma_issued = eng == LORA_ENGINE_TC ? tc_fma_per_point(p) : eng == LORA_ENGINE_RDG_CUDA ? cuda_fma_per_point(p) : p.fma_direct;
+  int fk = o ? o->fuse_k : 0;
+  if (fk < 0) { err = "fuse_k must be >= 0"; return LORA_ERR_INVALID_ARG; }
+  p.fuse_k = fk == 0 ? 1 : fk;
+  p.tile_m = eng == LORA_ENGINE_TC ? 64 : (p.ndim == 2 ? 64 : 8);
+  p.tile_n = eng == LORA_ENGINE_TC ? 64 : 32;
+  return LORA_OK;
+}
+
+}  // namespace lora
