@@ -1,0 +1,331 @@
+"""bench.py — GStencil/s (eq. 18) of the LoRAStencil hot path on B200.
+
+A "step" is one call of the C-ABI `lora_stencil_run` over the whole workload: T = 100 Jacobi
+time steps of Box-2D49P on a 10240^2 FP64 grid (BASELINE.json configs[2], the north-star
+target) unless --workload says otherwise.  value = T * prod(N_i) * n_ranks / t (GStencil/s).
+
+    python bench.py [--gpus N --steps K --warmup W] [--workload NAME] [--engine auto|tc|rdg_cuda|direct]
+    python bench.py --impl reference ...   # the CPU oracle (oracle/) on host cores, bounded sample
+
+N > 1 runs under torch.distributed.run, one rank per GPU: weak scaling, every rank owns a slab
+of the same local shape and exchanges halos through lora_stencil_run_dist (NCCL).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "GStencil/s FP64 per stencil at 1/2/4/8 B200; % of HBM roofline"
+UNIT = "GStencil/s"
+BYTES_PER_POINT = 16.0  # algorithmic HBM bytes per point per time step: read 8 + write 8
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="box2d49p-10240")
+    ap.add_argument("--engine", default="auto")
+    ap.add_argument("--fuse", type=int, default=0)
+    ap.add_argument("--per-stencil", action="store_true", help="also time the other single-GPU configs")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ clocks (NVML) during the timed region
+_REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+            0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+            0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+
+class ClockSampler:
+    def __init__(self, index):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _loop(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in _REASONS.items():
+                    if r & bit and bit != 0x1:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.02)
+
+    def __enter__(self):
+        if self.nv:
+            self.t = threading.Thread(target=self._loop, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.nv:
+            self.t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons)}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic(workload, engine):
+    """dram bytes per launch from the committed ncu --set full summary, if one matches."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    d = json.load(open(p))
+    return d.get(f"{workload}/{engine}")
+
+
+def cpu_oracle_sample(W, cfg, budget_s=12.0):
+    """The oracle as it stands, on all host cores, on a bounded sample of the workload: a band of
+    full-width rows (2D) or planes (3D) of the same grid, stepped T_s times (T_s sized to ~budget_s)."""
+    import oracle
+    import synth
+    h = cfg["radius"]
+    shape = list(cfg["shape"])
+    shape[0] = min(shape[0], 256 if cfg["ndim"] == 2 else 16)
+    padded = tuple(n + 2 * h for n in shape)
+    g = synth.grid(padded, cfg["seed"])
+    t0 = time.perf_counter(); oracle.run(W, g, 1); t1 = time.perf_counter() - t0
+    Ts = int(max(1, min(cfg["T"], budget_s / max(t1, 1e-6))))
+    t0 = time.perf_counter(); oracle.run(W, g, Ts); dt = time.perf_counter() - t0
+    pts = float(np.prod(shape)) * Ts
+    return {"value": pts / dt / 1e9, "unit": UNIT, "cores": oracle.max_threads(), "kind": "oracle",
+            "sample": f"{'x'.join(map(str, shape))} interior band of {cfg['name']}, {Ts} steps, {dt:.1f} s"}
+
+
+def host_info():
+    try:
+        model = [l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo") if l.startswith("model name")][0]
+    except Exception:
+        model = "?"
+    return {"nproc": os.cpu_count(), "cpu_model": model}
+
+
+# ------------------------------------------------------------------ reference arm: the CPU oracle
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    import synth
+    W, cfg = synth.config(args.workload)
+    cfg["name"] = args.workload
+    h = cfg["radius"]
+    # size one step so that (W + K) steps take ~150 s in total
+    budget = max(2.0, 150.0 / (args.steps + args.warmup))
+    shape = list(cfg["shape"])
+    shape[0] = min(shape[0], 128 if cfg["ndim"] == 2 else 8)
+    g = synth.grid(tuple(n + 2 * h for n in shape), cfg["seed"])
+    t0 = time.perf_counter(); oracle.run(W, g, 1); t1 = time.perf_counter() - t0
+    Ts = int(max(1, min(cfg["T"], budget / max(t1, 1e-6))))
+    for _ in range(args.warmup):
+        oracle.run(W, g, Ts)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter(); oracle.run(W, g, Ts); times.append(time.perf_counter() - t0)
+    tot = sum(times)
+    pts = float(np.prod(shape)) * Ts
+    value = pts * args.steps / tot / 1e9
+    sample = f"{'x'.join(map(str, shape))} interior band of {args.workload}, {Ts} steps per bench step"
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic (SplitMix64 grid, seeded rsym weights)",
+            "impl": "reference",
+            "config": {"workload": args.workload, "grid": cfg["shape"], "T": cfg["T"], "radius": h},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": oracle.max_threads(), "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "host": host_info()}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ our arm
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sc_zhanglyczcy24_b200 as L
+    import synth
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+
+    W, cfg = synth.config(args.workload)
+    cfg["name"] = args.workload
+    h, T = cfg["radius"], cfg["T"]
+    shape = tuple(cfg["shape"])                      # per-rank local interior (weak scaling)
+    padded = tuple(n + 2 * h for n in shape)
+    st = L.Stencil(W, shape, engine=args.engine, fuse_k=args.fuse)
+    info = st.info()
+    comm = None
+    if world > 1:
+        uid = L.lora_stencil_comm_get_id() if rank == 0 else None
+        obj = [uid]
+        dist.broadcast_object_list(obj, src=0)
+        comm = L.lora_stencil_comm_init(world, rank, obj[0])
+
+    # seeded synthetic input (SplitMix64 over the padded array; each rank its own seed offset)
+    g = synth.grid(padded, cfg["seed"] + 1000 * rank)
+    host_in = torch.from_numpy(g).pin_memory()
+    host_out = torch.empty_like(host_in).pin_memory()
+    x = host_in.to(dev)
+    y = torch.empty_like(x)
+    stream = torch.cuda.current_stream(dev)
+    sptr = stream.cuda_stream
+
+    def step():
+        if comm is None:
+            L.lora_stencil_run(st.plan, x.data_ptr(), y.data_ptr(), T, sptr)
+        else:
+            L.lora_stencil_run_dist(st.plan, comm, x.data_ptr(), y.data_ptr(), T, sptr)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        e0.record(stream)
+        for _ in range(args.steps):
+            step()
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    t = e0.elapsed_time(e1) / 1e3
+    if world > 1:
+        tt = torch.tensor([t], device=dev, dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t = float(tt.item())
+    pts_per_step = float(np.prod(shape)) * T * world
+    value = pts_per_step * args.steps / t / 1e9
+    fuse = info["fuse_k"]
+    launches_per_step = -(-T // fuse) + 2      # stencil launches + 2 halo-copy launches
+
+    # roofline for the dominant kernel (the stencil kernel): algorithmic bytes per launch / avg launch time
+    peak, peak_src = load_peaks()
+    per_launch_bytes = BYTES_PER_POINT * float(np.prod(shape))      # per launch: one (fused) superstep
+    avg_launch_s = t / args.steps / (-(-T // fuse))
+    achieved = per_launch_bytes / avg_launch_s / 1e9
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+            "traffic": ncu_traffic(args.workload, info["engine_name"]), "peak_source": peak_src,
+            "kernel": f"{info['engine_name']} stencil step", "algorithmic_bytes_per_launch": per_launch_bytes,
+            "avg_launch_ms": avg_launch_s * 1e3,
+            "gstencil_roofline": peak / BYTES_PER_POINT * world}
+
+    # e2e: through the C-ABI with HOST buffers (H2D of the input + D2H of the result inside the region)
+    e2e = None
+    if not args.no_e2e and comm is None:
+        L.lora_stencil_run_host(st.plan, host_in.numpy(), host_out.numpy(), T, sptr)
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            L.lora_stencil_run_host(st.plan, host_in.numpy(), host_out.numpy(), T, sptr)
+        te = time.perf_counter() - t0
+        nbytes = host_in.numel() * 8
+        e2e = {"value": pts_per_step * args.steps / te / 1e9, "unit": UNIT, "h2d_bytes_per_step": nbytes,
+               "d2h_bytes_per_step": nbytes, "api": "lora_stencil_run_host (pinned host buffers)"}
+
+    per_stencil = None
+    if args.per_stencil and rank == 0 and world == 1:
+        per_stencil = {}
+        for name in ("heat2d-256", "box2d9p-10240", "box2d49p-10240", "heat3d-512", "box3d27p-512"):
+            Wn, cn = synth.config(name)
+            s2 = L.Stencil(Wn, cn["shape"], engine=args.engine)
+            xa = torch.rand(cn["padded"], dtype=torch.float64, device=dev) + 0.5
+            ya = torch.empty_like(xa)
+            L.lora_stencil_run(s2.plan, xa.data_ptr(), ya.data_ptr(), cn["T"], sptr)
+            torch.cuda.synchronize(dev)
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            for _ in range(3):
+                L.lora_stencil_run(s2.plan, xa.data_ptr(), ya.data_ptr(), cn["T"], sptr)
+            a1.record(stream)
+            torch.cuda.synchronize(dev)
+            ts = a0.elapsed_time(a1) / 3e3
+            gs = float(np.prod(cn["shape"])) * cn["T"] / ts / 1e9
+            per_stencil[name] = {"GStencil_s": gs, "frac_hbm_roofline": gs / (peak / BYTES_PER_POINT),
+                                 "engine": s2.info()["engine_name"], "ms": ts * 1e3}
+            s2.close()
+            del xa, ya
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_oracle_sample(W, cfg)
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": 1e3 * t / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic: SplitMix64 grid in [0.5,1.5) over the padded array, seeded radially symmetric weights",
+                "config": {"workload": args.workload, "grid_per_rank": list(shape), "T": T, "radius": h,
+                           "ndim": cfg["ndim"], "global_grid": [shape[0] * world] + list(shape[1:]),
+                           "engine": info["engine_name"], "fuse_k": fuse, "n_terms": info["n_terms"],
+                           "parallelism": f"slab{world}" if world > 1 else "single",
+                           "l2": "inputs (%.2f GB per buffer) larger than the 126 MB L2" % (8 * np.prod(padded) / 1e9)},
+                "clocks": clk.summary(), "gpu_launches": launches_per_step * args.steps,
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+                "fma_per_point": {"issued": info["fma_per_point_issued"], "direct": info["fma_per_point_direct"],
+                                  "separable": info["fma_per_point_separable"]},
+                "host": host_info()}
+        if per_stencil:
+            line["per_stencil"] = per_stencil
+        print(json.dumps(line), flush=True)
+    if comm is not None:
+        L.lora_stencil_comm_destroy(comm)
+    st.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

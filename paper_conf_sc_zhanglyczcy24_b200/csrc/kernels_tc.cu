@@ -21,7 +21,11 @@
 // (8 rows x 4 cols) LDS.64 patterns bank-conflict free.
 #include <cuda_runtime.h>
 
+#include <algorithm>
+#include <cstring>
+
 #include "kernels.hpp"
+#include "pipe.cuh"
 
 namespace lora {
 namespace {
@@ -137,22 +141,8 @@ __device__ __forceinline__ void point_term(const double* __restrict__ X, int w, 
 
 
 template <int R>
-__global__ void __launch_bounds__(256, 2) tc2d_kernel(const double* __restrict__ in, double* __restrict__ out,
-                                                      int64_t N0, int64_t N1, const __grid_constant__ TcParams prm) {
-  extern __shared__ double X[];
-  constexpr int SH = tc_rows<R>();
-  constexpr int SWL = 72;  // staged columns (T blocks 0..8)
-  const int64_t P1 = N1 + 2 * R, P0 = N0 + 2 * R;
-  const int64_t y0 = int64_t(blockIdx.y) * TC_BM, x0 = int64_t(blockIdx.x) * TC_BN;
-  for (int i = threadIdx.x; i < SH * SWL; i += blockDim.x) {
-    const int r = i / SWL, c = i - r * SWL;
-    const int64_t gy = y0 + r, gx = x0 + c;
-    X[r * TC_PITCH + c] = (gy < P0 && gx < P1) ? __ldg(in + gy * P1 + gx) : 0.0;
-  }
-  __syncthreads();
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int g = lane >> 2, t = lane & 3;
-  double P[8][2];
+__device__ __forceinline__ void tc_tile(const double* __restrict__ X, int w, int g, int t, const TcParams& prm,
+                                        double (&P)[8][2]) {
 #pragma unroll
   for (int ob = 0; ob < 8; ++ob) { P[ob][0] = 0.0; P[ob][1] = 0.0; }
   for (int k = 0; k < prm.nterms; ++k) {
@@ -192,14 +182,72 @@ __global__ void __launch_bounds__(256, 2) tc2d_kernel(const double* __restrict__
         point_term<R>(X, w, g, t, tm, P);
     }
   }
-  const int64_t gy = y0 + 8 * w + g;
-  if (gy >= N0) return;
-  double* orow = out + (gy + R) * P1 + R;
+}
+
+// Persistent CTAs walk the 64x64 output tiles; tile i+1 is staged (TMA + mbarrier, or LDGSTS when
+// TMA's 16-byte pitch rule fails) while tile i is computed.
+template <int R, bool TMA>
+__global__ void __launch_bounds__(256, 2) tc2d_kernel(const double* __restrict__ in, double* __restrict__ out,
+                                                      int64_t N0, int64_t N1, int ntx, int ntiles,
+                                                      const __grid_constant__ CUtensorMap tmap,
+                                                      const __grid_constant__ TcParams prm) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  constexpr int SH = tc_rows<R>();
+  constexpr int BUF = ((SH * TC_PITCH * 8 + 127) / 128) * 128 / 8;  // doubles per buffer
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw);
+  double* buf0 = reinterpret_cast<double*>(smem_raw + 128);
+  const int64_t P1 = N1 + 2 * R, P0 = N0 + 2 * R;
+  const int tid = threadIdx.x;
+  if (TMA && tid == 0) {
+    prefetch_tmap(&tmap);
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    fence_barrier_init();
+  }
+  __syncthreads();
+  auto issue = [&](int tile, int b) {
+    const int64_t y0 = int64_t(tile / ntx) * TC_BM, x0 = int64_t(tile % ntx) * TC_BN;
+    double* dst = buf0 + b * BUF;
+    if constexpr (TMA) {
+      if (tid == 0) {
+        mbar_arrive_expect_tx(&bar[b], SH * TC_PITCH * 8);
+        tma_load_2d(dst, &tmap, (int)x0, (int)y0, &bar[b]);
+      }
+    } else {
+      box_fill_cpasync(dst, in, P0, P1, y0, x0, SH, TC_PITCH);
+      cp_async_commit();
+    }
+  };
+  const int lane = tid & 31, w = tid >> 5;
+  const int g = lane >> 2, t = lane & 3;
+  int it = 0;
+  int tile = blockIdx.x;
+  if (tile < ntiles) issue(tile, 0);
+  for (; tile < ntiles; tile += gridDim.x, ++it) {
+    const int b = it & 1;
+    const int next = tile + gridDim.x;
+    if (next < ntiles) issue(next, b ^ 1);
+    if constexpr (TMA) {
+      mbar_wait(&bar[b], (it >> 1) & 1);
+    } else {
+      if (next < ntiles) cp_async_wait<1>(); else cp_async_wait<0>();
+      __syncthreads();
+    }
+    const double* X = buf0 + b * BUF;
+    double P[8][2];
+    tc_tile<R>(X, w, g, t, prm, P);
+    const int64_t y0 = int64_t(tile / ntx) * TC_BM, x0 = int64_t(tile % ntx) * TC_BN;
+    const int64_t gy = y0 + 8 * w + g;
+    if (gy < N0) {
+      double* orow = out + (gy + R) * P1 + R;
 #pragma unroll
-  for (int ob = 0; ob < 8; ++ob) {
-    const int64_t gx = x0 + 8 * ob + 2 * t;
-    if (gx < N1) orow[gx] = P[ob][0];
-    if (gx + 1 < N1) orow[gx + 1] = P[ob][1];
+      for (int ob = 0; ob < 8; ++ob) {
+        const int64_t gx = x0 + 8 * ob + 2 * t;
+        if (gx < N1) orow[gx] = P[ob][0];
+        if (gx + 1 < N1) orow[gx + 1] = P[ob][1];
+      }
+    }
+    __syncthreads();  // buffer b is free for the issue of iteration it+1
   }
 }
 
@@ -226,19 +274,33 @@ TcParams make_params(const Plan& p) {
   return prm;
 }
 
+template <int R, bool TMA>
+cudaError_t tc_launch(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map) {
+  constexpr int SH = tc_rows<R>();
+  constexpr size_t BUF = ((SH * TC_PITCH * 8 + 127) / 128) * 128;
+  const size_t smem = 128 + 2 * BUF;
+  const int ntx = (int)((p.N[1] + TC_BN - 1) / TC_BN), nty = (int)((p.N[0] + TC_BM - 1) / TC_BM);
+  const int64_t ntiles = int64_t(ntx) * nty;
+  static int max_grid = 0;
+  if (max_grid == 0) {
+    cudaError_t e = cudaFuncSetAttribute(tc2d_kernel<R, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    max_grid = persistent_grid((const void*)tc2d_kernel<R, TMA>, 256, smem, int64_t(1) << 40);
+  }
+  const int grid = (int)std::min<int64_t>(max_grid, ntiles);
+  const TcParams prm = make_params(p);
+  tc2d_kernel<R, TMA><<<grid, 256, smem, s>>>(src, dst, p.N[0], p.N[1], ntx, (int)ntiles, map, prm);
+  return cudaGetLastError();
+}
+
 template <int R>
 cudaError_t tc_r(const Plan& p, const double* src, double* dst, cudaStream_t s) {
-  static bool attr = false;
-  const size_t smem = size_t(tc_rows<R>()) * TC_PITCH * sizeof(double);
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(tc2d_kernel<R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    attr = true;
-  }
-  const TcParams prm = make_params(p);
-  dim3 grid((unsigned)((p.N[1] + TC_BN - 1) / TC_BN), (unsigned)((p.N[0] + TC_BM - 1) / TC_BM));
-  tc2d_kernel<R><<<grid, 256, smem, s>>>(src, dst, p.N[0], p.N[1], prm);
-  return cudaGetLastError();
+  CUtensorMap map;
+  const int64_t padded[2] = {p.P[0], p.P[1]};
+  const int box[2] = {tc_rows<R>(), TC_PITCH};
+  if (!p.force_no_tma && encode_tmap(&map, src, 2, padded, box)) return tc_launch<R, true>(p, src, dst, s, map);
+  std::memset(&map, 0, sizeof(map));
+  return tc_launch<R, false>(p, src, dst, s, map);
 }
 
 }  // namespace

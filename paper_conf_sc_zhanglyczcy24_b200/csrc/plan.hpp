@@ -34,6 +34,7 @@ struct Plan {
   int fuse_k = 1;
   int tile_m = 0, tile_n = 0;
   int z_symmetric = 0;
+  int force_no_tma = 0;   // LORA_NO_TMA=1: use the LDGSTS staging path (tests both loaders)
   int n_planes_point = 0;
   double recon_err = 0, growth = 0;
   double fma_issued = 0, fma_direct = 0, fma_separable = 0;

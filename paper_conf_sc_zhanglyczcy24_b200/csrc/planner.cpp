@@ -8,6 +8,7 @@
 // DESIGN.md reading Q6: star arms, rank-revealing stop, complete-pivot elimination.
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -256,6 +257,10 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
   int fk = o ? o->fuse_k : 0;
   if (fk < 0) { err = "fuse_k must be >= 0"; return LORA_ERR_INVALID_ARG; }
   p.fuse_k = fk == 0 ? 1 : fk;
+  {
+    const char* e = std::getenv("LORA_NO_TMA");
+    p.force_no_tma = (e && e[0] == '1') ? 1 : 0;
+  }
   p.tile_m = eng == LORA_ENGINE_TC ? 64 : (p.ndim == 2 ? 64 : 8);
   p.tile_n = eng == LORA_ENGINE_TC ? 64 : 32;
   return LORA_OK;
