@@ -11,7 +11,7 @@ from tests._gpu_helpers import rel_err, run_gpu
 
 pytestmark = pytest.mark.gpu
 
-ENGINES_2D = ["direct", "tc"]
+ENGINES_2D = ["direct", "tc", "rdg_cuda"]
 
 
 def _weights(kind, d, h, seed):
