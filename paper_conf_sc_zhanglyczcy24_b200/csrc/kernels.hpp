@@ -19,7 +19,11 @@ cudaError_t launch_tc2d(const Plan& p, const double* src, double* dst, cudaStrea
 // K6 (2D): RDG chains as banded passes on the FP64 CUDA-core pipe, one step.
 cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s);
 
+// K2 on CUDA cores (3D, Alg. 2 with RDG per plane), one step.
+cudaError_t launch_rdg3d(const Plan& p, const double* src, double* dst, cudaStream_t s);
+
 bool tc2d_supported(const Plan& p);
+bool rdg3d_supported(const Plan& p);
 bool rdg2d_supported(const Plan& p);
 
 }  // namespace lora

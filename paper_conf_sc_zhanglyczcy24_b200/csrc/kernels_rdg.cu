@@ -296,12 +296,14 @@ cudaError_t rdg_r(const Plan& p, const double* src, double* dst, cudaStream_t s)
 }  // namespace
 
 bool rdg2d_supported(const Plan& p) {
+  if (p.ndim == 3) return rdg3d_supported(p);
   if (p.ndim != 2) return false;
   RdgParams prm;
   return signature(p, prm) >= 0;
 }
 
 cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  if (p.ndim == 3) return launch_rdg3d(p, src, dst, s);
   switch (p.R) {
     case 1: return rdg_r<1>(p, src, dst, s);
     case 2: return rdg_r<2>(p, src, dst, s);

@@ -1,0 +1,341 @@
+// K2/K3 on CUDA cores — LoRAStencil-3D (§IV-C Alg. 2) with RDG per plane.
+//
+// Alg. 2: the (2R+1)^3 stencil is the sum over its 2R+1 z-planes W_{a0} of 2D stencils applied
+// to the input planes; a plane holding a single weight is a point-wise multiply-add on CUDA cores
+// (lines 3-5), any other plane is a 2D LoRAStencil (lines 7-8) — here its rank-1 terms u v^T
+// (planner, eq. 8/15) evaluated as the two banded gathers of RDG (horizontal v-pass, vertical
+// u-pass), or the two arms of a star plane.  Result for output plane z: sum_{a0} W_{a0} * X_{z+a0}.
+//
+// B200 mapping: one warp streams a 64-column x BY-row column of the domain along z through a
+// chunk of ZC output planes.  Input planes arrive by TMA (3D box 1 x (BY+2R) x (64+2R), zero
+// fill) into a per-warp ring; each input plane p is read from shared memory ONCE and contributes
+// to the 2R+1 output planes z = p - a0 held in a register ring.  When W_{a0} == W_{2R-a0}
+// (z-symmetric, e.g. Box-3D27P and Heat-3D) the plane result is computed once and added to both
+// output planes.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <utility>
+#include <vector>
+
+#include "kernels.hpp"
+#include "pipe.cuh"
+
+namespace lora {
+namespace {
+
+constexpr int R3_WARPS = 4;
+constexpr int R3_NS = 4;
+template <int R> constexpr int BY = (R == 1 ? 4 : 2);
+constexpr int R3_ZC = 64;
+constexpr int R3_MAXK = 5;   // rank-1 terms per plane (<= 2R+1 for R <= 2)
+
+enum { PM_NONE = 0, PM_POINT = 1, PM_CHAINS = 2, PM_STAR = 3 };
+
+struct R3Params {
+  int mode[5];               // per plane a0
+  int K[5];                  // chain terms per plane
+  int mirror[5];             // plane a0 (< R) also feeds output z = p - (2R - a0)
+  double w[5];               // PM_POINT weight (centre)
+  double u[5][R3_MAXK][5];   // plane, term, tap (centred, length 2R+1)
+  double v[5][R3_MAXK][5];
+};
+
+template <int R>
+struct G3 {
+  static constexpr int n = 2 * R + 1;
+  static constexpr int ROWS = BY<R> + 2 * R;
+  static constexpr int BW = 64 + 2 * R;
+  static constexpr int STAGE = ((ROWS * BW * 8 + 127) / 128) * 128;
+  static constexpr int SI = ((R3_ZC + 2 * R + n - 1) / n) * n;   // planes streamed per item (multiple of n)
+  static constexpr int WARP_BYTES = R3_NS * STAGE;
+  static constexpr int SMEM = 128 + R3_WARPS * WARP_BYTES;
+};
+
+__host__ __device__ constexpr int pm(int a, int n) { return ((a % n) + n) % n; }
+
+// Applies plane operator a0 to the staged plane (registers x) and adds into the ring slot(s).
+template <int R, int A0, int I>
+__device__ __forceinline__ void apply_plane(const double (&x)[BY<R> + 2 * R][2 * R + 2],
+                                            double (&acc)[2 * R + 1][BY<R>][2], const R3Params& P) {
+  constexpr int n = 2 * R + 1;
+  constexpr int s1 = pm(I - A0, n);           // output plane z = p - a0
+  constexpr int s2 = pm(I - (n - 1 - A0), n); // mirrored plane
+  const int mode = P.mode[A0];
+  if (mode == PM_NONE) return;
+  double d[BY<R>][2];
+  if (mode == PM_POINT) {
+#pragma unroll
+    for (int y = 0; y < BY<R>; ++y) {
+      d[y][0] = P.w[A0] * x[y + R][R];
+      d[y][1] = P.w[A0] * x[y + R][R + 1];
+    }
+  } else if (mode == PM_STAR) {
+    // horizontal arm v (u = e_R) on the centre row, vertical arm u (v = e_R) on the centre column
+#pragma unroll
+    for (int y = 0; y < BY<R>; ++y) {
+      double t0 = 0.0, t1 = 0.0;
+#pragma unroll
+      for (int b = -R; b <= R; ++b) {
+        t0 = fma(P.v[A0][0][R + b], x[y + R][R + b], t0);
+        t1 = fma(P.v[A0][0][R + b], x[y + R][R + b + 1], t1);
+      }
+#pragma unroll
+      for (int a = -R; a <= R; ++a) {
+        t0 = fma(P.u[A0][1][R + a], x[y + R + a][R], t0);
+        t1 = fma(P.u[A0][1][R + a], x[y + R + a][R + 1], t1);
+      }
+      d[y][0] = t0;
+      d[y][1] = t1;
+    }
+  } else {
+#pragma unroll
+    for (int y = 0; y < BY<R>; ++y) { d[y][0] = 0.0; d[y][1] = 0.0; }
+#pragma unroll
+    for (int k = 0; k < R3_MAXK; ++k) {
+      if (k < P.K[A0]) {
+        double T[BY<R> + 2 * R][2];
+#pragma unroll
+        for (int r = 0; r < BY<R> + 2 * R; ++r) {      // horizontal gather (v-pass)
+          double t0 = 0.0, t1 = 0.0;
+#pragma unroll
+          for (int b = -R; b <= R; ++b) {
+            t0 = fma(P.v[A0][k][R + b], x[r][R + b], t0);
+            t1 = fma(P.v[A0][k][R + b], x[r][R + b + 1], t1);
+          }
+          T[r][0] = t0;
+          T[r][1] = t1;
+        }
+#pragma unroll
+        for (int y = 0; y < BY<R>; ++y)                 // vertical gather (u-pass)
+#pragma unroll
+          for (int a = -R; a <= R; ++a) {
+            d[y][0] = fma(P.u[A0][k][R + a], T[y + R + a][0], d[y][0]);
+            d[y][1] = fma(P.u[A0][k][R + a], T[y + R + a][1], d[y][1]);
+          }
+      }
+    }
+  }
+#pragma unroll
+  for (int y = 0; y < BY<R>; ++y) {
+    acc[s1][y][0] += d[y][0];
+    acc[s1][y][1] += d[y][1];
+  }
+  if (A0 < R && P.mirror[A0]) {
+#pragma unroll
+    for (int y = 0; y < BY<R>; ++y) {
+      acc[s2][y][0] += d[y][0];
+      acc[s2][y][1] += d[y][1];
+    }
+  }
+}
+
+template <int R, int A0, int I>
+__device__ __forceinline__ void apply_all(const double (&x)[BY<R> + 2 * R][2 * R + 2],
+                                          double (&acc)[2 * R + 1][BY<R>][2], const R3Params& P) {
+  if constexpr (A0 < 2 * R + 1) {
+    if (!(A0 > R && P.mirror[2 * R - A0])) apply_plane<R, A0, I>(x, acc, P);
+    apply_all<R, A0 + 1, I>(x, acc, P);
+  }
+}
+
+template <int R, bool TMA>
+__global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* __restrict__ in, double* __restrict__ out,
+                                                                 int64_t N0, int64_t N1, int64_t N2, int nbx, int nby,
+                                                                 int nitems, const __grid_constant__ CUtensorMap tmap,
+                                                                 const __grid_constant__ R3Params prm) {
+  using G = G3<R>;
+  constexpr int n = 2 * R + 1;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw) + wl * R3_NS;
+  unsigned char* ring = smem_raw + 128 + wl * G::WARP_BYTES;
+  const int64_t P0 = N0 + 2 * R, P1 = N1 + 2 * R, P2 = N2 + 2 * R;
+  const int gw = blockIdx.x * R3_WARPS + wl, TW = gridDim.x * R3_WARPS;
+  const int my_items = gw < nitems ? (nitems - 1 - gw) / TW + 1 : 0;
+  const int nstages = my_items * G::SI;
+  if (TMA && lane == 0) {
+    for (int s = 0; s < R3_NS; ++s) mbar_init(&bars[s], 1);
+    fence_barrier_init();
+  }
+  __syncwarp();
+  auto coords = [&](int q, int64_t& z, int64_t& y, int64_t& x) {
+    const int item = gw + (q / G::SI) * TW, j = q % G::SI;
+    const int bx = item % nbx, rest = item / nbx, by = rest % nby, bz = rest / nby;
+    z = int64_t(bz) * R3_ZC + j;         // padded input plane
+    y = int64_t(by) * BY<R>;             // padded row of the tile origin
+    x = int64_t(bx) * 64;
+  };
+  auto issue = [&](int q) {
+    int64_t z, y, x;
+    coords(q, z, y, x);
+    double* dst = reinterpret_cast<double*>(ring + (q % R3_NS) * G::STAGE);
+    if constexpr (TMA) {
+      if (lane == 0) {
+        mbar_arrive_expect_tx(&bars[q % R3_NS], G::ROWS * G::BW * 8);
+        tma_load_3d(dst, &tmap, (int)x, (int)y, (int)z, &bars[q % R3_NS]);
+      }
+    } else {
+      for (int i = lane; i < G::ROWS * G::BW; i += 32) {
+        const int r = i / G::BW, c = i - r * G::BW;
+        const int64_t gy = y + r, gx = x + c;
+        if (z < P0 && gy < P1 && gx < P2) cp_async8(dst + i, in + (z * P1 + gy) * P2 + gx);
+        else dst[i] = 0.0;
+      }
+      cp_async_commit();
+    }
+  };
+  for (int q = 0; q < R3_NS - 1; ++q) {
+    if (q < nstages) issue(q);
+    else if constexpr (!TMA) cp_async_commit();
+  }
+  double acc[n][BY<R>][2];
+  // consumer: stages in groups of n so that the ring slot of every plane offset is static
+  for (int q0 = 0; q0 < nstages; q0 += n) {
+    auto one = [&](auto Ic) {
+      constexpr int I = decltype(Ic)::value;
+      const int q = q0 + I;
+      if (q + R3_NS - 1 < nstages) issue(q + R3_NS - 1);
+      else if constexpr (!TMA) cp_async_commit();
+      if constexpr (TMA) {
+        mbar_wait(&bars[q % R3_NS], (q / R3_NS) & 1);
+      } else {
+        cp_async_wait<R3_NS - 1>();
+        __syncwarp();
+      }
+      int64_t zp, y0, x0;
+      coords(q, zp, y0, x0);
+      const int j = q % G::SI;
+      if (j == 0) {
+#pragma unroll
+        for (int s = 0; s < n; ++s)
+#pragma unroll
+          for (int y = 0; y < BY<R>; ++y) { acc[s][y][0] = 0.0; acc[s][y][1] = 0.0; }
+      }
+      const double* st = reinterpret_cast<const double*>(ring + (q % R3_NS) * G::STAGE);
+      double x[BY<R> + 2 * R][2 * R + 2];
+#pragma unroll
+      for (int r = 0; r < BY<R> + 2 * R; ++r)
+#pragma unroll
+        for (int m = 0; m <= R; ++m) {
+          const double2 t = *reinterpret_cast<const double2*>(st + r * G::BW + 2 * lane + 2 * m);
+          x[r][2 * m] = t.x;
+          x[r][2 * m + 1] = t.y;
+        }
+      __syncwarp();  // slot consumed
+      apply_all<R, 0, I>(x, acc, prm);
+      // output plane zi = zp - 2R (interior index) is complete: slot (I - 2R) mod n == (I + 1) mod n
+      constexpr int s = (I + 1) % n;
+      const int64_t zi = zp - 2 * R;
+      const int64_t zc0 = zp - j;  // first interior output plane of the chunk
+      if (zi >= zc0 && zi < zc0 + R3_ZC && zi < N0) {
+        const int64_t col = x0 + 2 * lane;
+#pragma unroll
+        for (int y = 0; y < BY<R>; ++y) {
+          const int64_t gy = y0 + y;
+          if (gy < N1) {
+            double* o = out + ((zi + R) * P1 + gy + R) * P2 + R + col;
+            if (col < N2) o[0] = acc[s][y][0];
+            if (col + 1 < N2) o[1] = acc[s][y][1];
+          }
+        }
+      }
+#pragma unroll
+      for (int y = 0; y < BY<R>; ++y) { acc[s][y][0] = 0.0; acc[s][y][1] = 0.0; }
+    };
+    [&]<int... Is>(std::integer_sequence<int, Is...>) {
+      (one(std::integral_constant<int, Is>{}), ...);
+    }(std::make_integer_sequence<int, n>{});
+  }
+}
+
+bool make_params3(const Plan& p, R3Params& prm) {
+  std::memset(&prm, 0, sizeof(prm));
+  const int R = p.R, n = 2 * R + 1;
+  if (p.ndim != 3 || R > 2) return false;
+  for (int a0 = 0; a0 < n; ++a0) {
+    std::vector<const Term*> ts;
+    for (const Term& t : p.terms)
+      if (t.plane == a0) ts.push_back(&t);
+    if (ts.empty()) { prm.mode[a0] = PM_NONE; continue; }
+    if (ts.size() == 1 && ts[0]->kind == kPoint && ts[0]->u[R] == 1.0 && ts[0]->v[R] != 0.0) {
+      bool centre = true;
+      for (int i = 0; i < n; ++i)
+        if (i != R && (ts[0]->u[i] != 0.0 || ts[0]->v[i] != 0.0)) centre = false;
+      if (centre) { prm.mode[a0] = PM_POINT; prm.w[a0] = ts[0]->v[R]; continue; }
+    }
+    if (ts.size() == 2 && ts[0]->kind == kArm && ts[1]->kind == kArm && ts[0]->u[R] == 1.0 && ts[1]->v[R] == 1.0) {
+      bool ok = true;
+      for (int i = 0; i < n; ++i)
+        if (i != R && (ts[0]->u[i] != 0.0 || ts[1]->v[i] != 0.0)) ok = false;
+      if (ok) {
+        prm.mode[a0] = PM_STAR;
+        for (int i = 0; i < n; ++i) { prm.v[a0][0][i] = ts[0]->v[i]; prm.u[a0][1][i] = ts[1]->u[i]; }
+        continue;
+      }
+    }
+    if ((int)ts.size() > R3_MAXK) return false;
+    prm.mode[a0] = PM_CHAINS;
+    prm.K[a0] = (int)ts.size();
+    for (size_t k = 0; k < ts.size(); ++k)
+      for (int i = 0; i < n; ++i) { prm.u[a0][k][i] = ts[k]->u[i]; prm.v[a0][k][i] = ts[k]->v[i]; }
+  }
+  // z-symmetry per plane pair: identical weights => mirror
+  for (int a0 = 0; a0 < R; ++a0) {
+    bool same = true;
+    for (int e = 0; e < n * n; ++e)
+      if (p.W[size_t(a0) * n * n + e] != p.W[size_t(n - 1 - a0) * n * n + e]) { same = false; break; }
+    prm.mirror[a0] = same ? 1 : 0;
+  }
+  return true;
+}
+
+template <int R, bool TMA>
+cudaError_t rdg3d_launch(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
+                         const R3Params& prm) {
+  using G = G3<R>;
+  static int max_grid = 0;
+  if (max_grid == 0) {
+    cudaError_t e = cudaFuncSetAttribute(rdg3d_kernel<R, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, G::SMEM);
+    if (e != cudaSuccess) return e;
+    max_grid = persistent_grid((const void*)rdg3d_kernel<R, TMA>, R3_WARPS * 32, G::SMEM, int64_t(1) << 40);
+  }
+  const int nbx = (int)((p.N[2] + 63) / 64), nby = (int)((p.N[1] + BY<R> - 1) / BY<R>);
+  const int nbz = (int)((p.N[0] + R3_ZC - 1) / R3_ZC);
+  const int64_t nitems = int64_t(nbx) * nby * nbz;
+  const int grid = (int)std::min<int64_t>(max_grid, (nitems + R3_WARPS - 1) / R3_WARPS);
+  rdg3d_kernel<R, TMA><<<grid, R3_WARPS * 32, G::SMEM, s>>>(src, dst, p.N[0], p.N[1], p.N[2], nbx, nby, (int)nitems,
+                                                           map, prm);
+  return cudaGetLastError();
+}
+
+template <int R>
+cudaError_t rdg3d_r(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  using G = G3<R>;
+  R3Params prm;
+  if (!make_params3(p, prm)) return cudaErrorNotSupported;
+  CUtensorMap map;
+  const int64_t padded[3] = {p.P[0], p.P[1], p.P[2]};
+  const int box[3] = {1, G::ROWS, G::BW};
+  if (!p.force_no_tma && encode_tmap(&map, src, 3, padded, box)) return rdg3d_launch<R, true>(p, src, dst, s, map, prm);
+  std::memset(&map, 0, sizeof(map));
+  return rdg3d_launch<R, false>(p, src, dst, s, map, prm);
+}
+
+}  // namespace
+
+bool rdg3d_supported(const Plan& p) {
+  R3Params prm;
+  return make_params3(p, prm);
+}
+
+cudaError_t launch_rdg3d(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  switch (p.R) {
+    case 1: return rdg3d_r<1>(p, src, dst, s);
+    case 2: return rdg3d_r<2>(p, src, dst, s);
+  }
+  return cudaErrorNotSupported;
+}
+
+}  // namespace lora

@@ -160,13 +160,43 @@ double tc_fma_per_point(const Plan& p) {
   return f;
 }
 
-// Issued FMAs per point for the CUDA-core RDG engine: two banded passes per chain term.
+// Issued FMAs per point for the CUDA-core RDG engine (kernels_rdg.cu / kernels_rdg3d.cu): the
+// PMA and star signatures issue each term at its own radius; the general signature issues every
+// term at the full radius R.  3D: per plane (Alg. 2), a mirrored plane pair (W_a == W_{2R-a})
+// is computed once and added twice.
 double cuda_fma_per_point(const Plan& p) {
+  const int n = 2 * p.R + 1;
+  auto plane_cost = [&](int q) {
+    double f = 0;
+    int cnt = 0;
+    bool all_arms = true, pma_like = true;
+    for (const Term& t : p.terms) {
+      if (t.plane != q) continue;
+      ++cnt;
+      if (t.kind != kArm) all_arms = false;
+      if (t.kind == kPoint) f += 1;
+      else if (t.kind == kArm) f += 2 * t.r + 1;
+      else f += 2.0 * (2 * t.r + 1);
+    }
+    (void)pma_like;
+    if (p.ndim == 3 && cnt > 0 && !(cnt == 1) && !(cnt == 2 && all_arms)) f = cnt * 2.0 * n;  // general chains
+    return f;
+  };
+  if (p.ndim == 2) {
+    double f = plane_cost(0);
+    return f;
+  }
   double f = 0;
-  for (const Term& t : p.terms) {
-    if (t.kind == kPoint) f += 1;
-    else if (t.kind == kArm) f += 2 * t.r + 1;
-    else f += 2.0 * (2 * t.r + 1);
+  for (int q = 0; q < n; ++q) {
+    bool mirrored = false;
+    if (q > p.R) {
+      const int m = 2 * p.R - q;
+      mirrored = true;
+      for (int e = 0; e < n * n; ++e)
+        if (p.W[size_t(q) * n * n + e] != p.W[size_t(m) * n * n + e]) { mirrored = false; break; }
+    }
+    if (!mirrored) f += plane_cost(q);
+    else f += 1;  // the extra add into the mirrored output plane
   }
   return f;
 }
@@ -241,7 +271,8 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
   // DMMA 37 TF, DFMA 34 TF, one shared FP64 budget).
   int eng = o ? o->engine : LORA_ENGINE_AUTO;
   if (eng < 0 || eng > LORA_ENGINE_DIRECT) { err = "unknown engine"; return LORA_ERR_INVALID_ARG; }
-  const double c_tc = tc_fma_per_point(p) / 37.0, c_rdg = cuda_fma_per_point(p) / 34.0, c_dir = p.fma_direct / 34.0;
+  const double dense = p.ndim == 2 ? double(n) * n : double(n) * n * n;  // the direct kernel issues every tap
+  const double c_tc = tc_fma_per_point(p) / 37.0, c_rdg = cuda_fma_per_point(p) / 34.0, c_dir = dense / 34.0;
   const bool ok_tc = tc2d_supported(p), ok_rdg = rdg2d_supported(p);
   if (eng == LORA_ENGINE_AUTO) {
     eng = LORA_ENGINE_DIRECT;
@@ -253,7 +284,7 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
     return LORA_ERR_UNSUPPORTED;
   }
   p.engine = eng;
-  p.fma_issued = eng == LORA_ENGINE_TC ? tc_fma_per_point(p) : eng == LORA_ENGINE_RDG_CUDA ? cuda_fma_per_point(p) : p.fma_direct;
+  p.fma_issued = eng == LORA_ENGINE_TC ? tc_fma_per_point(p) : eng == LORA_ENGINE_RDG_CUDA ? cuda_fma_per_point(p) : dense;
   int fk = o ? o->fuse_k : 0;
   if (fk < 0) { err = "fuse_k must be >= 0"; return LORA_ERR_INVALID_ARG; }
   p.fuse_k = fk == 0 ? 1 : fk;

@@ -66,16 +66,37 @@ def test_integer_exact_bitwise(engine):
     assert np.array_equal(out, ref)
 
 
+ENGINES_3D = ["direct", "rdg_cuda"]
+
+
+@pytest.mark.parametrize("engine", ENGINES_3D)
 @pytest.mark.parametrize("h", [1, 2])
-@pytest.mark.parametrize("kind", ["rsym", "star", "asym"])
-@pytest.mark.parametrize("shape", [(1, 1, 1), (3, 4, 5), (17, 9, 33), (70, 12, 40)])
-def test_3d_parity_small(h, kind, shape):
-    W = _weights(kind, 3, h, 3 + h)
+@pytest.mark.parametrize("kind", ["rsym", "star", "asym", "heat3d"])
+@pytest.mark.parametrize("shape", [(1, 1, 1), (3, 4, 5), (17, 9, 33), (70, 12, 40), (130, 6, 66)])
+def test_3d_parity_small(engine, h, kind, shape):
+    if kind == "heat3d":
+        if h != 1:
+            pytest.skip("preset is radius 1")
+        W = synth.preset("heat3d")
+    else:
+        W = _weights(kind, 3, h, 3 + h)
     g = synth.grid(tuple(n + 2 * h for n in shape), 5)
-    for T in (1, 2):
-        out, info = run_gpu(W, g, T)
+    for T in (1, 2, 3):
+        out, info = run_gpu(W, g, T, engine=engine)
         ref = oracle.run(W, g, T)
-        assert rel_err(out, ref) <= 1e-12
+        assert info["engine_name"] == engine
+        assert rel_err(out, ref) <= 1e-12, (T, rel_err(out, ref))
+
+
+@pytest.mark.parametrize("engine", ENGINES_3D)
+def test_3d_staging_paths_agree(engine, monkeypatch):
+    W = synth.rsym_weights(3, 1, 8)
+    g = synth.grid((34, 20, 66), 12)
+    a, _ = run_gpu(W, g, 3, engine=engine)
+    monkeypatch.setenv("LORA_NO_TMA", "1")
+    b, _ = run_gpu(W, g, 3, engine=engine)
+    assert np.array_equal(a, b)
+    assert rel_err(a, oracle.run(W, g, 3)) <= 1e-12
 
 
 @pytest.mark.parametrize("engine", ENGINES_2D)

@@ -1,0 +1,165 @@
+"""Host-side tests (no GPU): the C-ABI library loads and exports every symbol the header declares,
+and the planner's factorisation satisfies what the paper fixes (eq. 8/9/15)
+and DESIGN.md reading Q6 for the cases the paper leaves open."""
+import json
+import math
+import os
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def L():
+    from paper_conf_sc_zhanglyczcy24_b200 import _build
+    _build.build()
+    import paper_conf_sc_zhanglyczcy24_b200 as L
+    return L
+
+
+def test_library_exports_every_header_symbol(L):
+    hdr = open(os.path.join(ROOT, "include", "lora_stencil.h")).read()
+    declared = set(re.findall(r"\b(lora_stencil_\w+)\s*\(", hdr))
+    assert len(declared) >= 14
+    import ctypes
+    lib = ctypes.CDLL(L.LIB_PATH)
+    for name in declared:
+        assert hasattr(lib, name), name
+    assert set(L.EXPORTED) == declared
+    assert "sm_100a" in L.lora_stencil_version()
+
+
+def test_library_has_no_oracle_dependency():
+    """The product library must not link or embed the oracle (task rule ③)."""
+    import subprocess
+    lib = os.path.join(ROOT, "paper_conf_sc_zhanglyczcy24_b200", "liblora_stencil.so")
+    syms = subprocess.run(["nm", "-D", lib], capture_output=True, text=True).stdout
+    assert "oracle" not in syms
+    deps = subprocess.run(["ldd", lib], capture_output=True, text=True).stdout
+    assert "oracle" not in deps
+
+
+def _recon(terms, plane_shape_n, nplanes=1):
+    n = plane_shape_n
+    W = np.zeros((nplanes, n, n))
+    for t in terms:
+        W[t["plane"]] += np.outer(t["u"], t["v"])
+    return W
+
+
+@pytest.mark.parametrize("h", [1, 2, 3, 4])
+def test_pma_rsym_plan_matches_paper_pyramid(L, h):
+    """Radially symmetric W: h+1 terms, sizes 2h+3-2i (eq. 15), the last a scalar,
+    reconstruction <= 1e-14, and the same factors as the oracle's step-by-step PMA."""
+    W = synth.rsym_weights(2, h, 200 + h)
+    st = L.Stencil(W, (100, 100), engine="rdg_cuda")
+    terms = st.terms()
+    assert [t["radius"] for t in terms] == list(range(h, 0, -1)) + [0]
+    assert [t["kind"] for t in terms] == [0] * h + [2]
+    R = _recon(terms, 2 * h + 1)[0]
+    assert np.abs(R - W).max() <= 1e-14 * np.abs(W).max()
+    ref = oracle.pma(W)
+    for t, (u, v) in zip(terms, ref):
+        m = len(u)
+        o = h - (m - 1) // 2
+        np.testing.assert_allclose(t["u"][o:o + m], u, rtol=0, atol=1e-15)
+        np.testing.assert_allclose(t["v"][o:o + m], v, rtol=0, atol=1e-17)
+    info = st.info()
+    assert info["recon_err"] <= 1e-14 and info["n_tc_chain"] == h and info["n_cuda"] == 1
+
+
+def test_star_gives_two_arms(L):
+    for h in (1, 2, 3):
+        W = synth.star_weights(2, h, 5)
+        st = L.Stencil(W, (10, 10))
+        terms = st.terms()
+        assert [t["kind"] for t in terms] == [1, 1]
+        assert np.abs(_recon(terms, 2 * h + 1)[0] - W).max() <= 1e-16
+
+
+def test_separable_weights_give_one_term_no_nan(L):
+    """A separable W (Box-2D9P composed, Gaussian) makes naive PMA divide 0/0 in ring 2;
+    the rank-revealing stop must give a single term (Q6)."""
+    v = np.array([1.0, 4.0, 6.0, 4.0, 1.0]); W = np.outer(v, v) / 256.0
+    st = L.Stencil(W, (10, 10))
+    terms = st.terms()
+    assert len(terms) == 1 and all(np.isfinite(t["u"]).all() and np.isfinite(t["v"]).all() for t in terms)
+    assert st.info()["recon_err"] <= 1e-15
+
+
+def test_asymmetric_uses_elimination(L):
+    for h in (1, 2, 3, 4):
+        W = synth.asym_weights(2, h, 7)
+        st = L.Stencil(W, (10, 10))
+        terms = st.terms()
+        assert len(terms) <= 2 * h + 1
+        assert np.abs(_recon(terms, 2 * h + 1)[0] - W).max() <= 1e-14 * np.abs(W).max()
+
+
+def test_zero_and_single_weight_planes(L):
+    W = np.zeros((3, 3)); W[0, 2] = 0.5
+    st = L.Stencil(W, (4, 4))
+    t = st.terms()
+    assert len(t) == 1 and t[0]["kind"] == 2
+    W = np.zeros((3, 3, 3)); W[1] = synth.rsym_weights(2, 1, 3) * 0.5; W[0, 1, 1] = W[2, 1, 1] = 0.25
+    st = L.Stencil(W, (4, 4, 4))
+    info = st.info()
+    assert info["n_planes_pointwise"] == 2 and info["z_symmetric"] == 1
+
+
+def test_integer_pyramid_factors_are_exact(L):
+    W = synth.integer_pyramid_weights()
+    terms = L.Stencil(W, (8, 8)).terms()
+    assert np.array_equal(terms[0]["u"], [1, 2, 3, 4, 3, 2, 1])
+    assert np.array_equal(terms[1]["v"][1:6], [1, 1, 2, 1, 1])
+    assert np.array_equal(terms[2]["v"][2:5], [2, 4, 2]) and terms[3]["v"][3] == 3.0
+    assert np.array_equal(_recon(terms, 7)[0], W)
+
+
+@pytest.mark.parametrize("name", ["heat3d", "box3d27p"])
+def test_3d_plane_decomposition_alg2(L, name):
+    """Alg. 2: every plane factored; sum over planes reconstructs W; Heat-3D has
+    two single-weight planes (CUDA-core point-wise) and a star centre plane."""
+    W = synth.preset("heat3d") if name == "heat3d" else synth.rsym_weights(3, 1, 9)
+    st = L.Stencil(W, (8, 8, 8))
+    R = _recon(st.terms(), 3, 3)
+    assert np.abs(R - W).max() <= 1e-15
+    info = st.info()
+    assert info["z_symmetric"] == 1
+    if name == "heat3d":
+        assert info["n_planes_pointwise"] == 2 and info["n_tc_single"] == 2
+
+
+def test_invalid_arguments(L):
+    W = synth.rsym_weights(2, 1, 1)
+    with pytest.raises(L.LoraError):
+        L.lora_stencil_plan(W, 4, 1, [10, 10])
+    with pytest.raises(L.LoraError):
+        L.lora_stencil_plan(np.zeros((11, 11)), 2, 5, [10, 10])          # radius > 4
+    with pytest.raises(L.LoraError):
+        L.lora_stencil_plan(W, 2, 1, [0, 10])
+    bad = W.copy(); bad[0, 0] = np.nan
+    with pytest.raises(L.LoraError):
+        L.lora_stencil_plan(bad, 2, 1, [10, 10])
+    assert "finite" in L.lora_stencil_last_error()
+
+
+def test_cost_model_reproduces_paper_counts():
+    """Paper's analytic counts (tests/golden/paper_counts.json) from their formulas:
+    eq. 14 ratio ceil((2h+1)^2/4)/(h+1); eq. 16 MMA count at h = 3 vs ConvStencil's 26."""
+    gold = json.load(open(os.path.join(ROOT, "tests", "golden", "paper_counts.json")))
+    r = lambda h: math.ceil((2 * h + 1) ** 2 / 4) / (h + 1)
+    assert r(3) == gold["eq14_convstencil_over_rdg"]["h3"] and r(4) == gold["eq14_convstencil_over_rdg"]["h4"]
+    assert round(1 - 1 / r(3), 4) == gold["eq14_redundancy_eliminated"]["h3"]
+    assert round(1 - 1 / r(4), 4) == gold["eq14_redundancy_eliminated"]["h4"]
+    h = 3
+    lora = 2 * h * math.ceil(h / 2) * (2 * math.ceil(h / 4) + 1)          # eq. 16 per (32 ceil(h/2) ceil(h/4)) points
+    conv = 2 * math.ceil((2 * h + 1) ** 2 / 4)                             # eq. 13 per 8(2h+2) points ... per same block
+    assert lora == gold["eq16_mma_ratio_h3"]["lora"] and conv == gold["eq16_mma_ratio_h3"]["convstencil"]
+    assert gold["fusion_fragment_waste"]["saved"] / gold["fusion_fragment_waste"]["total"] == pytest.approx(0.6154, abs=1e-4)
