@@ -145,6 +145,14 @@ int lora_stencil_run_dist(lora_plan* p, lora_comm* c, const double* in_local, do
                           void* stream);
 void lora_stencil_comm_destroy(lora_comm* c);
 
+/* Host-only: the halo exchange `rank` of `nranks` performs after every step of
+ * lora_stencil_run_dist on a buffer of plan p's local padded shape (used by the run itself and by
+ * the CPU tests).  Writes up to 4 entries, in issue order inside one NCCL group: kind[i]
+ * (0 = send, 1 = recv), peer[i], offset[i] (elements from the buffer start) and count[i]
+ * (elements, contiguous).  Returns the number of entries (0..4) or a negative lora_status. */
+int lora_stencil_dist_exchange_plan(const lora_plan* p, int rank, int nranks, int64_t* kind, int64_t* peer,
+                                    int64_t* offset, int64_t* count);
+
 /* Thread-local message for the last failure on this thread ("" if none). */
 const char* lora_stencil_last_error(void);
 /* Library version string. */

@@ -73,6 +73,7 @@ _sig = {
     "lora_stencil_comm_init": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_int, _P]),
     "lora_stencil_run_dist": (ctypes.c_int, [_P, _P, _P, _P, ctypes.c_int64, _P]),
     "lora_stencil_comm_destroy": (None, [_P]),
+    "lora_stencil_dist_exchange_plan": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_int, _P, _P, _P, _P]),
     "lora_stencil_last_error": (ctypes.c_char_p, []),
     "lora_stencil_version": (ctypes.c_char_p, []),
 }
@@ -178,6 +179,15 @@ def lora_stencil_run_dist(plan, comm, in_ptr: int, out_ptr: int, timesteps: int,
 
 def lora_stencil_comm_destroy(comm) -> None:
     _lib.lora_stencil_comm_destroy(comm)
+
+
+def lora_stencil_dist_exchange_plan(plan, rank: int, nranks: int):
+    """[(kind 'send'|'recv', peer, element offset, element count)] in NCCL-group issue order."""
+    a = [np.zeros(4, np.int64) for _ in range(4)]
+    m = _lib.lora_stencil_dist_exchange_plan(plan, int(rank), int(nranks), *[x.ctypes.data for x in a])
+    if m < 0:
+        raise LoraError(m, lora_stencil_last_error())
+    return [("send" if a[0][i] == 0 else "recv", int(a[1][i]), int(a[2][i]), int(a[3][i])) for i in range(m)]
 
 
 class Stencil:

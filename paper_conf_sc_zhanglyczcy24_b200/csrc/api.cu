@@ -12,13 +12,11 @@
 #include "kernels.hpp"
 #include "plan.hpp"
 
-struct lora_plan : lora::Plan {};
-
 namespace lora {
 thread_local std::string g_err;
 int fail(int code, const std::string& msg) { g_err = msg; return code; }
-int cuda_fail(cudaError_t e, const char* what) {
-  g_err = std::string(what) + ": " + cudaGetErrorString(e);
+int cuda_fail(int e, const char* what) {
+  g_err = std::string(what) + ": " + cudaGetErrorString(static_cast<cudaError_t>(e));
   return LORA_ERR_CUDA;
 }
 bool sync_check() {
@@ -46,6 +44,12 @@ cudaError_t step(const Plan& p, const double* src, double* dst, cudaStream_t s) 
     case LORA_ENGINE_RDG_CUDA: return launch_rdg2d(p, src, dst, s);
     default: return launch_direct(p, src, dst, s);
   }
+}
+int step_launch(const Plan& p, const double* src, double* dst, void* stream) {
+  return (int)step(p, src, dst, static_cast<cudaStream_t>(stream));
+}
+int copy_halo_launch(const Plan& p, const double* in, double* dst, void* stream) {
+  return (int)launch_copy_halo(p, in, dst, static_cast<cudaStream_t>(stream));
 }
 
 int run_device(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s) {

@@ -1,12 +1,200 @@
-// Multi-GPU slab decomposition (placeholder until the NCCL path lands).
-#include <cstddef>
+// Multi-GPU: slab decomposition along the slowest axis with a per-step halo exchange over NCCL
+// (north star (d); the paper itself is single-GPU).
+//
+// Rank q owns interior rows (2D) or planes (3D) [s_q, s_q + n_q) of the global grid and a padded
+// local array of n_q + 2R rows/planes.  Halo rows/planes are contiguous, so ncclSend/ncclRecv move
+// them in place (no pack kernel).  Per time step t: step src -> dst on this rank's slab, then a
+// grouped exchange fills dst's slab-edge halos with the neighbours' step-t edge rows (rank 0's low
+// halo and rank n-1's high halo are the physical Dirichlet boundary and are never exchanged).
+// Every point is computed with the single-GPU kernels, so the result is bitwise equal to a
+// single-GPU run of the global grid (pin P10).
+//
+// NCCL is loaded at run time (dlopen of the libnccl.so.2 the process already has — torch's — or
+// the system one), so the library has no link-time NCCL dependency.
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <string>
 
 #include "lora_stencil.h"
+#include "plan.hpp"
+
+namespace {
+using ncclComm_t = struct ncclComm*;
+struct ncclUniqueId { char internal[128]; };
+using ncclResult_t = int;
+constexpr int kNcclFloat64 = 8;
+
+struct Nccl {
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*Send)(const void*, size_t, int, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Recv)(void*, size_t, int, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*GroupStart)() = nullptr;
+  ncclResult_t (*GroupEnd)() = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+  bool ok = false;
+};
+
+Nccl& nccl() {
+  static Nccl n;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return;
+    n.GetUniqueId = (decltype(n.GetUniqueId))dlsym(h, "ncclGetUniqueId");
+    n.CommInitRank = (decltype(n.CommInitRank))dlsym(h, "ncclCommInitRank");
+    n.CommDestroy = (decltype(n.CommDestroy))dlsym(h, "ncclCommDestroy");
+    n.Send = (decltype(n.Send))dlsym(h, "ncclSend");
+    n.Recv = (decltype(n.Recv))dlsym(h, "ncclRecv");
+    n.GroupStart = (decltype(n.GroupStart))dlsym(h, "ncclGroupStart");
+    n.GroupEnd = (decltype(n.GroupEnd))dlsym(h, "ncclGroupEnd");
+    n.GetErrorString = (decltype(n.GetErrorString))dlsym(h, "ncclGetErrorString");
+    n.ok = n.GetUniqueId && n.CommInitRank && n.CommDestroy && n.Send && n.Recv && n.GroupStart && n.GroupEnd;
+  });
+  return n;
+}
+
+int nccl_fail(ncclResult_t r, const char* what) {
+  std::string m = std::string(what) + ": NCCL error " + std::to_string(r);
+  if (nccl().GetErrorString) m += std::string(" (") + nccl().GetErrorString(r) + ")";
+  return lora::fail(LORA_ERR_NCCL, m);
+}
+}  // namespace
+
+struct lora_comm {
+  ncclComm_t comm = nullptr;
+  int rank = 0, nranks = 1, device = -1;
+};
+
+namespace {
+int exchange_plan(const lora_plan* p, int rank, int nranks, int64_t* kind, int64_t* peer, int64_t* off, int64_t* cnt) {
+  const int R = p->R;
+  const int64_t row = p->ndim == 2 ? p->P[1] : p->P[1] * p->P[2];   // elements per padded row/plane
+  const int64_t n0 = p->N[0];
+  int k = 0;
+  if (rank > 0) {  // my first R interior rows go down; the neighbour's last R fill my low halo
+    kind[k] = 0; peer[k] = rank - 1; off[k] = R * row; cnt[k] = R * row; ++k;
+    kind[k] = 1; peer[k] = rank - 1; off[k] = 0; cnt[k] = R * row; ++k;
+  }
+  if (rank < nranks - 1) {  // my last R interior rows go up; the neighbour's first R fill my high halo
+    kind[k] = 0; peer[k] = rank + 1; off[k] = n0 * row; cnt[k] = R * row; ++k;
+    kind[k] = 1; peer[k] = rank + 1; off[k] = (n0 + R) * row; cnt[k] = R * row; ++k;
+  }
+  return k;
+}
+
+// Fills buf's slab-edge halos from the neighbours (one NCCL group, stream-ordered).
+int exchange(const lora_plan* p, lora_comm* c, double* buf, cudaStream_t s) {
+  if (c->nranks == 1) return LORA_OK;
+  int64_t kind[4], peer[4], off[4], cnt[4];
+  const int m = exchange_plan(p, c->rank, c->nranks, kind, peer, off, cnt);
+  Nccl& n = nccl();
+  ncclResult_t r = n.GroupStart();
+  if (r) return nccl_fail(r, "ncclGroupStart");
+  for (int i = 0; i < m; ++i) {
+    r = kind[i] == 0 ? n.Send(buf + off[i], size_t(cnt[i]), kNcclFloat64, (int)peer[i], c->comm, s)
+                     : n.Recv(buf + off[i], size_t(cnt[i]), kNcclFloat64, (int)peer[i], c->comm, s);
+    if (r) { n.GroupEnd(); return nccl_fail(r, kind[i] == 0 ? "ncclSend" : "ncclRecv"); }
+  }
+  if ((r = n.GroupEnd())) return nccl_fail(r, "ncclGroupEnd");
+  return LORA_OK;
+}
+}  // namespace
 
 extern "C" {
-size_t lora_stencil_comm_id_size(void) { return 128; }
-int lora_stencil_comm_get_id(void*) { return LORA_ERR_NCCL; }
-int lora_stencil_comm_init(lora_comm**, int, int, const void*) { return LORA_ERR_NCCL; }
-int lora_stencil_run_dist(lora_plan*, lora_comm*, const double*, double*, int64_t, void*) { return LORA_ERR_NCCL; }
-void lora_stencil_comm_destroy(lora_comm*) {}
+
+size_t lora_stencil_comm_id_size(void) { return sizeof(ncclUniqueId); }
+
+int lora_stencil_dist_exchange_plan(const lora_plan* p, int rank, int nranks, int64_t* kind, int64_t* peer,
+                                    int64_t* offset, int64_t* count) {
+  if (!p || !kind || !peer || !offset || !count || nranks < 1 || rank < 0 || rank >= nranks)
+    return lora::fail(LORA_ERR_INVALID_ARG, "bad exchange-plan arguments");
+  if (nranks > 1 && p->N[0] < p->R) return lora::fail(LORA_ERR_INVALID_ARG, "each slab needs >= radius rows/planes");
+  return exchange_plan(p, rank, nranks, kind, peer, offset, count);
 }
+
+int lora_stencil_comm_get_id(void* id_out) {
+  if (!id_out) return lora::fail(LORA_ERR_INVALID_ARG, "NULL id buffer");
+  if (!nccl().ok) return lora::fail(LORA_ERR_NCCL, "libnccl.so.2 could not be loaded");
+  ncclUniqueId id;
+  ncclResult_t r = nccl().GetUniqueId(&id);
+  if (r) return nccl_fail(r, "ncclGetUniqueId");
+  std::memcpy(id_out, &id, sizeof(id));
+  return LORA_OK;
+}
+
+int lora_stencil_comm_init(lora_comm** c, int nranks, int rank, const void* nccl_unique_id) {
+  if (!c || !nccl_unique_id || nranks < 1 || rank < 0 || rank >= nranks)
+    return lora::fail(LORA_ERR_INVALID_ARG, "bad comm arguments");
+  *c = nullptr;
+  lora_comm* cc = new (std::nothrow) lora_comm();
+  if (!cc) return lora::fail(LORA_ERR_OOM, "out of host memory");
+  cc->rank = rank;
+  cc->nranks = nranks;
+  cudaGetDevice(&cc->device);
+  if (nranks > 1) {
+    if (!nccl().ok) { delete cc; return lora::fail(LORA_ERR_NCCL, "libnccl.so.2 could not be loaded"); }
+    ncclUniqueId id;
+    std::memcpy(&id, nccl_unique_id, sizeof(id));
+    ncclResult_t r = nccl().CommInitRank(&cc->comm, nranks, id, rank);
+    if (r) { delete cc; return nccl_fail(r, "ncclCommInitRank"); }
+  }
+  *c = cc;
+  return LORA_OK;
+}
+
+int lora_stencil_run_dist(lora_plan* p, lora_comm* c, const double* in_local, double* out_local, int64_t timesteps,
+                          void* stream) {
+  using namespace lora;
+  if (!p || !c || !in_local || !out_local) return fail(LORA_ERR_INVALID_ARG, "NULL plan, comm, in or out");
+  if (timesteps < 0) return fail(LORA_ERR_INVALID_ARG, "timesteps must be >= 0");
+  if (c->nranks > 1 && p->N[0] < p->R) return fail(LORA_ERR_INVALID_ARG, "each slab needs >= radius rows/planes");
+  const size_t bytes = p->elems * sizeof(double);
+  const char* a = reinterpret_cast<const char*>(in_local);
+  const char* b = reinterpret_cast<const char*>(out_local);
+  if (a < b + bytes && b < a + bytes) return fail(LORA_ERR_ALIAS, "in and out overlap");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (timesteps == 0) {
+    cudaError_t e = cudaMemcpyAsync(out_local, in_local, bytes, cudaMemcpyDeviceToDevice, s);
+    return e == cudaSuccess ? LORA_OK : cuda_fail(e, "cudaMemcpyAsync");
+  }
+  int rc = ensure_device(*p, timesteps >= 2);
+  if (rc) return rc;
+  int e = copy_halo_launch(*p, in_local, out_local, s);
+  if (e) return cuda_fail(e, "copy_halo launch");
+  if (timesteps >= 2) {
+    e = copy_halo_launch(*p, in_local, p->scratch, s);
+    if (e) return cuda_fail(e, "copy_halo launch");
+  }
+  // in_local's slab-edge halos hold the neighbours' initial rows (a slice of the global padded
+  // array); every later buffer gets them from the exchange after each step.
+  const double* src = in_local;
+  for (int64_t t = 1; t <= timesteps; ++t) {
+    double* dst = ((timesteps - t) % 2 == 0) ? out_local : p->scratch;
+    e = step_launch(*p, src, dst, s);
+    if (e) return cuda_fail(e, "stencil kernel launch");
+    rc = exchange(p, c, dst, s);
+    if (rc) return rc;
+    src = dst;
+  }
+  if (sync_check()) {
+    cudaError_t ce = cudaStreamSynchronize(s);
+    if (ce != cudaSuccess) return cuda_fail(ce, "LORA_SYNC_CHECK stream sync");
+  }
+  return LORA_OK;
+}
+
+void lora_stencil_comm_destroy(lora_comm* c) {
+  if (!c) return;
+  if (c->comm && nccl().ok) nccl().CommDestroy(c->comm);
+  delete c;
+}
+
+}  // extern "C"

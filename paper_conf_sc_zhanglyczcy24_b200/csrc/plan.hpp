@@ -53,4 +53,14 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
 double tc_fma_per_point(const Plan& p);
 double cuda_fma_per_point(const Plan& p);
 
+// api.cu
+int fail(int code, const std::string& msg);
+int cuda_fail(int /*cudaError_t*/ e, const char* what);
+int ensure_device(Plan& p, bool want_scratch);
+int step_launch(const Plan& p, const double* src, double* dst, void* stream);       // cudaError_t
+int copy_halo_launch(const Plan& p, const double* in, double* dst, void* stream);   // cudaError_t
+bool sync_check();
+
 }  // namespace lora
+
+struct lora_plan : lora::Plan {};
