@@ -38,10 +38,11 @@ int ensure_device(Plan& p, bool want_scratch) {
   return LORA_OK;
 }
 
-cudaError_t step(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+// One launch advancing `k` time steps (k > 1 only for engines that fuse, see plan.fuse_k).
+cudaError_t step(const Plan& p, const double* src, double* dst, cudaStream_t s, int k = 1) {
   switch (p.engine) {
     case LORA_ENGINE_TC: return launch_tc2d(p, src, dst, s);
-    case LORA_ENGINE_RDG_CUDA: return launch_rdg2d(p, src, dst, s);
+    case LORA_ENGINE_RDG_CUDA: return launch_rdg2d(p, src, dst, s, k);
     default: return launch_direct(p, src, dst, s);
   }
 }
@@ -58,19 +59,24 @@ int run_device(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s
     cudaError_t e = cudaMemcpyAsync(out, in, bytes, cudaMemcpyDeviceToDevice, s);
     return e == cudaSuccess ? LORA_OK : cuda_fail(e, "cudaMemcpyAsync");
   }
-  int rc = ensure_device(p, T >= 2);
+  const bool two = (T + (p.fuse_k < 1 ? 1 : p.fuse_k) - 1) / (p.fuse_k < 1 ? 1 : p.fuse_k) >= 2;
+  int rc = ensure_device(p, two);
   if (rc) return rc;
   cudaError_t e = launch_copy_halo(p, in, out, s);
   if (e != cudaSuccess) return cuda_fail(e, "copy_halo launch");
-  if (T >= 2) {
+  if (two) {
     e = launch_copy_halo(p, in, p.scratch, s);
     if (e != cudaSuccess) return cuda_fail(e, "copy_halo launch");
   }
-  // step t (1..T) writes `out` when (T - t) is even, else the scratch buffer.
+  // ceil(T / k) launches of k fused steps (the last one takes the remainder); launch i writes
+  // `out` when (L - 1 - i) is even, else the scratch buffer, so the last lands in `out`.
+  const int64_t k = p.fuse_k < 1 ? 1 : p.fuse_k;
+  const int64_t L = (T + k - 1) / k;
   const double* src = in;
-  for (int64_t t = 1; t <= T; ++t) {
-    double* dst = ((T - t) % 2 == 0) ? out : p.scratch;
-    e = step(p, src, dst, s);
+  for (int64_t i = 0; i < L; ++i) {
+    const int64_t steps = (i == L - 1) ? T - k * (L - 1) : k;
+    double* dst = ((L - 1 - i) % 2 == 0) ? out : p.scratch;
+    e = step(p, src, dst, s, (int)steps);
     if (e != cudaSuccess) return cuda_fail(e, "stencil kernel launch");
     src = dst;
   }

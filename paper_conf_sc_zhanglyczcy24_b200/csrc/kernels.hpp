@@ -16,8 +16,10 @@ cudaError_t launch_direct(const Plan& p, const double* src, double* dst, cudaStr
 // K1 (2D): RDG chains U_k X V_k on FP64 tensor cores (DMMA m8n8k4) with BVS, one step.
 cudaError_t launch_tc2d(const Plan& p, const double* src, double* dst, cudaStream_t s);
 
-// K6 (2D): RDG chains as banded passes on the FP64 CUDA-core pipe, one step.
-cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s);
+// K6 (2D): RDG chains as banded passes on the FP64 CUDA-core pipe, k fused steps (exact temporal
+// blocking, halo re-imposed every sub-step); 3D dispatches to launch_rdg3d (k = 1).
+cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s, int k);
+int rdg2d_max_fuse(const Plan& p);
 
 // K2 on CUDA cores (3D, Alg. 2 with RDG per plane), one step.
 cudaError_t launch_rdg3d(const Plan& p, const double* src, double* dst, cudaStream_t s);

@@ -28,7 +28,7 @@ namespace {
 
 constexpr int RDG_RC = 128;     // output rows per work item (chunk)
 constexpr int RDG_WARPS = 4;    // warps per CTA (independent streams)
-constexpr int RDG_NS = 4;       // ring stages per warp
+constexpr int RDG_NS = 3;       // ring stages per warp (3 keeps 4 CTAs = 16 warps per SM)
 
 enum { SIG_PMA = 0, SIG_STAR = 1, SIG_FULL = 2 };
 
@@ -66,15 +66,24 @@ __device__ __forceinline__ void row_body(const double* __restrict__ xs, int p, d
     x[2 * q + 1] = t.y;
   }
   if constexpr (SIG == SIG_PMA) {
-    // PMA pyramid (eq. 15): term k has radius R-k; the last one is the scalar C_{h+1}.
+    // PMA pyramid (eq. 15): term k has radius R-k; the last one is the scalar C_{h+1}.  The PMA
+    // factors of a reflection-symmetric W are exactly palindromic (the planner takes the
+    // PMA route only for exactly symmetric remainders), so the horizontal gather pairs the taps:
+    // T = v_0 x_0 + sum_b v_b (x_{-b} + x_{+b}); the pair sums are shared by all terms.
+    double sp0[R + 1], sp1[R + 1];
+#pragma unroll
+    for (int b = 1; b <= R; ++b) {
+      sp0[b] = x[R - b] + x[R + b];
+      sp1[b] = x[R - b + 1] + x[R + b + 1];
+    }
 #pragma unroll
     for (int k = 0; k < R; ++k) {
       const int H = R - k;
-      double t0 = 0.0, t1 = 0.0;
+      double t0 = P.v[k][R] * x[R], t1 = P.v[k][R] * x[R + 1];
 #pragma unroll
-      for (int b = -H; b <= H; ++b) {
-        t0 = fma(P.v[k][R + b], x[R + b], t0);
-        t1 = fma(P.v[k][R + b], x[R + b + 1], t1);
+      for (int b = 1; b <= H; ++b) {
+        t0 = fma(P.v[k][R + b], sp0[b], t0);
+        t1 = fma(P.v[k][R + b], sp1[b], t1);
       }
 #pragma unroll
       for (int a = -H; a <= H; ++a) {
@@ -125,65 +134,141 @@ __device__ __forceinline__ void row_body(const double* __restrict__ xs, int p, d
   }
 }
 
-template <int R, int SIG, int I>
-__device__ __forceinline__ void stage_rows(const double* __restrict__ st, int p, double (&acc)[2 * R + 1][2],
-                                           const RdgParams& P, int rbase, double* __restrict__ orow0, int64_t P1,
-                                           int rows_valid, bool c0ok, bool c1ok, bool vec) {
+// ---------------------------------------------------------------------------------------------
+// Exact temporal fusion (§IV-A; reading Q5): K time steps per HBM
+// round trip.  Stage 1 consumes the staged input rows; every completed step-s row is written to a
+// per-warp shared row buffer (double-buffered by row parity) that stage s+1 consumes exactly like
+// an input row, so the K steps form a software pipeline down the stream (stage s lags by s*R
+// rows).  Each intermediate row re-imposes the fixed Dirichlet halo (rows/columns of the halo take
+// the input values, P:21 Jacobi semantics), so the result equals K separate steps.  The lane
+// columns lose R valid columns per fused step at each band edge: bands overlap, stride
+// S = 64 - 2R(K-1) (minus 2 when R(K-1) is odd, so that the staged tile starts on an even column:
+// TMA faults on a box whose innermost start is not 16-byte aligned, tools/ubench/tma_probe.cu).
+struct Item {
+  int64_t X0;    // padded column of lane column 0
+  int64_t A;     // first final output row (padded)
+  int64_t q0;    // first consumed input row (padded)
+};
+
+template <int R, int SIG, int K, int I0, int S>
+__device__ __forceinline__ void fused_stage(const double* __restrict__ src, int p, double (&acc)[K][2 * R + 1][2],
+                                            const RdgParams& P, int64_t q, double* const* __restrict__ bufs, int par,
+                                            const double* __restrict__ in, double* __restrict__ out, int64_t P0,
+                                            int64_t P1, const Item& it, int RC, const int64_t (&c)[2],
+                                            const bool (&inside)[2], const bool (&colhalo)[2], const bool (&valid)[2],
+                                            bool vec) {
   constexpr int n = 2 * R + 1;
-  if constexpr (I < Geom<R>::SROWS) {
-    row_body<R, SIG, I % n>(st + I * Geom<R>::BW, p, acc, P);
-    // output row y = r - 2R is complete; its ring slot is (I + 1) mod n
-    constexpr int s = (I + 1) % n;
-    const int y = rbase + I - 2 * R;
-    if (y >= 0 && y < rows_valid) {
-      double* o = orow0 + int64_t(y) * P1;
+  constexpr int Is = pmod(I0 - (S - 1) * R, n);   // row index mod n of stage S's input row
+  row_body<R, SIG, Is>(src, p, acc[S - 1], P);
+  constexpr int cs = (Is + 1) % n;                // slot of the row this stage just completed
+  const int64_t y = q - int64_t(S) * R;           // its padded row index
+  double v0 = acc[S - 1][cs][0], v1 = acc[S - 1][cs][1];
+  acc[S - 1][cs][0] = 0.0;
+  acc[S - 1][cs][1] = 0.0;
+  if constexpr (S < K) {
+    const bool row_in = y >= 0 && y < P0;
+    const bool row_halo = y < R || y >= P0 - R;
+    if (row_halo) {
+      v0 = (row_in && inside[0]) ? in[y * P1 + c[0]] : 0.0;
+      v1 = (row_in && inside[1]) ? in[y * P1 + c[1]] : 0.0;
+    } else {
+      if (colhalo[0]) v0 = in[y * P1 + c[0]];
+      if (colhalo[1]) v1 = in[y * P1 + c[1]];
+      if (!inside[0]) v0 = 0.0;
+      if (!inside[1]) v1 = 0.0;
+    }
+    double* b = bufs[2 * (S - 1) + par];
+    b[R + 2 * p] = v0;
+    b[R + 2 * p + 1] = v1;
+    __syncwarp();
+    fused_stage<R, SIG, K, I0, S + 1>(b, p, acc, P, q, bufs, par, in, out, P0, P1, it, RC, c, inside, colhalo, valid,
+                                      vec);
+  } else {
+    if (y >= it.A && y < it.A + RC && y < P0 - R) {
+      double* o = out + y * P1;
       if (vec) {
-        *reinterpret_cast<double2*>(o) = make_double2(acc[s][0], acc[s][1]);
+        *reinterpret_cast<double2*>(o + c[0]) = make_double2(v0, v1);
       } else {
-        if (c0ok) o[0] = acc[s][0];
-        if (c1ok) o[1] = acc[s][1];
+        if (valid[0]) o[c[0]] = v0;
+        if (valid[1]) o[c[1]] = v1;
       }
     }
-    acc[s][0] = 0.0;
-    acc[s][1] = 0.0;
-    stage_rows<R, SIG, I + 1>(st, p, acc, P, rbase, orow0, P1, rows_valid, c0ok, c1ok, vec);
   }
 }
 
-template <int R, int SIG, bool TMA>
-__global__ void __launch_bounds__(RDG_WARPS * 32, 4) rdg2d_kernel(const double* __restrict__ in, double* __restrict__ out,
-                                                              int64_t N0, int64_t N1, int nbands, int nitems,
-                                                              const __grid_constant__ CUtensorMap tmap,
+template <int R, int SIG, int K, int I>
+__device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p, double (&acc)[K][2 * R + 1][2],
+                                           const RdgParams& P, int64_t qbase, double* const* __restrict__ bufs,
+                                           const double* __restrict__ in, double* __restrict__ out, int64_t P0,
+                                           int64_t P1, const Item& it, int RC, const int64_t (&c)[2],
+                                           const bool (&inside)[2], const bool (&colhalo)[2], const bool (&valid)[2],
+                                           bool vec) {
+  constexpr int n = 2 * R + 1;
+  if constexpr (I < Geom<R>::SROWS) {
+    constexpr int OFF = pmod(R - K * R, n);  // q0 mod n (RC is a multiple of n)
+    const int64_t q = qbase + I;
+    fused_stage<R, SIG, K, pmod(I + OFF, n), 1>(st + I * Geom<R>::BW, p, acc, P, q, bufs, (int)(q & 1), in, out, P0,
+                                                P1, it, RC, c, inside, colhalo, valid, vec);
+    fused_rows<R, SIG, K, I + 1>(st, p, acc, P, qbase, bufs, in, out, P0, P1, it, RC, c, inside, colhalo, valid, vec);
+  }
+}
+
+template <int R, int SIG, int K, bool TMA>
+__global__ void __launch_bounds__(RDG_WARPS * 32, (K == 1 ? 4 : 3)) rdg2d_kernel(const double* __restrict__ in, double* __restrict__ out,
+                                                              int64_t N0, int64_t N1, int nbands, int nitems, int RC,
+                                                              int SI, const __grid_constant__ CUtensorMap tmap,
                                                               const __grid_constant__ RdgParams prm) {
   using G = Geom<R>;
+  constexpr int SG = (R * (K - 1)) & 1;           // shift keeping the staged origin even (TMA: 16-B aligned start)
+  constexpr int BS = 64 - 2 * R * (K - 1) - 2 * SG;  // band stride (valid final columns per band)
+  constexpr int BUFD = ((G::BW + 15) / 16) * 16;  // doubles per intermediate row buffer
   extern __shared__ __align__(128) unsigned char smem_raw[];
   const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw) + wl * RDG_NS;
-  unsigned char* ring = smem_raw + 128 + wl * G::WARP_BYTES;
+  unsigned char* wbase = smem_raw + 128 + wl * (G::WARP_BYTES + 2 * (K - 1) * BUFD * 8);
+  unsigned char* ring = wbase;
+  double* bufmem = reinterpret_cast<double*>(wbase + G::WARP_BYTES);
+  double* bufs[2 * K];                          // [stage][parity]
+#pragma unroll
+  for (int i = 0; i < 2 * (K - 1); ++i) bufs[i] = bufmem + i * BUFD;
+  for (int i = lane; i < 2 * (K - 1) * BUFD; i += 32) bufmem[i] = 0.0;  // margins stay zero
   const int64_t P1 = N1 + 2 * R, P0 = N0 + 2 * R;
   const int gw = blockIdx.x * RDG_WARPS + wl, TW = gridDim.x * RDG_WARPS;
   const int my_items = gw < nitems ? (nitems - 1 - gw) / TW + 1 : 0;
-  const int nstages = my_items * G::SI;
+  const int nstages = my_items * SI;
   if (TMA && lane == 0) {
     for (int s = 0; s < RDG_NS; ++s) mbar_init(&bars[s], 1);
     fence_barrier_init();
   }
   __syncwarp();
-  auto issue = [&](int q) {  // stage q of this warp's sequence into slot q % NS
-    const int item = gw + (q / G::SI) * TW, j = q % G::SI;
+  auto item_of = [&](int q) {
+    const int item = gw + (q / SI) * TW;
     const int band = item % nbands, chunk = item / nbands;
-    const int64_t y = int64_t(chunk) * RDG_RC + int64_t(j) * G::SROWS, x = int64_t(band) * 64;
+    Item it;
+    it.X0 = R + int64_t(band) * BS - int64_t(R) * (K - 1) - SG;
+    it.A = R + int64_t(chunk) * RC;
+    it.q0 = it.A - int64_t(K) * R;
+    return it;
+  };
+  auto issue = [&](int q) {  // stage q of this warp's sequence into slot q % NS
+    const Item it = item_of(q);
+    const int64_t y = it.q0 + int64_t(q % SI) * G::SROWS, x = it.X0 - R;
     double* dst = reinterpret_cast<double*>(ring + (q % RDG_NS) * G::STAGE);
     if constexpr (TMA) {
-      if (lane == 0) {
+      if (x < 0 || y < 0) {  // first band / chunk of a fused launch: no TMA for negative boxes
+        warp_box_fill_sync(dst, in, P0, P1, y, x, G::SROWS, G::BW, lane);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&bars[q % RDG_NS]);
+      } else if (lane == 0) {
+        fence_proxy_async();
         mbar_arrive_expect_tx(&bars[q % RDG_NS], G::SROWS * G::BW * 8);
         tma_load_2d(dst, &tmap, (int)x, (int)y, &bars[q % RDG_NS]);
       }
     } else {
       for (int i = lane; i < G::SROWS * G::BW; i += 32) {
-        const int r = i / G::BW, c = i - r * G::BW;
-        const int64_t gy = y + r, gx = x + c;
-        if (gy < P0 && gx < P1) cp_async8(dst + i, in + gy * P1 + gx);
+        const int r = i / G::BW, cc = i - r * G::BW;
+        const int64_t gy = y + r, gx = x + cc;
+        if (gy >= 0 && gy < P0 && gx >= 0 && gx < P1) cp_async8(dst + i, in + gy * P1 + gx);
         else dst[i] = 0.0;
       }
       cp_async_commit();
@@ -193,7 +278,11 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, 4) rdg2d_kernel(const double* 
     if (q < nstages) issue(q);
     else if constexpr (!TMA) cp_async_commit();  // empty group: keeps wait_group<NS-1> exact
   }
-  double acc[2 * R + 1][2];
+  double acc[K][2 * R + 1][2];
+  Item it{};
+  int64_t c[2] = {0, 0};
+  bool inside[2] = {false, false}, colhalo[2] = {false, false}, valid[2] = {false, false};
+  bool vec = false;
   for (int q = 0; q < nstages; ++q) {
     if (q + RDG_NS - 1 < nstages) issue(q + RDG_NS - 1);
     else if constexpr (!TMA) cp_async_commit();  // keep the group count uniform
@@ -203,20 +292,25 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, 4) rdg2d_kernel(const double* 
       cp_async_wait<RDG_NS - 1>();
       __syncwarp();
     }
-    const int item = gw + (q / G::SI) * TW, j = q % G::SI;
-    const int band = item % nbands, chunk = item / nbands;
+    const int j = q % SI;
     if (j == 0) {
+      it = item_of(q);
 #pragma unroll
-      for (int s = 0; s < 2 * R + 1; ++s) { acc[s][0] = 0.0; acc[s][1] = 0.0; }
+      for (int k = 0; k < K; ++k)
+#pragma unroll
+        for (int s = 0; s < 2 * R + 1; ++s) { acc[k][s][0] = 0.0; acc[k][s][1] = 0.0; }
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        c[e] = it.X0 + 2 * lane + e;
+        inside[e] = c[e] >= 0 && c[e] < P1;
+        colhalo[e] = inside[e] && (c[e] < R || c[e] >= P1 - R);
+        valid[e] = c[e] >= it.X0 + R * (K - 1) && c[e] < it.X0 + 64 - R * (K - 1) && c[e] >= R && c[e] < P1 - R;
+      }
+      vec = valid[0] && valid[1] && ((reinterpret_cast<uintptr_t>(out + c[0]) & 15) == 0) && ((P1 & 1) == 0);
     }
-    const int64_t row0 = int64_t(chunk) * RDG_RC;             // first output row (interior) of the chunk
-    const int64_t col = int64_t(band) * 64 + 2 * lane;        // first output column (interior) of the lane
-    const int rows_valid = (int)std::min<int64_t>(RDG_RC, N0 - row0);
-    double* orow0 = out + (row0 + R) * P1 + R + col;
-    const bool c0ok = col < N1, c1ok = col + 1 < N1;
-    const bool vec = c1ok && ((reinterpret_cast<uintptr_t>(orow0) & 15) == 0) && ((P1 & 1) == 0);
     const double* st = reinterpret_cast<const double*>(ring + (q % RDG_NS) * G::STAGE);
-    stage_rows<R, SIG, 0>(st, lane, acc, prm, j * G::SROWS, orow0, P1, rows_valid, c0ok, c1ok, vec);
+    fused_rows<R, SIG, K, 0>(st, lane, acc, prm, it.q0 + int64_t(j) * G::SROWS, bufs, in, out, P0, P1, it, RC, c,
+                             inside, colhalo, valid, vec);
     __syncwarp();  // every lane is done with slot q % NS before it is refilled
   }
 }
@@ -255,41 +349,67 @@ int signature(const Plan& p, RdgParams& prm) {
   return SIG_FULL;
 }
 
-template <int R, int SIG, bool TMA>
+template <int R, int SIG, int K, bool TMA>
 cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
                        const RdgParams& prm) {
   using G = Geom<R>;
+  constexpr int n = 2 * R + 1;
+  constexpr int BS = 64 - 2 * R * (K - 1) - 2 * ((R * (K - 1)) & 1);
+  constexpr int BUFD = ((G::BW + 15) / 16) * 16;
+  const int smem = 128 + RDG_WARPS * (G::WARP_BYTES + 2 * (K - 1) * BUFD * 8);
   static int max_grid = 0;
   if (max_grid == 0) {
-    cudaError_t e = cudaFuncSetAttribute(rdg2d_kernel<R, SIG, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, G::SMEM);
+    cudaError_t e = cudaFuncSetAttribute(rdg2d_kernel<R, SIG, K, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
-    max_grid = persistent_grid((const void*)rdg2d_kernel<R, SIG, TMA>, RDG_WARPS * 32, G::SMEM, int64_t(1) << 40);
+    max_grid = persistent_grid((const void*)rdg2d_kernel<R, SIG, K, TMA>, RDG_WARPS * 32, smem, int64_t(1) << 40);
   }
-  const int nbands = (int)((p.N[1] + 63) / 64), nchunks = (int)((p.N[0] + RDG_RC - 1) / RDG_RC);
+  const int RC = ((RDG_RC + n - 1) / n) * n;  // chunk rows: a multiple of 2R+1 (static ring slots)
+  const int SI = (RC + 2 * K * R + G::SROWS - 1) / G::SROWS;
+  const int nbands = (int)((p.N[1] + BS - 1) / BS), nchunks = (int)((p.N[0] + RC - 1) / RC);
   const int nitems = nbands * nchunks;
   const int grid = (int)std::min<int64_t>(max_grid, (nitems + RDG_WARPS - 1) / RDG_WARPS);
-  rdg2d_kernel<R, SIG, TMA><<<grid, RDG_WARPS * 32, G::SMEM, s>>>(src, dst, p.N[0], p.N[1], nbands, nitems, map, prm);
+  rdg2d_kernel<R, SIG, K, TMA><<<grid, RDG_WARPS * 32, smem, s>>>(src, dst, p.N[0], p.N[1], nbands, nitems, RC, SI,
+                                                                   map, prm);
   return cudaGetLastError();
 }
 
-template <int R, int SIG>
+template <int R, int SIG, int K>
 cudaError_t rdg_sig(const Plan& p, const double* src, double* dst, cudaStream_t s, const RdgParams& prm) {
   using G = Geom<R>;
   CUtensorMap map;
   const int64_t padded[2] = {p.P[0], p.P[1]};
   const int box[2] = {G::SROWS, G::BW};
-  if (!p.force_no_tma && encode_tmap(&map, src, 2, padded, box)) return rdg_launch<R, SIG, true>(p, src, dst, s, map, prm);
+  if (!p.force_no_tma && encode_tmap(&map, src, 2, padded, box))
+    return rdg_launch<R, SIG, K, true>(p, src, dst, s, map, prm);
   std::memset(&map, 0, sizeof(map));
-  return rdg_launch<R, SIG, false>(p, src, dst, s, map, prm);
+  return rdg_launch<R, SIG, K, false>(p, src, dst, s, map, prm);
+}
+
+constexpr int max_fuse(int R) { return R == 1 ? 4 : (R == 2 ? 3 : 2); }
+
+template <int R, int SIG>
+cudaError_t rdg_k(const Plan& p, const double* src, double* dst, cudaStream_t s, const RdgParams& prm, int k) {
+  if constexpr (SIG == SIG_FULL) {
+    if (k != 1) return cudaErrorNotSupported;
+    return rdg_sig<R, SIG, 1>(p, src, dst, s, prm);
+  } else {
+    switch (k) {
+      case 1: return rdg_sig<R, SIG, 1>(p, src, dst, s, prm);
+      case 2: return rdg_sig<R, SIG, 2>(p, src, dst, s, prm);
+      case 3: if constexpr (max_fuse(R) >= 3) return rdg_sig<R, SIG, (max_fuse(R) >= 3 ? 3 : 1)>(p, src, dst, s, prm); break;
+      case 4: if constexpr (max_fuse(R) >= 4) return rdg_sig<R, SIG, (max_fuse(R) >= 4 ? 4 : 1)>(p, src, dst, s, prm); break;
+    }
+    return cudaErrorNotSupported;
+  }
 }
 
 template <int R>
-cudaError_t rdg_r(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+cudaError_t rdg_r(const Plan& p, const double* src, double* dst, cudaStream_t s, int k) {
   RdgParams prm;
   const int sig = signature(p, prm);
-  if (sig == SIG_PMA) return rdg_sig<R, SIG_PMA>(p, src, dst, s, prm);
-  if (sig == SIG_STAR) return rdg_sig<R, SIG_STAR>(p, src, dst, s, prm);
-  if (sig == SIG_FULL) return rdg_sig<R, SIG_FULL>(p, src, dst, s, prm);
+  if (sig == SIG_PMA) return rdg_k<R, SIG_PMA>(p, src, dst, s, prm, k);
+  if (sig == SIG_STAR) return rdg_k<R, SIG_STAR>(p, src, dst, s, prm, k);
+  if (sig == SIG_FULL) return rdg_k<R, SIG_FULL>(p, src, dst, s, prm, k);
   return cudaErrorNotSupported;
 }
 
@@ -302,13 +422,21 @@ bool rdg2d_supported(const Plan& p) {
   return signature(p, prm) >= 0;
 }
 
-cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s) {
-  if (p.ndim == 3) return launch_rdg3d(p, src, dst, s);
+int rdg2d_max_fuse(const Plan& p) {
+  if (p.ndim != 2) return 1;
+  RdgParams prm;
+  const int sig = signature(p, prm);
+  if (sig < 0 || sig == SIG_FULL) return 1;
+  return max_fuse(p.R);
+}
+
+cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s, int k) {
+  if (p.ndim == 3) return k == 1 ? launch_rdg3d(p, src, dst, s) : cudaErrorNotSupported;
   switch (p.R) {
-    case 1: return rdg_r<1>(p, src, dst, s);
-    case 2: return rdg_r<2>(p, src, dst, s);
-    case 3: return rdg_r<3>(p, src, dst, s);
-    case 4: return rdg_r<4>(p, src, dst, s);
+    case 1: return rdg_r<1>(p, src, dst, s, k);
+    case 2: return rdg_r<2>(p, src, dst, s, k);
+    case 3: return rdg_r<3>(p, src, dst, s, k);
+    case 4: return rdg_r<4>(p, src, dst, s, k);
   }
   return cudaErrorInvalidValue;
 }

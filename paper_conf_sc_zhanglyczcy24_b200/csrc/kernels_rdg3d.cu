@@ -31,13 +31,13 @@ template <int R> constexpr int BY = (R == 1 ? 4 : 2);
 constexpr int R3_ZC = 64;
 constexpr int R3_MAXK = 5;   // rank-1 terms per plane (<= 2R+1 for R <= 2)
 
-enum { PM_NONE = 0, PM_POINT = 1, PM_CHAINS = 2, PM_STAR = 3 };
+enum { PM_NONE = 0, PM_POINT = 1, PM_CHAINS = 2, PM_STAR = 3, PM_PMA1 = 4 };
 
 struct R3Params {
   int mode[5];               // per plane a0
   int K[5];                  // chain terms per plane
   int mirror[5];             // plane a0 (< R) also feeds output z = p - (2R - a0)
-  double w[5];               // PM_POINT weight (centre)
+  double w[5];               // PM_POINT weight (centre) / PM_PMA1 scalar C_{h+1}
   double u[5][R3_MAXK][5];   // plane, term, tap (centred, length 2R+1)
   double v[5][R3_MAXK][5];
 };
@@ -88,6 +88,25 @@ __device__ __forceinline__ void apply_plane(const double (&x)[BY<R> + 2 * R][2 *
       }
       d[y][0] = t0;
       d[y][1] = t1;
+    }
+  } else if (mode == PM_PMA1) {
+    // radius-1 radially symmetric plane (PMA, eq. 15): one 3x3 rank-1 chain + the centre scalar;
+    // palindromic factors: T = v0 x0 + v1 (x_-1 + x_+1)
+#pragma unroll
+    for (int y = 0; y < BY<R>; ++y) {
+      d[y][0] = P.w[A0] * x[y + R][R];
+      d[y][1] = P.w[A0] * x[y + R][R + 1];
+    }
+    double T[BY<R> + 2 * R][2];
+#pragma unroll
+    for (int r = 0; r < BY<R> + 2 * R; ++r) {
+      T[r][0] = fma(P.v[A0][0][R + 1], x[r][R - 1] + x[r][R + 1], P.v[A0][0][R] * x[r][R]);
+      T[r][1] = fma(P.v[A0][0][R + 1], x[r][R] + x[r][R + 2], P.v[A0][0][R] * x[r][R + 1]);
+    }
+#pragma unroll
+    for (int y = 0; y < BY<R>; ++y) {
+      d[y][0] = fma(P.u[A0][0][R + 1], T[y + R - 1][0] + T[y + R + 1][0], fma(P.u[A0][0][R], T[y + R][0], d[y][0]));
+      d[y][1] = fma(P.u[A0][0][R + 1], T[y + R - 1][1] + T[y + R + 1][1], fma(P.u[A0][0][R], T[y + R][1], d[y][1]));
     }
   } else {
 #pragma unroll
@@ -274,6 +293,13 @@ bool make_params3(const Plan& p, R3Params& prm) {
         for (int i = 0; i < n; ++i) { prm.v[a0][0][i] = ts[0]->v[i]; prm.u[a0][1][i] = ts[1]->u[i]; }
         continue;
       }
+    }
+    if (R == 1 && ts.size() == 2 && ts[0]->kind == kChain && ts[0]->r == 1 && ts[1]->kind == kPoint &&
+        ts[1]->r == 0 && ts[1]->u[R] == 1.0 && ts[0]->u[0] == ts[0]->u[2] && ts[0]->v[0] == ts[0]->v[2]) {
+      prm.mode[a0] = PM_PMA1;  // palindromic chain + centre scalar
+      for (int i = 0; i < n; ++i) { prm.u[a0][0][i] = ts[0]->u[i]; prm.v[a0][0][i] = ts[0]->v[i]; }
+      prm.w[a0] = ts[1]->v[R];
+      continue;
     }
     if ((int)ts.size() > R3_MAXK) return false;
     prm.mode[a0] = PM_CHAINS;

@@ -30,6 +30,16 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
 }
 
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+// Orders this thread's earlier generic-proxy shared-memory accesses before later async-proxy
+// (TMA) accesses to the same buffer.
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   asm volatile(
       "{\n"
@@ -68,6 +78,19 @@ __device__ __forceinline__ void cp_async8(void* dst, const void* src) {
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+// Boxes that start at a negative coordinate are filled by the warp with plain loads (zero
+// outside the array) and completed on the same mbarrier with a plain arrive.  (TMA itself faults
+// with "illegal instruction" when the innermost box start is not 16-byte aligned — an odd FP64
+// column — see tools/ubench/tma_probe.cu; every caller keeps that coordinate even.)
+__device__ __forceinline__ void warp_box_fill_sync(double* dst, const double* __restrict__ src, int64_t P0, int64_t P1,
+                                                   int64_t y, int64_t x, int rows, int cols, int lane) {
+  for (int i = lane; i < rows * cols; i += 32) {
+    const int r = i / cols, c = i - r * cols;
+    const int64_t gy = y + r, gx = x + c;
+    dst[i] = (gy >= 0 && gy < P0 && gx >= 0 && gx < P1) ? __ldg(src + gy * P1 + gx) : 0.0;
+  }
+}
 
 // Fallback fill of a rows x cols box at padded coordinate (y, x) of a P0 x P1 array (2D) by all
 // threads of the CTA with LDGSTS; zero outside the array.  Completion: cp_async_wait + barrier.

@@ -97,7 +97,7 @@ void factor_plane(const Mat& P, int R, int plane, double tol, std::vector<Term>&
       for (int j = k; j < n - k; ++j) {
         bool on_border = (i == k || i == n - 1 - k || j == k || j == n - 1 - k);
         if (on_border && std::fabs(Rm(i, j)) > tol) border_zero = false;
-        if (std::fabs(Rm(i, j) - Rm(n - 1 - i, j)) > tol || std::fabs(Rm(i, j) - Rm(i, n - 1 - j)) > tol) sym = false;
+        if (Rm(i, j) != Rm(n - 1 - i, j) || Rm(i, j) != Rm(i, n - 1 - j)) sym = false;  // exact: PMA factors stay exactly palindromic
       }
     if (border_zero) continue;               // ring already empty: skip it
     const double piv = Rm(k, k);
@@ -179,7 +179,10 @@ double cuda_fma_per_point(const Plan& p) {
       else f += 2.0 * (2 * t.r + 1);
     }
     (void)pma_like;
-    if (p.ndim == 3 && cnt > 0 && !(cnt == 1) && !(cnt == 2 && all_arms)) f = cnt * 2.0 * n;  // general chains
+    if (p.ndim == 3 && cnt > 0 && !(cnt == 1) && !(cnt == 2 && all_arms)) {
+      bool pma1 = p.R == 1 && cnt == 2;
+      f = pma1 ? 3.0 * 1.5 + 3.0 + 1.0 : cnt * 2.0 * n;  // PM_PMA1 (BY = 4: 6 T rows per 4 outputs) / general
+    }
     return f;
   };
   if (p.ndim == 2) {
@@ -287,7 +290,14 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
   p.fma_issued = eng == LORA_ENGINE_TC ? tc_fma_per_point(p) : eng == LORA_ENGINE_RDG_CUDA ? cuda_fma_per_point(p) : dense;
   int fk = o ? o->fuse_k : 0;
   if (fk < 0) { err = "fuse_k must be >= 0"; return LORA_ERR_INVALID_ARG; }
-  p.fuse_k = fk == 0 ? 1 : fk;
+  const int max_k = eng == LORA_ENGINE_RDG_CUDA ? rdg2d_max_fuse(p) : 1;
+  if (fk > max_k) { err = "fuse_k exceeds what the chosen engine supports for this stencil"; return LORA_ERR_UNSUPPORTED; }
+  if (fk == 0) {
+    // default fusion depth (exact temporal blocking): measured on B200
+    static const int dflt[5] = {1, 3, 2, 1, 1};  // by radius; tools/quickbench.py, gpurun_out/qb6.jsonl
+    fk = std::min(max_k, dflt[radius]);
+  }
+  p.fuse_k = fk;
   {
     const char* e = std::getenv("LORA_NO_TMA");
     p.force_no_tma = (e && e[0] == '1') ? 1 : 0;

@@ -134,3 +134,33 @@ def test_2d_staging_paths_agree(engine, shape, monkeypatch):
     b, _ = run_gpu(W, g, 3, engine=engine)
     assert np.array_equal(a, b)
     assert rel_err(a, oracle.run(W, g, 3)) <= 1e-12
+
+
+FUSE_MAX = {1: 4, 2: 3, 3: 2, 4: 2}
+
+
+@pytest.mark.parametrize("h", [1, 2, 3, 4])
+@pytest.mark.parametrize("kind", ["rsym", "star"])
+@pytest.mark.parametrize("shape", [(1, 1), (3, 5), (67, 129), (300, 200), (130, 70)])
+def test_2d_temporal_fusion_exact(h, kind, shape):
+    """Exact temporal blocking (Q5): k fused sub-steps with the halo re-imposed every
+    sub-step equal k single steps BITWISE (same per-point arithmetic) and the oracle to 1e-12,
+    for T = 1, k-1, k, k+1, 2k+1 (remainder launches) and ragged / tiny grids."""
+    W = _weights(kind, 2, h, 40 + h)
+    g = synth.grid(tuple(n + 2 * h for n in shape), 77 + h)
+    for k in range(2, FUSE_MAX[h] + 1):
+        for T in sorted({1, k - 1, k, k + 1, 2 * k + 1}):
+            a, info = run_gpu(W, g, T, engine="rdg_cuda", fuse_k=k)
+            assert info["fuse_k"] == k
+            b, _ = run_gpu(W, g, T, engine="rdg_cuda", fuse_k=1)
+            assert np.array_equal(a, b), (k, T, float(np.max(np.abs(a - b))))
+            assert rel_err(a, oracle.run(W, g, T)) <= 1e-12
+
+
+def test_fusion_staging_paths_agree(monkeypatch):
+    W = synth.rsym_weights(2, 3, 5)
+    g = synth.grid((206, 136), 11)
+    a, _ = run_gpu(W, g, 5, engine="rdg_cuda", fuse_k=2)
+    monkeypatch.setenv("LORA_NO_TMA", "1")
+    b, _ = run_gpu(W, g, 5, engine="rdg_cuda", fuse_k=2)
+    assert np.array_equal(a, b)
