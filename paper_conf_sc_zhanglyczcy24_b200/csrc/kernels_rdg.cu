@@ -144,53 +144,61 @@ __device__ __forceinline__ void row_body(const double* __restrict__ xs, int p, d
 // columns lose R valid columns per fused step at each band edge: bands overlap, stride
 // S = 64 - 2R(K-1) (minus 2 when R(K-1) is odd, so that the staged tile starts on an even column:
 // TMA faults on a box whose innermost start is not 16-byte aligned, tools/ubench/tma_probe.cu).
-struct Item {
-  int64_t X0;    // padded column of lane column 0
-  int64_t A;     // first final output row (padded)
-  int64_t q0;    // first consumed input row (padded)
+// Per-stage precomputed bookkeeping (32-bit, relative to the stage's first input row) so that the
+// unrolled row code carries no 64-bit index arithmetic.
+template <int K>
+struct StageCtx {
+  int lo, hi;               // final rows: stage-local rows I with lo <= I < hi are stored
+  int64_t ooff;             // element offset of (final row for I = 0, lane column c0)
+  int hlo[K], hhi[K];       // intermediate stage S: row I is halo if I < hlo or I >= hhi
+  int rlo[K], rhi[K];       //                     row I is inside the array if rlo <= I < rhi
+  int64_t ioff[K];          //                     element offset of (row for I = 0, column 0) in `in`
 };
 
-template <int R, int SIG, int K, int I0, int S>
+struct LaneCtx {
+  int c0;                   // padded column of the lane's first column (may be < 0)
+  bool inside0, inside1, colhalo0, colhalo1, valid0, valid1, vec;
+};
+
+template <int R, int SIG, int K, int I0, int I, int S>
 __device__ __forceinline__ void fused_stage(const double* __restrict__ src, int p, double (&acc)[K][2 * R + 1][2],
-                                            const RdgParams& P, int64_t q, double* const* __restrict__ bufs, int par,
-                                            const double* __restrict__ in, double* __restrict__ out, int64_t P0,
-                                            int64_t P1, const Item& it, int RC, const int64_t (&c)[2],
-                                            const bool (&inside)[2], const bool (&colhalo)[2], const bool (&valid)[2],
-                                            bool vec) {
+                                            const RdgParams& P, double* const* __restrict__ bufs, int par,
+                                            const double* __restrict__ in, double* __restrict__ out, int64_t P1,
+                                            const StageCtx<K>& sc, const LaneCtx& lc) {
   constexpr int n = 2 * R + 1;
   constexpr int Is = pmod(I0 - (S - 1) * R, n);   // row index mod n of stage S's input row
   row_body<R, SIG, Is>(src, p, acc[S - 1], P);
   constexpr int cs = (Is + 1) % n;                // slot of the row this stage just completed
-  const int64_t y = q - int64_t(S) * R;           // its padded row index
   double v0 = acc[S - 1][cs][0], v1 = acc[S - 1][cs][1];
   acc[S - 1][cs][0] = 0.0;
   acc[S - 1][cs][1] = 0.0;
   if constexpr (S < K) {
-    const bool row_in = y >= 0 && y < P0;
-    const bool row_halo = y < R || y >= P0 - R;
-    if (row_halo) {
-      v0 = (row_in && inside[0]) ? in[y * P1 + c[0]] : 0.0;
-      v1 = (row_in && inside[1]) ? in[y * P1 + c[1]] : 0.0;
-    } else {
-      if (colhalo[0]) v0 = in[y * P1 + c[0]];
-      if (colhalo[1]) v1 = in[y * P1 + c[1]];
-      if (!inside[0]) v0 = 0.0;
-      if (!inside[1]) v1 = 0.0;
+    // re-impose the fixed Dirichlet halo on the intermediate row (exact temporal blocking)
+    if (I < sc.hlo[S - 1] || I >= sc.hhi[S - 1]) {
+      const bool row_in = I >= sc.rlo[S - 1] && I < sc.rhi[S - 1];
+      const double* ir = in + sc.ioff[S - 1] + int64_t(I) * P1 + lc.c0;
+      v0 = (row_in && lc.inside0) ? ir[0] : 0.0;
+      v1 = (row_in && lc.inside1) ? ir[1] : 0.0;
+    } else if (lc.colhalo0 | lc.colhalo1 | !lc.inside0 | !lc.inside1) {
+      const double* ir = in + sc.ioff[S - 1] + int64_t(I) * P1 + lc.c0;
+      if (lc.colhalo0) v0 = ir[0];
+      if (lc.colhalo1) v1 = ir[1];
+      if (!lc.inside0) v0 = 0.0;
+      if (!lc.inside1) v1 = 0.0;
     }
     double* b = bufs[2 * (S - 1) + par];
     b[R + 2 * p] = v0;
     b[R + 2 * p + 1] = v1;
     __syncwarp();
-    fused_stage<R, SIG, K, I0, S + 1>(b, p, acc, P, q, bufs, par, in, out, P0, P1, it, RC, c, inside, colhalo, valid,
-                                      vec);
+    fused_stage<R, SIG, K, I0, I, S + 1>(b, p, acc, P, bufs, par, in, out, P1, sc, lc);
   } else {
-    if (y >= it.A && y < it.A + RC && y < P0 - R) {
-      double* o = out + y * P1;
-      if (vec) {
-        *reinterpret_cast<double2*>(o + c[0]) = make_double2(v0, v1);
+    if (I >= sc.lo && I < sc.hi) {
+      double* o = out + sc.ooff + int64_t(I) * P1;
+      if (lc.vec) {
+        *reinterpret_cast<double2*>(o) = make_double2(v0, v1);
       } else {
-        if (valid[0]) o[c[0]] = v0;
-        if (valid[1]) o[c[1]] = v1;
+        if (lc.valid0) o[0] = v0;
+        if (lc.valid1) o[1] = v1;
       }
     }
   }
@@ -198,18 +206,15 @@ __device__ __forceinline__ void fused_stage(const double* __restrict__ src, int 
 
 template <int R, int SIG, int K, int I>
 __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p, double (&acc)[K][2 * R + 1][2],
-                                           const RdgParams& P, int64_t qbase, double* const* __restrict__ bufs,
-                                           const double* __restrict__ in, double* __restrict__ out, int64_t P0,
-                                           int64_t P1, const Item& it, int RC, const int64_t (&c)[2],
-                                           const bool (&inside)[2], const bool (&colhalo)[2], const bool (&valid)[2],
-                                           bool vec) {
+                                           const RdgParams& P, double* const* __restrict__ bufs,
+                                           const double* __restrict__ in, double* __restrict__ out, int64_t P1,
+                                           const StageCtx<K>& sc, const LaneCtx& lc, int par0) {
   constexpr int n = 2 * R + 1;
   if constexpr (I < Geom<R>::SROWS) {
     constexpr int OFF = pmod(R - K * R, n);  // q0 mod n (RC is a multiple of n)
-    const int64_t q = qbase + I;
-    fused_stage<R, SIG, K, pmod(I + OFF, n), 1>(st + I * Geom<R>::BW, p, acc, P, q, bufs, (int)(q & 1), in, out, P0,
-                                                P1, it, RC, c, inside, colhalo, valid, vec);
-    fused_rows<R, SIG, K, I + 1>(st, p, acc, P, qbase, bufs, in, out, P0, P1, it, RC, c, inside, colhalo, valid, vec);
+    fused_stage<R, SIG, K, pmod(I + OFF, n), I, 1>(st + I * Geom<R>::BW, p, acc, P, bufs, (par0 + I) & 1, in, out, P1,
+                                                   sc, lc);
+    fused_rows<R, SIG, K, I + 1>(st, p, acc, P, bufs, in, out, P1, sc, lc, par0);
   }
 }
 
@@ -232,7 +237,8 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (K == 1 ? 4 : 3)) rdg2d_kernel
 #pragma unroll
   for (int i = 0; i < 2 * (K - 1); ++i) bufs[i] = bufmem + i * BUFD;
   for (int i = lane; i < 2 * (K - 1) * BUFD; i += 32) bufmem[i] = 0.0;  // margins stay zero
-  const int64_t P1 = N1 + 2 * R, P0 = N0 + 2 * R;
+  const int64_t P1 = N1 + 2 * R;
+  const int P0 = (int)(N0 + 2 * R);
   const int gw = blockIdx.x * RDG_WARPS + wl, TW = gridDim.x * RDG_WARPS;
   const int my_items = gw < nitems ? (nitems - 1 - gw) / TW + 1 : 0;
   const int nstages = my_items * SI;
@@ -241,28 +247,27 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (K == 1 ? 4 : 3)) rdg2d_kernel
     fence_barrier_init();
   }
   __syncwarp();
-  auto item_of = [&](int q) {
-    const int item = gw + (q / SI) * TW;
+  // item geometry: band b -> lane column 0 at padded column X0; chunk c -> final rows from A
+  auto geom = [&](int item, int& X0, int& A) {
     const int band = item % nbands, chunk = item / nbands;
-    Item it;
-    it.X0 = R + int64_t(band) * BS - int64_t(R) * (K - 1) - SG;
-    it.A = R + int64_t(chunk) * RC;
-    it.q0 = it.A - int64_t(K) * R;
-    return it;
+    X0 = R + band * BS - R * (K - 1) - SG;
+    A = R + chunk * RC;
   };
-  auto issue = [&](int q) {  // stage q of this warp's sequence into slot q % NS
-    const Item it = item_of(q);
-    const int64_t y = it.q0 + int64_t(q % SI) * G::SROWS, x = it.X0 - R;
-    double* dst = reinterpret_cast<double*>(ring + (q % RDG_NS) * G::STAGE);
+  // producer position (next stage to stage into the ring)
+  int pitem = gw, pj = 0, pX0 = 0, pA = 0;
+  if (gw < nitems) geom(pitem, pX0, pA);
+  auto issue_next = [&](int slot) {
+    const int x = pX0 - R, y = pA - K * R + pj * G::SROWS;
+    double* dst = reinterpret_cast<double*>(ring + slot * G::STAGE);
     if constexpr (TMA) {
       if (x < 0 || y < 0) {  // first band / chunk of a fused launch: no TMA for negative boxes
         warp_box_fill_sync(dst, in, P0, P1, y, x, G::SROWS, G::BW, lane);
         __syncwarp();
-        if (lane == 0) mbar_arrive(&bars[q % RDG_NS]);
+        if (lane == 0) mbar_arrive(&bars[slot]);
       } else if (lane == 0) {
         fence_proxy_async();
-        mbar_arrive_expect_tx(&bars[q % RDG_NS], G::SROWS * G::BW * 8);
-        tma_load_2d(dst, &tmap, (int)x, (int)y, &bars[q % RDG_NS]);
+        mbar_arrive_expect_tx(&bars[slot], G::SROWS * G::BW * 8);
+        tma_load_2d(dst, &tmap, x, y, &bars[slot]);
       }
     } else {
       for (int i = lane; i < G::SROWS * G::BW; i += 32) {
@@ -273,45 +278,69 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (K == 1 ? 4 : 3)) rdg2d_kernel
       }
       cp_async_commit();
     }
+    if (++pj == SI) {
+      pj = 0;
+      pitem += TW;
+      if (pitem < nitems) geom(pitem, pX0, pA);
+    }
   };
   for (int q = 0; q < RDG_NS - 1; ++q) {
-    if (q < nstages) issue(q);
+    if (q < nstages) issue_next(q);
     else if constexpr (!TMA) cp_async_commit();  // empty group: keeps wait_group<NS-1> exact
   }
   double acc[K][2 * R + 1][2];
-  Item it{};
-  int64_t c[2] = {0, 0};
-  bool inside[2] = {false, false}, colhalo[2] = {false, false}, valid[2] = {false, false};
-  bool vec = false;
+  LaneCtx lc{};
+  StageCtx<K> sc{};
+  int citem = gw, cj = 0, X0 = 0, A = 0, rows_valid_end = 0;
+  int slot = 0, phase = 0;
   for (int q = 0; q < nstages; ++q) {
-    if (q + RDG_NS - 1 < nstages) issue(q + RDG_NS - 1);
+    if (q + RDG_NS - 1 < nstages) issue_next((slot + RDG_NS - 1) % RDG_NS);
     else if constexpr (!TMA) cp_async_commit();  // keep the group count uniform
     if constexpr (TMA) {
-      mbar_wait(&bars[q % RDG_NS], (q / RDG_NS) & 1);
+      mbar_wait(&bars[slot], phase);
     } else {
       cp_async_wait<RDG_NS - 1>();
       __syncwarp();
     }
-    const int j = q % SI;
-    if (j == 0) {
-      it = item_of(q);
+    if (cj == 0) {
+      geom(citem, X0, A);
 #pragma unroll
       for (int k = 0; k < K; ++k)
 #pragma unroll
         for (int s = 0; s < 2 * R + 1; ++s) { acc[k][s][0] = 0.0; acc[k][s][1] = 0.0; }
-#pragma unroll
-      for (int e = 0; e < 2; ++e) {
-        c[e] = it.X0 + 2 * lane + e;
-        inside[e] = c[e] >= 0 && c[e] < P1;
-        colhalo[e] = inside[e] && (c[e] < R || c[e] >= P1 - R);
-        valid[e] = c[e] >= it.X0 + R * (K - 1) && c[e] < it.X0 + 64 - R * (K - 1) && c[e] >= R && c[e] < P1 - R;
-      }
-      vec = valid[0] && valid[1] && ((reinterpret_cast<uintptr_t>(out + c[0]) & 15) == 0) && ((P1 & 1) == 0);
+      const int c0 = X0 + 2 * lane, c1 = c0 + 1;
+      lc.c0 = c0;
+      lc.inside0 = c0 >= 0 && c0 < P1;
+      lc.inside1 = c1 >= 0 && c1 < P1;
+      lc.colhalo0 = lc.inside0 && (c0 < R || c0 >= P1 - R);
+      lc.colhalo1 = lc.inside1 && (c1 < R || c1 >= P1 - R);
+      lc.valid0 = c0 >= X0 + R * (K - 1) && c0 < X0 + 64 - R * (K - 1) && c0 >= R && c0 < P1 - R;
+      lc.valid1 = c1 >= X0 + R * (K - 1) && c1 < X0 + 64 - R * (K - 1) && c1 >= R && c1 < P1 - R;
+      lc.vec = lc.valid0 && lc.valid1 && ((reinterpret_cast<uintptr_t>(out + c0) & 15) == 0) && ((P1 & 1) == 0);
+      rows_valid_end = min(A + RC, P0 - R);
     }
-    const double* st = reinterpret_cast<const double*>(ring + (q % RDG_NS) * G::STAGE);
-    fused_rows<R, SIG, K, 0>(st, lane, acc, prm, it.q0 + int64_t(j) * G::SROWS, bufs, in, out, P0, P1, it, RC, c,
-                             inside, colhalo, valid, vec);
-    __syncwarp();  // every lane is done with slot q % NS before it is refilled
+    // stage bookkeeping: input row I of this stage is padded row yb + I
+    const int yb = A - K * R + cj * G::SROWS;
+    {
+      const int yf = yb - K * R;  // final row produced by input row I = 0
+      sc.lo = A - yf;
+      sc.hi = rows_valid_end - yf;
+      sc.ooff = int64_t(yf) * P1 + lc.c0;
+#pragma unroll
+      for (int S = 1; S < K; ++S) {
+        const int ys = yb - S * R;  // stage-S row produced by input row I = 0
+        sc.hlo[S - 1] = R - ys;
+        sc.hhi[S - 1] = P0 - R - ys;
+        sc.rlo[S - 1] = -ys;
+        sc.rhi[S - 1] = P0 - ys;
+        sc.ioff[S - 1] = int64_t(ys) * P1;
+      }
+    }
+    const double* st = reinterpret_cast<const double*>(ring + slot * G::STAGE);
+    fused_rows<R, SIG, K, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1);
+    __syncwarp();  // every lane is done with this slot before it is refilled
+    if (++slot == RDG_NS) { slot = 0; phase ^= 1; }
+    if (++cj == SI) { cj = 0; citem += TW; }
   }
 }
 

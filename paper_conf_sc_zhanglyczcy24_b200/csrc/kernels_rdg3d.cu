@@ -170,7 +170,8 @@ __global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* _
   const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw) + wl * R3_NS;
   unsigned char* ring = smem_raw + 128 + wl * G::WARP_BYTES;
-  const int64_t P0 = N0 + 2 * R, P1 = N1 + 2 * R, P2 = N2 + 2 * R;
+  const int P0 = (int)(N0 + 2 * R);
+  const int64_t P1 = N1 + 2 * R, P2 = N2 + 2 * R;
   const int gw = blockIdx.x * R3_WARPS + wl, TW = gridDim.x * R3_WARPS;
   const int my_items = gw < nitems ? (nitems - 1 - gw) / TW + 1 : 0;
   const int nstages = my_items * G::SI;
@@ -179,60 +180,81 @@ __global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* _
     fence_barrier_init();
   }
   __syncwarp();
-  auto coords = [&](int q, int64_t& z, int64_t& y, int64_t& x) {
-    const int item = gw + (q / G::SI) * TW, j = q % G::SI;
+  // item -> (x band, y block, z chunk); producer and consumer walk their stage sequences with
+  // incremental counters (one division set per item, none per plane)
+  auto geom = [&](int item, int& bx0, int& by0, int& bz0) {
     const int bx = item % nbx, rest = item / nbx, by = rest % nby, bz = rest / nby;
-    z = int64_t(bz) * R3_ZC + j;         // padded input plane
-    y = int64_t(by) * BY<R>;             // padded row of the tile origin
-    x = int64_t(bx) * 64;
+    bx0 = bx * 64;           // padded column of the staged tile origin (= interior column of lane col 0)
+    by0 = by * BY<R>;        // padded row of the staged tile origin (= interior row of output row 0)
+    bz0 = bz * R3_ZC;        // first padded input plane (= first interior output plane) of the chunk
   };
-  auto issue = [&](int q) {
-    int64_t z, y, x;
-    coords(q, z, y, x);
-    double* dst = reinterpret_cast<double*>(ring + (q % R3_NS) * G::STAGE);
+  int pitem = gw, pj = 0, px = 0, py = 0, pz = 0;
+  if (gw < nitems) geom(pitem, px, py, pz);
+  auto issue_next = [&](int slot) {
+    double* dst = reinterpret_cast<double*>(ring + slot * G::STAGE);
+    const int z = pz + pj;
     if constexpr (TMA) {
       if (lane == 0) {
-        mbar_arrive_expect_tx(&bars[q % R3_NS], G::ROWS * G::BW * 8);
-        tma_load_3d(dst, &tmap, (int)x, (int)y, (int)z, &bars[q % R3_NS]);
+        fence_proxy_async();
+        mbar_arrive_expect_tx(&bars[slot], G::ROWS * G::BW * 8);
+        tma_load_3d(dst, &tmap, px, py, z, &bars[slot]);
       }
     } else {
       for (int i = lane; i < G::ROWS * G::BW; i += 32) {
         const int r = i / G::BW, c = i - r * G::BW;
-        const int64_t gy = y + r, gx = x + c;
-        if (z < P0 && gy < P1 && gx < P2) cp_async8(dst + i, in + (z * P1 + gy) * P2 + gx);
+        const int64_t gy = py + r, gx = px + c;
+        if (z < P0 && gy < P1 && gx < P2) cp_async8(dst + i, in + (int64_t(z) * P1 + gy) * P2 + gx);
         else dst[i] = 0.0;
       }
       cp_async_commit();
     }
+    if (++pj == G::SI) {
+      pj = 0;
+      pitem += TW;
+      if (pitem < nitems) geom(pitem, px, py, pz);
+    }
   };
   for (int q = 0; q < R3_NS - 1; ++q) {
-    if (q < nstages) issue(q);
+    if (q < nstages) issue_next(q);
     else if constexpr (!TMA) cp_async_commit();
   }
   double acc[n][BY<R>][2];
+  int citem = gw, cj = 0, slot = 0, phase = 0;
+  int cz = 0, zend = 0, rowmask = 0;
+  double* obase = out;
+  bool c0ok = false, c1ok = false, vec = false;
   // consumer: stages in groups of n so that the ring slot of every plane offset is static
   for (int q0 = 0; q0 < nstages; q0 += n) {
     auto one = [&](auto Ic) {
       constexpr int I = decltype(Ic)::value;
       const int q = q0 + I;
-      if (q + R3_NS - 1 < nstages) issue(q + R3_NS - 1);
+      if (q + R3_NS - 1 < nstages) issue_next((slot + R3_NS - 1) % R3_NS);
       else if constexpr (!TMA) cp_async_commit();
       if constexpr (TMA) {
-        mbar_wait(&bars[q % R3_NS], (q / R3_NS) & 1);
+        mbar_wait(&bars[slot], phase);
       } else {
         cp_async_wait<R3_NS - 1>();
         __syncwarp();
       }
-      int64_t zp, y0, x0;
-      coords(q, zp, y0, x0);
-      const int j = q % G::SI;
-      if (j == 0) {
+      if (cj == 0) {
+        int bx0, by0, bz0;
+        geom(citem, bx0, by0, bz0);
 #pragma unroll
         for (int s = 0; s < n; ++s)
 #pragma unroll
           for (int y = 0; y < BY<R>; ++y) { acc[s][y][0] = 0.0; acc[s][y][1] = 0.0; }
+        const int col = bx0 + 2 * lane;
+        c0ok = col < N2;
+        c1ok = col + 1 < N2;
+        cz = bz0;
+        zend = (int)(int64_t(bz0) + R3_ZC < N0 ? int64_t(bz0) + R3_ZC : N0);
+        rowmask = 0;
+#pragma unroll
+        for (int y = 0; y < BY<R>; ++y) rowmask |= (by0 + y < N1) ? (1 << y) : 0;
+        obase = out + (int64_t(R) * P1 + by0 + R) * P2 + R + col;   // (interior z = 0, row by0, column col)
+        vec = c0ok && c1ok && ((reinterpret_cast<uintptr_t>(obase) & 15) == 0) && ((P2 & 1) == 0);
       }
-      const double* st = reinterpret_cast<const double*>(ring + (q % R3_NS) * G::STAGE);
+      const double* st = reinterpret_cast<const double*>(ring + slot * G::STAGE);
       double x[BY<R> + 2 * R][2 * R + 2];
 #pragma unroll
       for (int r = 0; r < BY<R> + 2 * R; ++r)
@@ -244,24 +266,27 @@ __global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* _
         }
       __syncwarp();  // slot consumed
       apply_all<R, 0, I>(x, acc, prm);
-      // output plane zi = zp - 2R (interior index) is complete: slot (I - 2R) mod n == (I + 1) mod n
+      // output plane zi = (input plane) - 2R is complete: slot (I - 2R) mod n == (I + 1) mod n
       constexpr int s = (I + 1) % n;
-      const int64_t zi = zp - 2 * R;
-      const int64_t zc0 = zp - j;  // first interior output plane of the chunk
-      if (zi >= zc0 && zi < zc0 + R3_ZC && zi < N0) {
-        const int64_t col = x0 + 2 * lane;
+      const int zi = cz + cj - 2 * R;
+      if (cj >= 2 * R && zi < zend) {
+        double* o = obase + int64_t(zi) * P1 * P2;
 #pragma unroll
         for (int y = 0; y < BY<R>; ++y) {
-          const int64_t gy = y0 + y;
-          if (gy < N1) {
-            double* o = out + ((zi + R) * P1 + gy + R) * P2 + R + col;
-            if (col < N2) o[0] = acc[s][y][0];
-            if (col + 1 < N2) o[1] = acc[s][y][1];
+          if (rowmask & (1 << y)) {
+            if (vec) {
+              *reinterpret_cast<double2*>(o + int64_t(y) * P2) = make_double2(acc[s][y][0], acc[s][y][1]);
+            } else {
+              if (c0ok) o[int64_t(y) * P2] = acc[s][y][0];
+              if (c1ok) o[int64_t(y) * P2 + 1] = acc[s][y][1];
+            }
           }
         }
       }
 #pragma unroll
       for (int y = 0; y < BY<R>; ++y) { acc[s][y][0] = 0.0; acc[s][y][1] = 0.0; }
+      if (++slot == R3_NS) { slot = 0; phase ^= 1; }
+      if (++cj == G::SI) { cj = 0; citem += TW; }
     };
     [&]<int... Is>(std::integer_sequence<int, Is...>) {
       (one(std::integral_constant<int, Is>{}), ...);
