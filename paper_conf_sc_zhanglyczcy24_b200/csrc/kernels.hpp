@@ -24,6 +24,10 @@ int rdg2d_max_fuse(const Plan& p);
 // K2 on CUDA cores (3D, Alg. 2 with RDG per plane), one step.
 cudaError_t launch_rdg3d(const Plan& p, const double* src, double* dst, cudaStream_t s);
 
+// K2 on tensor cores (3D, Alg. 2 with DMMA chains per plane, point-wise planes on DFMA), R = 1.
+cudaError_t launch_tc3d(const Plan& p, const double* src, double* dst, cudaStream_t s);
+bool tc3d_supported(const Plan& p);
+
 bool tc2d_supported(const Plan& p);
 bool rdg3d_supported(const Plan& p);
 bool rdg2d_supported(const Plan& p);

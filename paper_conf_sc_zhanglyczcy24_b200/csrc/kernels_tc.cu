@@ -26,163 +26,12 @@
 
 #include "kernels.hpp"
 #include "pipe.cuh"
+#include "tc_terms.cuh"
 
 namespace lora {
 namespace {
 
-constexpr int TC_MAXT = 16;
-struct TcTerm {
-  int kind, r, ic, jc;     // kind: 0 chain, 1 horizontal arm, 2 vertical arm, 3 point
-  double u[kMaxN], v[kMaxN];
-};
-struct TcParams {
-  int nterms;
-  TcTerm t[TC_MAXT];
-};
-
-constexpr int TC_BM = 64, TC_BN = 64, TC_PITCH = 76;
-
-__device__ __forceinline__ void dmma(double (&c)[2], double a, double b) {
-  asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
-               : "+d"(c[0]), "+d"(c[1])
-               : "d"(a), "d"(b));
-}
-
-template <int R>
-__host__ __device__ constexpr int tc_rows() { return TC_BM + 2 * R + 4; }
-
-// u/v are centred length 2R+1; a term of radius HR lives in [R-HR, R+HR].
-template <int R, int HR>
-__device__ __forceinline__ void chain_term(const double* __restrict__ X, int w, int g, int t, const TcTerm& tm,
-                                           double (&P)[8][2]) {
-  constexpr int K1 = ((8 + 2 * HR + 3) / 4) * 4, KS = K1 / 4;
-  constexpr int o = R - HR;
-  double a[KS];
-#pragma unroll
-  for (int kk = 0; kk < KS; ++kk) {
-    const int j = 4 * kk + t - g;
-    a[kk] = (j >= 0 && j <= 2 * HR) ? tm.u[o + j] : 0.0;
-  }
-  double T[9][2];
-#pragma unroll
-  for (int nb = 0; nb < 9; ++nb) { T[nb][0] = 0.0; T[nb][1] = 0.0; }
-  const double* xr = X + (8 * w + o + t) * TC_PITCH + g;
-#pragma unroll
-  for (int kk = 0; kk < KS; ++kk) {
-#pragma unroll
-    for (int nb = 0; nb < 9; ++nb) dmma(T[nb], a[kk], xr[4 * kk * TC_PITCH + 8 * nb]);
-  }
-  double vb[2][2];
-#pragma unroll
-  for (int j = 0; j < 2; ++j)
-#pragma unroll
-    for (int i = 0; i < 2; ++i) {
-      const int c = 8 * j + 2 * t + i - g;
-      vb[j][i] = (c >= 0 && c <= 2 * R) ? tm.v[c] : 0.0;
-    }
-#pragma unroll
-  for (int ob = 0; ob < 8; ++ob) {
-    dmma(P[ob], T[ob][0], vb[0][0]);
-    dmma(P[ob], T[ob][1], vb[0][1]);
-    dmma(P[ob], T[ob + 1][0], vb[1][0]);
-    dmma(P[ob], T[ob + 1][1], vb[1][1]);
-  }
-}
-
-// Horizontal arm (u = e_R): P[g][n] += sum_c X[8w+g+R][8ob+c] v[c-n]; A from smem, B = band of v.
-template <int R, int HR>
-__device__ __forceinline__ void harm_term(const double* __restrict__ X, int w, int g, int t, const TcTerm& tm,
-                                          double (&P)[8][2]) {
-  constexpr int K = ((8 + 2 * HR + 3) / 4) * 4, KS = K / 4;
-  constexpr int o = R - HR;
-  double b[KS];
-#pragma unroll
-  for (int kk = 0; kk < KS; ++kk) {
-    const int j = 4 * kk + t - g;
-    b[kk] = (j >= 0 && j <= 2 * HR) ? tm.v[o + j] : 0.0;
-  }
-  const double* xr = X + (8 * w + g + R) * TC_PITCH + o + t;
-#pragma unroll
-  for (int ob = 0; ob < 8; ++ob)
-#pragma unroll
-    for (int kk = 0; kk < KS; ++kk) dmma(P[ob], xr[8 * ob + 4 * kk], b[kk]);
-}
-
-// Vertical arm (v = e_R): P[g][n] += sum_k U[g][k] X[8w+o+k][8ob+n+R].
-template <int R, int HR>
-__device__ __forceinline__ void varm_term(const double* __restrict__ X, int w, int g, int t, const TcTerm& tm,
-                                          double (&P)[8][2]) {
-  constexpr int K1 = ((8 + 2 * HR + 3) / 4) * 4, KS = K1 / 4;
-  constexpr int o = R - HR;
-  double a[KS];
-#pragma unroll
-  for (int kk = 0; kk < KS; ++kk) {
-    const int j = 4 * kk + t - g;
-    a[kk] = (j >= 0 && j <= 2 * HR) ? tm.u[o + j] : 0.0;
-  }
-  const double* xr = X + (8 * w + o + t) * TC_PITCH + g + R;
-#pragma unroll
-  for (int ob = 0; ob < 8; ++ob)
-#pragma unroll
-    for (int kk = 0; kk < KS; ++kk) dmma(P[ob], a[kk], xr[4 * kk * TC_PITCH + 8 * ob]);
-}
-
-template <int R>
-__device__ __forceinline__ void point_term(const double* __restrict__ X, int w, int g, int t, const TcTerm& tm,
-                                           double (&P)[8][2]) {
-  const double wgt = tm.v[tm.jc];
-  const double* xr = X + (8 * w + g + tm.ic) * TC_PITCH + 2 * t + tm.jc;
-#pragma unroll
-  for (int ob = 0; ob < 8; ++ob) {
-    P[ob][0] = fma(wgt, xr[8 * ob], P[ob][0]);
-    P[ob][1] = fma(wgt, xr[8 * ob + 1], P[ob][1]);
-  }
-}
-
-
-template <int R>
-__device__ __forceinline__ void tc_tile(const double* __restrict__ X, int w, int g, int t, const TcParams& prm,
-                                        double (&P)[8][2]) {
-#pragma unroll
-  for (int ob = 0; ob < 8; ++ob) { P[ob][0] = 0.0; P[ob][1] = 0.0; }
-  for (int k = 0; k < prm.nterms; ++k) {
-    const TcTerm& tm = prm.t[k];
-    switch (tm.kind) {
-      case 0:
-        if (tm.r == 1) chain_term<R, 1>(X, w, g, t, tm, P);
-        else if constexpr (R >= 2) {
-          if (tm.r == 2) chain_term<R, (R >= 2 ? 2 : 1)>(X, w, g, t, tm, P);
-          else if constexpr (R >= 3) {
-            if (tm.r == 3) chain_term<R, (R >= 3 ? 3 : 1)>(X, w, g, t, tm, P);
-            else if constexpr (R >= 4) chain_term<R, 4>(X, w, g, t, tm, P);
-          }
-        }
-        break;
-      case 1:
-        if (tm.r <= 1) harm_term<R, 1>(X, w, g, t, tm, P);
-        else if constexpr (R >= 2) {
-          if (tm.r == 2) harm_term<R, (R >= 2 ? 2 : 1)>(X, w, g, t, tm, P);
-          else if constexpr (R >= 3) {
-            if (tm.r == 3) harm_term<R, (R >= 3 ? 3 : 1)>(X, w, g, t, tm, P);
-            else if constexpr (R >= 4) harm_term<R, 4>(X, w, g, t, tm, P);
-          }
-        }
-        break;
-      case 2:
-        if (tm.r <= 1) varm_term<R, 1>(X, w, g, t, tm, P);
-        else if constexpr (R >= 2) {
-          if (tm.r == 2) varm_term<R, (R >= 2 ? 2 : 1)>(X, w, g, t, tm, P);
-          else if constexpr (R >= 3) {
-            if (tm.r == 3) varm_term<R, (R >= 3 ? 3 : 1)>(X, w, g, t, tm, P);
-            else if constexpr (R >= 4) varm_term<R, 4>(X, w, g, t, tm, P);
-          }
-        }
-        break;
-      default:
-        point_term<R>(X, w, g, t, tm, P);
-    }
-  }
-}
+using namespace tc;
 
 // Persistent CTAs walk the 64x64 output tiles; tile i+1 is staged (TMA + mbarrier, or LDGSTS when
 // TMA's 16-byte pitch rule fails) while tile i is computed.
@@ -305,9 +154,13 @@ cudaError_t tc_r(const Plan& p, const double* src, double* dst, cudaStream_t s) 
 
 }  // namespace
 
-bool tc2d_supported(const Plan& p) { return p.ndim == 2 && (int)p.terms.size() <= TC_MAXT; }
+bool tc2d_supported(const Plan& p) {
+  if (p.ndim == 3) return tc3d_supported(p);
+  return p.ndim == 2 && (int)p.terms.size() <= TC_MAXT;
+}
 
 cudaError_t launch_tc2d(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  if (p.ndim == 3) return launch_tc3d(p, src, dst, s);
   if (!tc2d_supported(p)) return cudaErrorInvalidValue;
   switch (p.R) {
     case 1: return tc_r<1>(p, src, dst, s);

@@ -149,13 +149,28 @@ void factor_plane(const Mat& P, int R, int plane, double tol, std::vector<Term>&
 // point-wise terms are 1 DFMA.
 double tc_fma_per_point(const Plan& p) {
   const double BN = 64.0;
-  double f = 0;
-  for (const Term& t : p.terms) {
+  const int n = 2 * p.R + 1;
+  auto term_cost = [&](const Term& t) {
     const int r = t.r;
     const double K = 4.0 * std::ceil((8.0 + 2 * r) / 4.0);
-    if (t.kind == kPoint) f += 1;
-    else if (t.kind == kArm) f += K;
-    else f += K * (8.0 * std::ceil((BN + 2 * r) / 8.0)) / BN + 16.0;
+    if (t.kind == kPoint) return 1.0;
+    if (t.kind == kArm) return K;
+    return K * (8.0 * std::ceil((BN + 2 * r) / 8.0)) / BN + 16.0;
+  };
+  double f = 0;
+  const int nplanes = p.ndim == 2 ? 1 : n;
+  for (int q = 0; q < nplanes; ++q) {
+    bool mirrored = false;
+    if (p.ndim == 3 && q > p.R) {  // kernels_tc3d.cu computes a z-symmetric plane pair once
+      mirrored = true;
+      for (int e = 0; e < n * n; ++e)
+        if (p.W[size_t(q) * n * n + e] != p.W[size_t(2 * p.R - q) * n * n + e]) { mirrored = false; break; }
+    }
+    if (mirrored) { f += 1; continue; }
+    double fp = 0;
+    for (const Term& t : p.terms)
+      if (t.plane == q) fp += term_cost(t);
+    f += fp + (p.ndim == 3 && fp > 0 ? 1 : 0);  // + the add of the plane result into its output plane
   }
   return f;
 }

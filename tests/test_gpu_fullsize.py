@@ -27,8 +27,6 @@ def test_fullsize_sampled_parity(name, engine):
     import torch
     import paper_conf_sc_zhanglyczcy24_b200 as L
     W, c = synth.config(name)
-    if engine == "tc" and c["ndim"] == 3:
-        pytest.skip("tensor-core engine is 2D")
     g = synth.grid(c["padded"], c["seed"])
     st = L.Stencil(W, c["shape"], engine=engine)
     x = torch.from_numpy(g).cuda()
