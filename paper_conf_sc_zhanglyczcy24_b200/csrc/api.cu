@@ -53,20 +53,13 @@ int copy_halo_launch(const Plan& p, const double* in, double* dst, void* stream)
   return (int)launch_copy_halo(p, in, dst, static_cast<cudaStream_t>(stream));
 }
 
-int run_device(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s) {
-  const size_t bytes = p.elems * sizeof(double);
-  if (T == 0) {
-    cudaError_t e = cudaMemcpyAsync(out, in, bytes, cudaMemcpyDeviceToDevice, s);
-    return e == cudaSuccess ? LORA_OK : cuda_fail(e, "cudaMemcpyAsync");
-  }
-  const bool two = (T + (p.fuse_k < 1 ? 1 : p.fuse_k) - 1) / (p.fuse_k < 1 ? 1 : p.fuse_k) >= 2;
-  int rc = ensure_device(p, two);
-  if (rc) return rc;
+// Enqueues the whole time loop on stream s (no synchronisation).
+cudaError_t enqueue(Plan& p, const double* in, double* out, int64_t T, bool two, cudaStream_t s) {
   cudaError_t e = launch_copy_halo(p, in, out, s);
-  if (e != cudaSuccess) return cuda_fail(e, "copy_halo launch");
+  if (e != cudaSuccess) return e;
   if (two) {
     e = launch_copy_halo(p, in, p.scratch, s);
-    if (e != cudaSuccess) return cuda_fail(e, "copy_halo launch");
+    if (e != cudaSuccess) return e;
   }
   // ceil(T / k) launches of k fused steps (the last one takes the remainder); launch i writes
   // `out` when (L - 1 - i) is even, else the scratch buffer, so the last lands in `out`.
@@ -77,8 +70,62 @@ int run_device(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s
     const int64_t steps = (i == L - 1) ? T - k * (L - 1) : k;
     double* dst = ((L - 1 - i) % 2 == 0) ? out : p.scratch;
     e = step(p, src, dst, s, (int)steps);
-    if (e != cudaSuccess) return cuda_fail(e, "stencil kernel launch");
+    if (e != cudaSuccess) return e;
     src = dst;
+  }
+  return cudaSuccess;
+}
+
+// Launch-bound problems (small grids, many launches) replay the time loop as a CUDA graph: the
+// second identical call (same in, out, T, stream) captures it, later identical calls replay it.
+bool use_graph(const Plan& p, int64_t launches, cudaStream_t s) {
+  static int off = [] { const char* e = std::getenv("LORA_NO_GRAPH"); return e && e[0] == '1' ? 1 : 0; }();
+  // the legacy / per-thread default streams cannot be captured
+  if (s == nullptr || s == cudaStreamLegacy || s == cudaStreamPerThread) return false;
+  return !off && launches >= 4 && p.elems <= (size_t(1) << 22);
+}
+
+int run_device(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s) {
+  const size_t bytes = p.elems * sizeof(double);
+  if (T == 0) {
+    cudaError_t e = cudaMemcpyAsync(out, in, bytes, cudaMemcpyDeviceToDevice, s);
+    return e == cudaSuccess ? LORA_OK : cuda_fail(e, "cudaMemcpyAsync");
+  }
+  const int64_t k = p.fuse_k < 1 ? 1 : p.fuse_k;
+  const int64_t L = (T + k - 1) / k;
+  const bool two = L >= 2;
+  int rc = ensure_device(p, two);
+  if (rc) return rc;
+  cudaError_t e;
+  if (use_graph(p, L, s)) {
+    const bool same = p.g_in == in && p.g_out == out && p.g_T == T && p.g_stream == (void*)s;
+    if (same && p.graph_exec) {
+      e = cudaGraphLaunch(static_cast<cudaGraphExec_t>(p.graph_exec), s);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaGraphLaunch");
+    } else if (same) {  // second identical call: capture, instantiate, launch
+      cudaGraph_t g = nullptr;
+      e = cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaStreamBeginCapture");
+      cudaError_t le = enqueue(p, in, out, T, two, s);
+      e = cudaStreamEndCapture(s, &g);
+      if (le != cudaSuccess) { if (g) cudaGraphDestroy(g); return cuda_fail(le, "stencil kernel launch (capture)"); }
+      if (e != cudaSuccess) return cuda_fail(e, "cudaStreamEndCapture");
+      cudaGraphExec_t ex = nullptr;
+      e = cudaGraphInstantiate(&ex, g, 0);
+      cudaGraphDestroy(g);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaGraphInstantiate");
+      p.graph_exec = ex;
+      e = cudaGraphLaunch(ex, s);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaGraphLaunch");
+    } else {  // new key: run eagerly and remember it
+      if (p.graph_exec) { cudaGraphExecDestroy(static_cast<cudaGraphExec_t>(p.graph_exec)); p.graph_exec = nullptr; }
+      p.g_in = in; p.g_out = out; p.g_T = T; p.g_stream = (void*)s;
+      e = enqueue(p, in, out, T, two, s);
+      if (e != cudaSuccess) return cuda_fail(e, "stencil kernel launch");
+    }
+  } else {
+    e = enqueue(p, in, out, T, two, s);
+    if (e != cudaSuccess) return cuda_fail(e, "stencil kernel launch");
   }
   if (sync_check()) {
     e = cudaStreamSynchronize(s);
@@ -116,6 +163,7 @@ void lora_stencil_plan_destroy(lora_plan* p) {
     int cur = -1;
     cudaGetDevice(&cur);
     if (cur != p->device) cudaSetDevice(p->device);
+    if (p->graph_exec) cudaGraphExecDestroy(static_cast<cudaGraphExec_t>(p->graph_exec));
     if (p->scratch) cudaFree(p->scratch);
     if (p->dev_in) cudaFree(p->dev_in);
     if (p->dev_out) cudaFree(p->dev_out);

@@ -392,9 +392,16 @@ cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream
     if (e != cudaSuccess) return e;
     max_grid = persistent_grid((const void*)rdg2d_kernel<R, SIG, K, TMA>, RDG_WARPS * 32, smem, int64_t(1) << 40);
   }
-  const int RC = ((RDG_RC + n - 1) / n) * n;  // chunk rows: a multiple of 2R+1 (static ring slots)
+  // chunk rows: a multiple of 2R+1 (static ring slots), <= RDG_RC; small grids get shorter chunks
+  // so that every resident warp has a stream (>= 2 items per warp slot when the grid allows it)
+  const int nbands = (int)((p.N[1] + BS - 1) / BS);
+  const int64_t want = int64_t(max_grid) * RDG_WARPS * 2;
+  int64_t rc = (p.N[0] * nbands + want - 1) / want;
+  rc = std::max<int64_t>(rc, 4 * K * R);                      // keep the halo-row overhead bounded
+  rc = std::min<int64_t>(rc, RDG_RC);
+  const int RC = (int)(((rc + n - 1) / n) * n);
   const int SI = (RC + 2 * K * R + G::SROWS - 1) / G::SROWS;
-  const int nbands = (int)((p.N[1] + BS - 1) / BS), nchunks = (int)((p.N[0] + RC - 1) / RC);
+  const int nchunks = (int)((p.N[0] + RC - 1) / RC);
   const int nitems = nbands * nchunks;
   const int grid = (int)std::min<int64_t>(max_grid, (nitems + RDG_WARPS - 1) / RDG_WARPS);
   rdg2d_kernel<R, SIG, K, TMA><<<grid, RDG_WARPS * 32, smem, s>>>(src, dst, p.N[0], p.N[1], nbands, nitems, RC, SI,

@@ -44,6 +44,11 @@ struct Plan {
   double* dev_in = nullptr;       // run_host staging (device copies of host in/out)
   double* dev_out = nullptr;
   size_t elems = 0;               // padded element count
+  void* graph_exec = nullptr;     // cudaGraphExec_t of the cached time loop (small grids)
+  const double* g_in = nullptr;   // its key
+  double* g_out = nullptr;
+  int64_t g_T = -1;
+  void* g_stream = nullptr;
   int64_t P[3] = {1, 1, 1};       // padded extents
 };
 

@@ -17,6 +17,7 @@ ap.add_argument("--engines", default="direct,tc")
 ap.add_argument("--T", type=int, default=20)
 ap.add_argument("--fuse", default="1")
 args = ap.parse_args()
+torch.cuda.set_stream(torch.cuda.Stream())  # a capturable stream (CUDA graphs for small grids)
 for name in args.configs.split(","):
     W, c = synth.config(name)
     x = torch.rand(c["padded"], dtype=torch.float64, device="cuda") + 0.5
