@@ -395,11 +395,21 @@ cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream
   // chunk rows: a multiple of 2R+1 (static ring slots), <= RDG_RC; small grids get shorter chunks
   // so that every resident warp has a stream (>= 2 items per warp slot when the grid allows it)
   const int nbands = (int)((p.N[1] + BS - 1) / BS);
-  const int64_t want = int64_t(max_grid) * RDG_WARPS * 2;
+  const int64_t TWmax = int64_t(max_grid) * RDG_WARPS;
+  const int64_t want = TWmax * 2;
   int64_t rc = (p.N[0] * nbands + want - 1) / want;
   rc = std::max<int64_t>(rc, 4 * K * R);                      // keep the halo-row overhead bounded
   rc = std::min<int64_t>(rc, RDG_RC);
-  const int RC = (int)(((rc + n - 1) / n) * n);
+  rc = ((rc + n - 1) / n) * n;
+  {  // wave balance: the fewest whole rounds of TWmax items, then the shortest chunk that fits them
+    const int64_t nitems0 = nbands * ((p.N[0] + rc - 1) / rc);
+    const int64_t rounds = (nitems0 + TWmax - 1) / TWmax;
+    const int64_t nch = std::max<int64_t>(1, (rounds * TWmax) / nbands);
+    int64_t rc2 = (p.N[0] + nch - 1) / nch;
+    rc2 = ((rc2 + n - 1) / n) * n;
+    if (rc2 <= RDG_RC + n && rc2 >= 4 * K * R && nbands * ((p.N[0] + rc2 - 1) / rc2) <= rounds * TWmax) rc = rc2;
+  }
+  const int RC = (int)rc;
   const int SI = (RC + 2 * K * R + G::SROWS - 1) / G::SROWS;
   const int nchunks = (int)((p.N[0] + RC - 1) / RC);
   const int nitems = nbands * nchunks;

@@ -48,7 +48,6 @@ struct G3 {
   static constexpr int ROWS = BY<R> + 2 * R;
   static constexpr int BW = 64 + 2 * R;
   static constexpr int STAGE = ((ROWS * BW * 8 + 127) / 128) * 128;
-  static constexpr int SI = ((R3_ZC + 2 * R + n - 1) / n) * n;   // planes streamed per item (multiple of n)
   static constexpr int WARP_BYTES = R3_NS * STAGE;
   static constexpr int SMEM = 128 + R3_WARPS * WARP_BYTES;
 };
@@ -162,7 +161,7 @@ __device__ __forceinline__ void apply_all(const double (&x)[BY<R> + 2 * R][2 * R
 template <int R, bool TMA>
 __global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* __restrict__ in, double* __restrict__ out,
                                                                  int64_t N0, int64_t N1, int64_t N2, int nbx, int nby,
-                                                                 int nitems, const __grid_constant__ CUtensorMap tmap,
+                                                                 int nitems, int ZC, int SI, const __grid_constant__ CUtensorMap tmap,
                                                                  const __grid_constant__ R3Params prm) {
   using G = G3<R>;
   constexpr int n = 2 * R + 1;
@@ -174,7 +173,7 @@ __global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* _
   const int64_t P1 = N1 + 2 * R, P2 = N2 + 2 * R;
   const int gw = blockIdx.x * R3_WARPS + wl, TW = gridDim.x * R3_WARPS;
   const int my_items = gw < nitems ? (nitems - 1 - gw) / TW + 1 : 0;
-  const int nstages = my_items * G::SI;
+  const int nstages = my_items * SI;
   if (TMA && lane == 0) {
     for (int s = 0; s < R3_NS; ++s) mbar_init(&bars[s], 1);
     fence_barrier_init();
@@ -186,7 +185,7 @@ __global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* _
     const int bx = item % nbx, rest = item / nbx, by = rest % nby, bz = rest / nby;
     bx0 = bx * 64;           // padded column of the staged tile origin (= interior column of lane col 0)
     by0 = by * BY<R>;        // padded row of the staged tile origin (= interior row of output row 0)
-    bz0 = bz * R3_ZC;        // first padded input plane (= first interior output plane) of the chunk
+    bz0 = bz * ZC;           // first padded input plane (= first interior output plane) of the chunk
   };
   int pitem = gw, pj = 0, px = 0, py = 0, pz = 0;
   if (gw < nitems) geom(pitem, px, py, pz);
@@ -208,7 +207,7 @@ __global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* _
       }
       cp_async_commit();
     }
-    if (++pj == G::SI) {
+    if (++pj == SI) {
       pj = 0;
       pitem += TW;
       if (pitem < nitems) geom(pitem, px, py, pz);
@@ -247,7 +246,7 @@ __global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* _
         c0ok = col < N2;
         c1ok = col + 1 < N2;
         cz = bz0;
-        zend = (int)(int64_t(bz0) + R3_ZC < N0 ? int64_t(bz0) + R3_ZC : N0);
+        zend = (int)(int64_t(bz0) + ZC < N0 ? int64_t(bz0) + ZC : N0);
         rowmask = 0;
 #pragma unroll
         for (int y = 0; y < BY<R>; ++y) rowmask |= (by0 + y < N1) ? (1 << y) : 0;
@@ -286,7 +285,7 @@ __global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* _
 #pragma unroll
       for (int y = 0; y < BY<R>; ++y) { acc[s][y][0] = 0.0; acc[s][y][1] = 0.0; }
       if (++slot == R3_NS) { slot = 0; phase ^= 1; }
-      if (++cj == G::SI) { cj = 0; citem += TW; }
+      if (++cj == SI) { cj = 0; citem += TW; }
     };
     [&]<int... Is>(std::integer_sequence<int, Is...>) {
       (one(std::integral_constant<int, Is>{}), ...);
@@ -353,11 +352,23 @@ cudaError_t rdg3d_launch(const Plan& p, const double* src, double* dst, cudaStre
     max_grid = persistent_grid((const void*)rdg3d_kernel<R, TMA>, R3_WARPS * 32, G::SMEM, int64_t(1) << 40);
   }
   const int nbx = (int)((p.N[2] + 63) / 64), nby = (int)((p.N[1] + BY<R> - 1) / BY<R>);
-  const int nbz = (int)((p.N[0] + R3_ZC - 1) / R3_ZC);
+  // z-chunk length: the fewest whole rounds of resident warps, then the shortest chunk that fits
+  const int64_t TWmax = int64_t(max_grid) * R3_WARPS;
+  int64_t zc = R3_ZC;
+  {
+    const int64_t cols = int64_t(nbx) * nby;
+    const int64_t rounds = (cols * ((p.N[0] + zc - 1) / zc) + TWmax - 1) / TWmax;
+    const int64_t nch = std::max<int64_t>(1, rounds * TWmax / cols);
+    const int64_t zc2 = (p.N[0] + nch - 1) / nch;
+    if (zc2 >= 8 && zc2 <= 2 * R3_ZC && cols * ((p.N[0] + zc2 - 1) / zc2) <= rounds * TWmax) zc = zc2;
+  }
+  const int ZC = (int)zc;
+  const int SI = (int)(((ZC + 2 * R) + G::n - 1) / G::n * G::n);
+  const int nbz = (int)((p.N[0] + ZC - 1) / ZC);
   const int64_t nitems = int64_t(nbx) * nby * nbz;
   const int grid = (int)std::min<int64_t>(max_grid, (nitems + R3_WARPS - 1) / R3_WARPS);
   rdg3d_kernel<R, TMA><<<grid, R3_WARPS * 32, G::SMEM, s>>>(src, dst, p.N[0], p.N[1], p.N[2], nbx, nby, (int)nitems,
-                                                           map, prm);
+                                                           ZC, SI, map, prm);
   return cudaGetLastError();
 }
 
