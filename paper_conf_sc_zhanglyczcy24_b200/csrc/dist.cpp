@@ -9,11 +9,19 @@
 // Every point is computed with the single-GPU kernels, so the result is bitwise equal to a
 // single-GPU run of the global grid (pin P10).
 //
+// Overlap (boundary first): each step computes the two edge strips of the slab first, the exchange
+// of their edge rows then runs on the comm's own stream while the interior strip is computed; the
+// next step waits for the exchange.  A strip is launched as the same kernel on a row-range view of
+// the arrays (rows [r0, r1) with the rows around them as its halo), so no kernel needs a row-range
+// argument and every point is computed exactly as in the full launch.
+//
 // NCCL is loaded at run time (dlopen of the libnccl.so.2 the process already has — torch's — or
 // the system one), so the library has no link-time NCCL dependency.
 #include <cuda_runtime.h>
 #include <dlfcn.h>
 
+#include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <new>
@@ -71,6 +79,8 @@ int nccl_fail(ncclResult_t r, const char* what) {
 struct lora_comm {
   ncclComm_t comm = nullptr;
   int rank = 0, nranks = 1, device = -1;
+  cudaStream_t comm_stream = nullptr;   // halo exchange runs here, overlapped with interior compute
+  cudaEvent_t ev_edge = nullptr, ev_comm = nullptr;
 };
 
 namespace {
@@ -139,12 +149,19 @@ int lora_stencil_comm_init(lora_comm** c, int nranks, int rank, const void* nccl
   cc->rank = rank;
   cc->nranks = nranks;
   cudaGetDevice(&cc->device);
+  if (cudaStreamCreateWithFlags(&cc->comm_stream, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreateWithFlags(&cc->ev_edge, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&cc->ev_comm, cudaEventDisableTiming) != cudaSuccess) {
+    cudaGetLastError();
+    lora_stencil_comm_destroy(cc);
+    return lora::fail(LORA_ERR_CUDA, "stream/event creation failed");
+  }
   if (nranks > 1) {
-    if (!nccl().ok) { delete cc; return lora::fail(LORA_ERR_NCCL, "libnccl.so.2 could not be loaded"); }
+    if (!nccl().ok) { lora_stencil_comm_destroy(cc); return lora::fail(LORA_ERR_NCCL, "libnccl.so.2 could not be loaded"); }
     ncclUniqueId id;
     std::memcpy(&id, nccl_unique_id, sizeof(id));
     ncclResult_t r = nccl().CommInitRank(&cc->comm, nranks, id, rank);
-    if (r) { delete cc; return nccl_fail(r, "ncclCommInitRank"); }
+    if (r) { lora_stencil_comm_destroy(cc); return nccl_fail(r, "ncclCommInitRank"); }
   }
   *c = cc;
   return LORA_OK;
@@ -175,13 +192,40 @@ int lora_stencil_run_dist(lora_plan* p, lora_comm* c, const double* in_local, do
   }
   // in_local's slab-edge halos hold the neighbours' initial rows (a slice of the global padded
   // array); every later buffer gets them from the exchange after each step.
+  const int64_t n0 = p->N[0];
+  const int64_t row = p->ndim == 2 ? p->P[1] : p->P[1] * p->P[2];
+  const int64_t B = std::max<int64_t>(p->R, std::min<int64_t>(64, n0 / 4));   // edge strip height
+  const char* fs = std::getenv("LORA_DIST_SPLIT");  // tests: exercise the split path on one rank
+  const bool force_split = fs && fs[0] == '1';
+  const bool split = (c->nranks > 1 || force_split) && n0 >= 2 * B + 1;
+  auto view = [&](int64_t r0, int64_t r1) {  // rows [r0, r1) of the local slab as a stand-alone plan
+    lora::Plan v = *p;
+    v.N[0] = r1 - r0;
+    v.P[0] = v.N[0] + 2 * p->R;
+    v.elems = size_t(v.P[0]) * size_t(row);
+    v.graph_exec = nullptr;
+    return v;
+  };
+  const lora::Plan top = split ? view(0, B) : *p, bot = split ? view(n0 - B, n0) : *p, mid = split ? view(B, n0 - B) : *p;
   const double* src = in_local;
   for (int64_t t = 1; t <= timesteps; ++t) {
     double* dst = ((timesteps - t) % 2 == 0) ? out_local : p->scratch;
-    e = step_launch(*p, src, dst, s);
-    if (e) return cuda_fail(e, "stencil kernel launch");
-    rc = exchange(p, c, dst, s);
-    if (rc) return rc;
+    if (!split) {
+      e = step_launch(*p, src, dst, s);
+      if (e) return cuda_fail(e, "stencil kernel launch");
+      rc = exchange(p, c, dst, s);
+      if (rc) return rc;
+    } else {
+      if ((e = step_launch(top, src, dst, s))) return cuda_fail(e, "edge strip launch");
+      if ((e = step_launch(bot, src + (n0 - B) * row, dst + (n0 - B) * row, s))) return cuda_fail(e, "edge strip launch");
+      cudaEventRecord(c->ev_edge, s);
+      cudaStreamWaitEvent(c->comm_stream, c->ev_edge, 0);
+      rc = exchange(p, c, dst, c->comm_stream);
+      if (rc) return rc;
+      cudaEventRecord(c->ev_comm, c->comm_stream);
+      if ((e = step_launch(mid, src + B * row, dst + B * row, s))) return cuda_fail(e, "interior strip launch");
+      cudaStreamWaitEvent(s, c->ev_comm, 0);  // the next step reads dst's exchanged halo rows
+    }
     src = dst;
   }
   if (sync_check()) {
@@ -194,6 +238,9 @@ int lora_stencil_run_dist(lora_plan* p, lora_comm* c, const double* in_local, do
 void lora_stencil_comm_destroy(lora_comm* c) {
   if (!c) return;
   if (c->comm && nccl().ok) nccl().CommDestroy(c->comm);
+  if (c->ev_edge) cudaEventDestroy(c->ev_edge);
+  if (c->ev_comm) cudaEventDestroy(c->ev_comm);
+  if (c->comm_stream) cudaStreamDestroy(c->comm_stream);
   delete c;
 }
 
