@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--per-stencil", action="store_true", help="also time the other single-GPU configs")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-engines", action="store_true", help="skip the per-engine comparison on the workload")
     return ap.parse_args()
 
 
@@ -297,6 +298,31 @@ def main():
             s2.close()
             del xa, ya
 
+    # the same workload on every engine (the paper's tensor-core chain, the CUDA-core RDG, direct)
+    engines = None
+    if rank == 0 and world == 1 and not args.no_engines:
+        engines = {}
+        for eng in ("tc", "rdg_cuda", "direct"):
+            try:
+                s3 = L.Stencil(W, shape, engine=eng)
+            except L.LoraError as ex:
+                engines[eng] = {"unsupported": str(ex)}
+                continue
+            L.lora_stencil_run(s3.plan, x.data_ptr(), y.data_ptr(), T, sptr)
+            torch.cuda.synchronize(dev)
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            for _ in range(2):
+                L.lora_stencil_run(s3.plan, x.data_ptr(), y.data_ptr(), T, sptr)
+            a1.record(stream)
+            torch.cuda.synchronize(dev)
+            ts = a0.elapsed_time(a1) / 2e3
+            gs = float(np.prod(shape)) * T / ts / 1e9
+            i3 = s3.info()
+            engines[eng] = {"GStencil_s": gs, "frac_hbm_roofline": gs / (peak / BYTES_PER_POINT), "fuse_k": i3["fuse_k"],
+                            "fma_per_point_issued": i3["fma_per_point_issued"], "ms_per_step": ts * 1e3}
+            s3.close()
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         cpu = cpu_oracle_sample(W, cfg)
@@ -318,6 +344,8 @@ def main():
                 "host": host_info()}
         if per_stencil:
             line["per_stencil"] = per_stencil
+        if engines:
+            line["engines"] = engines
         print(json.dumps(line), flush=True)
     if comm is not None:
         L.lora_stencil_comm_destroy(comm)
