@@ -30,6 +30,9 @@ bool tc3d_supported(const Plan& p);
 
 bool tc2d_supported(const Plan& p);
 bool rdg3d_supported(const Plan& p);
+// Two fused 3D steps (radius 1), kernels_rdg3df.cu.
+cudaError_t launch_rdg3d_fused2(const Plan& p, const double* src, double* dst, cudaStream_t s);
+bool rdg3d_fused_supported(const Plan& p);
 bool rdg2d_supported(const Plan& p);
 
 }  // namespace lora

@@ -260,11 +260,7 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (K == 1 || R == 1) ? 4 : 3) rd
     const int x = pX0 - R, y = pA - K * R + pj * G::SROWS;
     double* dst = reinterpret_cast<double*>(ring + slot * G::STAGE);
     if constexpr (TMA) {
-      if (x < 0 || y < 0) {  // first band / chunk of a fused launch: no TMA for negative boxes
-        warp_box_fill_sync(dst, in, P0, P1, y, x, G::SROWS, G::BW, lane);
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&bars[slot]);
-      } else if (lane == 0) {
+      if (lane == 0) {  // x is even by construction; negative origins are zero-filled by TMA
         fence_proxy_async();
         mbar_arrive_expect_tx(&bars[slot], G::SROWS * G::BW * 8);
         tma_load_2d(dst, &tmap, x, y, &bars[slot]);
@@ -469,6 +465,7 @@ bool rdg2d_supported(const Plan& p) {
 }
 
 int rdg2d_max_fuse(const Plan& p) {
+  if (p.ndim == 3) return rdg3d_fused_supported(p) ? 2 : 1;
   if (p.ndim != 2) return 1;
   RdgParams prm;
   const int sig = signature(p, prm);
@@ -477,7 +474,7 @@ int rdg2d_max_fuse(const Plan& p) {
 }
 
 cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s, int k) {
-  if (p.ndim == 3) return k == 1 ? launch_rdg3d(p, src, dst, s) : cudaErrorNotSupported;
+  if (p.ndim == 3) return k == 1 ? launch_rdg3d(p, src, dst, s) : (k == 2 ? launch_rdg3d_fused2(p, src, dst, s) : cudaErrorNotSupported);
   switch (p.R) {
     case 1: return rdg_r<1>(p, src, dst, s, k);
     case 2: return rdg_r<2>(p, src, dst, s, k);

@@ -55,13 +55,19 @@ struct G3 {
 __host__ __device__ constexpr int pm(int a, int n) { return ((a % n) + n) % n; }
 
 // Applies plane operator a0 to the staged plane (registers x) and adds into the ring slot(s).
-template <int R, int A0, int I>
+// Mode signature of a specialised kernel: planes 0 and 1 modes (-1 = run time), plane-0/2 mirror.
+template <int M0, int M1, int MIR>
+struct Sig3 {
+  static constexpr int m0 = M0, m1 = M1, mir = MIR;
+};
+
+template <int R, int A0, int I, int MODE = -1, int MIR = -1>
 __device__ __forceinline__ void apply_plane(const double (&x)[BY<R> + 2 * R][2 * R + 2],
                                             double (&acc)[2 * R + 1][BY<R>][2], const R3Params& P) {
   constexpr int n = 2 * R + 1;
   constexpr int s1 = pm(I - A0, n);           // output plane z = p - a0
   constexpr int s2 = pm(I - (n - 1 - A0), n); // mirrored plane
-  const int mode = P.mode[A0];
+  const int mode = MODE >= 0 ? MODE : P.mode[A0];
   if (mode == PM_NONE) return;
   double d[BY<R>][2];
   if (mode == PM_POINT) {
@@ -140,7 +146,7 @@ __device__ __forceinline__ void apply_plane(const double (&x)[BY<R> + 2 * R][2 *
     acc[s1][y][0] += d[y][0];
     acc[s1][y][1] += d[y][1];
   }
-  if (A0 < R && P.mirror[A0]) {
+  if (A0 < R && (MIR >= 0 ? MIR == 1 : P.mirror[A0] != 0)) {
 #pragma unroll
     for (int y = 0; y < BY<R>; ++y) {
       acc[s2][y][0] += d[y][0];
@@ -149,16 +155,20 @@ __device__ __forceinline__ void apply_plane(const double (&x)[BY<R> + 2 * R][2 *
   }
 }
 
-template <int R, int A0, int I>
+template <int R, class SG, int A0, int I>
 __device__ __forceinline__ void apply_all(const double (&x)[BY<R> + 2 * R][2 * R + 2],
                                           double (&acc)[2 * R + 1][BY<R>][2], const R3Params& P) {
   if constexpr (A0 < 2 * R + 1) {
-    if (!(A0 > R && P.mirror[2 * R - A0])) apply_plane<R, A0, I>(x, acc, P);
-    apply_all<R, A0 + 1, I>(x, acc, P);
+    // specialised modes exist for R = 1 only (plane 0, plane 1, plane 2 == mirror of plane 0)
+    constexpr int MODE = R != 1 ? -1 : (A0 == 0 ? SG::m0 : (A0 == 1 ? SG::m1 : (SG::mir == 1 ? SG::m0 : -1)));
+    constexpr int MIR = R != 1 ? -1 : SG::mir;
+    const bool skip = A0 > R && (MIR >= 0 ? MIR == 1 : P.mirror[2 * R - A0] != 0);
+    if (!skip) apply_plane<R, A0, I, MODE, MIR>(x, acc, P);
+    apply_all<R, SG, A0 + 1, I>(x, acc, P);
   }
 }
 
-template <int R, bool TMA>
+template <int R, class SG, bool TMA>
 __global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* __restrict__ in, double* __restrict__ out,
                                                                  int64_t N0, int64_t N1, int64_t N2, int nbx, int nby,
                                                                  int nitems, int ZC, int SI, const __grid_constant__ CUtensorMap tmap,
@@ -264,7 +274,7 @@ __global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* _
           x[r][2 * m + 1] = t.y;
         }
       __syncwarp();  // slot consumed
-      apply_all<R, 0, I>(x, acc, prm);
+      apply_all<R, SG, 0, I>(x, acc, prm);
       // output plane zi = (input plane) - 2R is complete: slot (I - 2R) mod n == (I + 1) mod n
       constexpr int s = (I + 1) % n;
       const int zi = cz + cj - 2 * R;
@@ -341,15 +351,15 @@ bool make_params3(const Plan& p, R3Params& prm) {
   return true;
 }
 
-template <int R, bool TMA>
+template <int R, class SG, bool TMA>
 cudaError_t rdg3d_launch(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
                          const R3Params& prm) {
   using G = G3<R>;
   static int max_grid = 0;
   if (max_grid == 0) {
-    cudaError_t e = cudaFuncSetAttribute(rdg3d_kernel<R, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, G::SMEM);
+    cudaError_t e = cudaFuncSetAttribute(rdg3d_kernel<R, SG, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, G::SMEM);
     if (e != cudaSuccess) return e;
-    max_grid = persistent_grid((const void*)rdg3d_kernel<R, TMA>, R3_WARPS * 32, G::SMEM, int64_t(1) << 40);
+    max_grid = persistent_grid((const void*)rdg3d_kernel<R, SG, TMA>, R3_WARPS * 32, G::SMEM, int64_t(1) << 40);
   }
   const int nbx = (int)((p.N[2] + 63) / 64), nby = (int)((p.N[1] + BY<R> - 1) / BY<R>);
   // z-chunk length: the fewest whole rounds of resident warps, then the shortest chunk that fits
@@ -367,7 +377,7 @@ cudaError_t rdg3d_launch(const Plan& p, const double* src, double* dst, cudaStre
   const int nbz = (int)((p.N[0] + ZC - 1) / ZC);
   const int64_t nitems = int64_t(nbx) * nby * nbz;
   const int grid = (int)std::min<int64_t>(max_grid, (nitems + R3_WARPS - 1) / R3_WARPS);
-  rdg3d_kernel<R, TMA><<<grid, R3_WARPS * 32, G::SMEM, s>>>(src, dst, p.N[0], p.N[1], p.N[2], nbx, nby, (int)nitems,
+  rdg3d_kernel<R, SG, TMA><<<grid, R3_WARPS * 32, G::SMEM, s>>>(src, dst, p.N[0], p.N[1], p.N[2], nbx, nby, (int)nitems,
                                                            ZC, SI, map, prm);
   return cudaGetLastError();
 }
@@ -380,9 +390,18 @@ cudaError_t rdg3d_r(const Plan& p, const double* src, double* dst, cudaStream_t 
   CUtensorMap map;
   const int64_t padded[3] = {p.P[0], p.P[1], p.P[2]};
   const int box[3] = {1, G::ROWS, G::BW};
-  if (!p.force_no_tma && encode_tmap(&map, src, 3, padded, box)) return rdg3d_launch<R, true>(p, src, dst, s, map, prm);
-  std::memset(&map, 0, sizeof(map));
-  return rdg3d_launch<R, false>(p, src, dst, s, map, prm);
+  const bool tma = !p.force_no_tma && encode_tmap(&map, src, 3, padded, box);
+  if (!tma) std::memset(&map, 0, sizeof(map));
+  if constexpr (R == 1) {  // Box-3D27P-like and Heat-3D-like plane signatures
+    if (prm.mode[0] == PM_PMA1 && prm.mode[1] == PM_PMA1 && prm.mirror[0])
+      return tma ? rdg3d_launch<R, Sig3<PM_PMA1, PM_PMA1, 1>, true>(p, src, dst, s, map, prm)
+                 : rdg3d_launch<R, Sig3<PM_PMA1, PM_PMA1, 1>, false>(p, src, dst, s, map, prm);
+    if (prm.mode[0] == PM_POINT && prm.mode[1] == PM_STAR && prm.mirror[0])
+      return tma ? rdg3d_launch<R, Sig3<PM_POINT, PM_STAR, 1>, true>(p, src, dst, s, map, prm)
+                 : rdg3d_launch<R, Sig3<PM_POINT, PM_STAR, 1>, false>(p, src, dst, s, map, prm);
+  }
+  return tma ? rdg3d_launch<R, Sig3<-1, -1, -1>, true>(p, src, dst, s, map, prm)
+             : rdg3d_launch<R, Sig3<-1, -1, -1>, false>(p, src, dst, s, map, prm);
 }
 
 }  // namespace

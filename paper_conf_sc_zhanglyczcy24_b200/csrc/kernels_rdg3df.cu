@@ -1,0 +1,399 @@
+// Exact temporal fusion of two 3D time steps (SURVEY NEXT-2 "2.5D blocking") for the
+// radius-1 Alg. 2 CUDA-core engine.
+//
+// A CTA (8 warps) owns a column of the domain: 64 lane columns x 16 step-1 rows (14 final rows),
+// streaming along z through a chunk of ZC final planes.  For every input plane p (TMA 3D box
+// 18 x 66, 3-stage ring; zero fill outside the array):
+//   stage 1: warp w applies the plane operators (Alg. 2: PMA / star / point-wise / general rank-1
+//            chains per plane) to produce step-1 rows 2w, 2w+1 and scatters them into a register
+//            z-ring of 3 step-1 planes; the completed step-1 plane p-1 gets the fixed Dirichlet halo
+//            re-imposed and is written to a shared plane buffer (double-buffered);
+//   one __syncthreads;
+//   stage 2: warps 0..6 apply the same operators to that step-1 plane (final rows 2w, 2w+1) into a
+//            second z-ring; the completed final plane p-2 is stored.
+// Every point goes through the same arithmetic as two unfused steps of kernels_rdg3d.cu's mode
+// code, so the result equals two separate steps to rounding; halo handling makes it exact
+// temporal blocking (reading Q5).  The lane columns lose one valid column per side per
+// fused step: x bands overlap with stride 60 (even TMA origin).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <utility>
+#include <vector>
+
+#include "kernels.hpp"
+#include "pipe.cuh"
+
+namespace lora {
+namespace {
+
+constexpr int F_NS = 3;              // TMA ring stages
+constexpr int F_WARPS = 8;
+constexpr int F_S1 = 16;             // step-1 rows per CTA column (2 per warp)
+constexpr int F_TY = 14;             // final rows per CTA column
+constexpr int F_IN = 18;             // staged input rows
+constexpr int F_BW = 66;             // staged columns (64 + 2R)
+constexpr int F_BS = 60;             // x band stride (valid final columns per band, even TMA origin)
+constexpr int F_S1W = 72;            // step-1 plane buffer row pitch (doubles): data at [1, 65)
+constexpr int F_ZC = 64;
+
+enum { PM_NONE = 0, PM_POINT = 1, PM_CHAINS = 2, PM_STAR = 3, PM_PMA1 = 4 };
+constexpr int F_MAXK = 3;
+
+struct FParams {
+  int mode[3], K[3], mirror[3];
+  double w[3];
+  double u[3][F_MAXK][3], v[3][F_MAXK][3];
+};
+
+__host__ __device__ constexpr int pm3(int a) { return ((a % 3) + 3) % 3; }
+
+// Plane operator A0 on 2 output rows: rows 0..3 of `x` (4 consecutive input rows, 4 columns each:
+// the lane's 2 columns +-1) -> d[2][2].  Same arithmetic as kernels_rdg3d.cu's apply_plane (R = 1).
+template <int A0, int MODE>
+__device__ __forceinline__ bool plane2(const double (&x)[4][4], const FParams& P, double (&d)[2][2]) {
+  const int mode = MODE >= 0 ? MODE : P.mode[A0];  // MODE >= 0: the kernel is specialised on it
+  if (mode == PM_NONE) return false;
+  if (mode == PM_POINT) {
+#pragma unroll
+    for (int y = 0; y < 2; ++y) { d[y][0] = P.w[A0] * x[y + 1][1]; d[y][1] = P.w[A0] * x[y + 1][2]; }
+  } else if (mode == PM_STAR) {
+#pragma unroll
+    for (int y = 0; y < 2; ++y) {
+      double t0 = 0.0, t1 = 0.0;
+#pragma unroll
+      for (int b = -1; b <= 1; ++b) {
+        t0 = fma(P.v[A0][0][1 + b], x[y + 1][1 + b], t0);
+        t1 = fma(P.v[A0][0][1 + b], x[y + 1][2 + b], t1);
+      }
+#pragma unroll
+      for (int a = -1; a <= 1; ++a) {
+        t0 = fma(P.u[A0][1][1 + a], x[y + 1 + a][1], t0);
+        t1 = fma(P.u[A0][1][1 + a], x[y + 1 + a][2], t1);
+      }
+      d[y][0] = t0; d[y][1] = t1;
+    }
+  } else if (mode == PM_PMA1) {
+    double T[4][2];
+#pragma unroll
+    for (int r = 0; r < 4; ++r) {
+      T[r][0] = fma(P.v[A0][0][2], x[r][0] + x[r][2], P.v[A0][0][1] * x[r][1]);
+      T[r][1] = fma(P.v[A0][0][2], x[r][1] + x[r][3], P.v[A0][0][1] * x[r][2]);
+    }
+#pragma unroll
+    for (int y = 0; y < 2; ++y) {
+      d[y][0] = fma(P.u[A0][0][2], T[y][0] + T[y + 2][0], fma(P.u[A0][0][1], T[y + 1][0], P.w[A0] * x[y + 1][1]));
+      d[y][1] = fma(P.u[A0][0][2], T[y][1] + T[y + 2][1], fma(P.u[A0][0][1], T[y + 1][1], P.w[A0] * x[y + 1][2]));
+    }
+  } else {
+#pragma unroll
+    for (int y = 0; y < 2; ++y) { d[y][0] = 0.0; d[y][1] = 0.0; }
+#pragma unroll
+    for (int k = 0; k < F_MAXK; ++k) {
+      if (k < P.K[A0]) {
+        double T[4][2];
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+          double t0 = 0.0, t1 = 0.0;
+#pragma unroll
+          for (int b = -1; b <= 1; ++b) {
+            t0 = fma(P.v[A0][k][1 + b], x[r][1 + b], t0);
+            t1 = fma(P.v[A0][k][1 + b], x[r][2 + b], t1);
+          }
+          T[r][0] = t0; T[r][1] = t1;
+        }
+#pragma unroll
+        for (int y = 0; y < 2; ++y)
+#pragma unroll
+          for (int a = -1; a <= 1; ++a) {
+            d[y][0] = fma(P.u[A0][k][1 + a], T[y + 1 + a][0], d[y][0]);
+            d[y][1] = fma(P.u[A0][k][1 + a], T[y + 1 + a][1], d[y][1]);
+          }
+      }
+    }
+  }
+  return true;
+}
+
+// Mode signature of a specialised kernel: modes of planes 0 and 1 (-1 = read at run time) and
+// whether plane 2 mirrors plane 0 (-1 = read at run time).
+template <int M0, int M1, int MIR>
+struct Sig3 {
+  static constexpr int m0 = M0, m1 = M1, mir = MIR;
+};
+
+// All plane operators of one input plane (ring position I) into a z-ring of 3 planes x 2 rows.
+template <class SG, int I, int A0>
+__device__ __forceinline__ void planes2(const double (&x)[4][4], const FParams& P, double (&acc)[3][2][2]) {
+  if constexpr (A0 < 3) {
+    const bool mirror = SG::mir >= 0 ? SG::mir == 1 : P.mirror[0] != 0;
+    constexpr int MODE = A0 == 0 ? SG::m0 : (A0 == 1 ? SG::m1 : (SG::mir == 1 ? SG::m0 : -1));
+    if (!(A0 == 2 && mirror)) {
+      double d[2][2];
+      if (plane2<A0, MODE>(x, P, d)) {
+        constexpr int s1 = pm3(I - A0);
+#pragma unroll
+        for (int y = 0; y < 2; ++y) { acc[s1][y][0] += d[y][0]; acc[s1][y][1] += d[y][1]; }
+        if (A0 == 0 && mirror) {
+          constexpr int s2 = pm3(I - 2);
+#pragma unroll
+          for (int y = 0; y < 2; ++y) { acc[s2][y][0] += d[y][0]; acc[s2][y][1] += d[y][1]; }
+        }
+      }
+    }
+    planes2<SG, I, A0 + 1>(x, P, acc);
+  }
+}
+
+__device__ __forceinline__ void load_rows(const double* __restrict__ base, int pitch, int lane, double (&x)[4][4]) {
+#pragma unroll
+  for (int r = 0; r < 4; ++r) {
+    const double2 a = *reinterpret_cast<const double2*>(base + r * pitch + 2 * lane);
+    const double2 b = *reinterpret_cast<const double2*>(base + r * pitch + 2 * lane + 2);
+    x[r][0] = a.x; x[r][1] = a.y; x[r][2] = b.x; x[r][3] = b.y;
+  }
+}
+
+template <class SG, bool TMA>
+__global__ void __launch_bounds__(F_WARPS * 32, 2) rdg3df_kernel(const double* __restrict__ in, double* __restrict__ out,
+                                                                 int64_t N0, int64_t N1, int64_t N2, int nbx, int nby,
+                                                                 int nitems, int ZC, int SI,
+                                                                 const __grid_constant__ CUtensorMap tmap,
+                                                                 const __grid_constant__ FParams prm) {
+  constexpr int STAGE = ((F_IN * F_BW * 8 + 127) / 128) * 128;
+  constexpr int S1B = F_S1 * F_S1W;  // doubles per step-1 plane buffer
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw);
+  unsigned char* ring = smem_raw + 128;
+  double* s1buf = reinterpret_cast<double*>(smem_raw + 128 + F_NS * STAGE);  // [2][F_S1][F_S1W]
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  const int P0 = (int)(N0 + 2), P1 = (int)(N1 + 2), P2 = (int)(N2 + 2);
+  for (int i = tid; i < 2 * S1B; i += blockDim.x) s1buf[i] = 0.0;   // margins stay zero
+  const int my_items = blockIdx.x < nitems ? (nitems - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+  const int nstages = my_items * SI;
+  if (TMA && tid == 0) {
+    for (int s = 0; s < F_NS; ++s) mbar_init(&bar[s], 1);
+    fence_barrier_init();
+  }
+  __syncthreads();
+  // item -> lane column 0 at padded X0, final rows from padded Y0, final planes from padded Z0
+  auto geom = [&](int item, int& X0, int& Y0, int& Z0) {
+    const int bx = item % nbx, rest = item / nbx, by = rest % nby, bz = rest / nby;
+    X0 = 1 + bx * F_BS - 1 - 1;        // R + b*BS - R(K-1) - SG   (X0 - R even)
+    Y0 = 1 + by * F_TY;
+    Z0 = 1 + bz * ZC;
+  };
+  int pitem = blockIdx.x, pj = 0, pX = 0, pY = 0, pZ = 0;
+  if (pitem < nitems) geom(pitem, pX, pY, pZ);
+  auto issue_next = [&](int slot) {
+    double* dst = reinterpret_cast<double*>(ring + slot * STAGE);
+    const int x = pX - 1, y = pY - 2, z = pZ - 2 + pj;
+    if constexpr (TMA) {  // x even by construction; negative origins are zero-filled by TMA
+      if (tid == 0) {
+        fence_proxy_async();
+        mbar_arrive_expect_tx(&bar[slot], F_IN * F_BW * 8);
+        tma_load_3d(dst, &tmap, x, y, z, &bar[slot]);
+      }
+    } else {  // no TMA (row pitch not a multiple of 16 B): the CTA fills the box itself
+      for (int i = tid; i < F_IN * F_BW; i += blockDim.x) {
+        const int r = i / F_BW, c = i - r * F_BW;
+        const int gy = y + r, gx = x + c;
+        dst[i] = (z >= 0 && z < P0 && gy >= 0 && gy < P1 && gx >= 0 && gx < P2)
+                     ? __ldg(in + (int64_t(z) * P1 + gy) * P2 + gx) : 0.0;
+      }
+      __syncthreads();
+    }
+    if (++pj == SI) {
+      pj = 0;
+      pitem += gridDim.x;
+      if (pitem < nitems) geom(pitem, pX, pY, pZ);
+    }
+  };
+  // prologue (uniform across the CTA: issue_next may contain __syncthreads)
+  for (int q = 0; q < F_NS - 1; ++q)
+    if (q < nstages) issue_next(q);
+  double acc1[3][2][2], acc2[3][2][2];
+  int citem = blockIdx.x, cj = 0, slot = 0, phase = 0;
+  int X0 = 0, Y0 = 0, Z0 = 0, zend = 0;
+  const int c0 = 2 * lane;  // lane's first column (relative to X0)
+  for (int q0 = 0; q0 < nstages; q0 += 3) {
+    auto one = [&](auto Ic) {
+      constexpr int I = decltype(Ic)::value;
+      const int q = q0 + I;
+      if (TMA) mbar_wait(&bar[slot], phase);
+      else __syncthreads();
+      if (cj == 0) {
+        geom(citem, X0, Y0, Z0);
+        zend = min(Z0 + ZC, P0 - 1);
+#pragma unroll
+        for (int s = 0; s < 3; ++s)
+#pragma unroll
+          for (int y = 0; y < 2; ++y) { acc1[s][y][0] = acc1[s][y][1] = 0.0; acc2[s][y][0] = acc2[s][y][1] = 0.0; }
+      }
+      const int p = Z0 - 2 + cj;  // padded input plane
+      // ---------------- stage 1: step-1 rows 2w, 2w+1 from input tile rows 2w .. 2w+3
+      {
+        const double* st = reinterpret_cast<const double*>(ring + slot * STAGE);
+        double x[4][4];
+        load_rows(st + (2 * w) * F_BW, F_BW, lane, x);
+        planes2<SG, I, 0>(x, prm, acc1);
+      }
+      // step-1 plane z1 = p - 1 is complete (ring slot (I + 1) % 3); re-impose the halo, publish it
+      {
+        constexpr int s = (I + 1) % 3;
+        const int z1 = p - 1;
+        const int par = q & 1;
+        double* S = s1buf + par * S1B;
+#pragma unroll
+        for (int y = 0; y < 2; ++y) {
+          double v0 = acc1[s][y][0], v1 = acc1[s][y][1];
+          acc1[s][y][0] = 0.0; acc1[s][y][1] = 0.0;
+          const int gy = Y0 - 1 + 2 * w + y;  // padded row of this step-1 row
+          const int gx = X0 + c0;
+          const bool zin = z1 >= 0 && z1 < P0, yin = gy >= 0 && gy < P1;
+          const bool zh = z1 < 1 || z1 >= P0 - 1, yh = gy < 1 || gy >= P1 - 1;
+#pragma unroll
+          for (int e = 0; e < 2; ++e) {
+            const int cx = gx + e;
+            const bool xin = cx >= 0 && cx < P2, xh = cx < 1 || cx >= P2 - 1;
+            double v = e ? v1 : v0;
+            if (!(zin && yin && xin)) v = 0.0;
+            else if (zh || yh || xh) v = in[(int64_t(z1) * P1 + gy) * P2 + cx];
+            S[(2 * w + y) * F_S1W + 1 + c0 + e] = v;
+          }
+        }
+      }
+      __syncthreads();  // step-1 plane visible; every warp is done with the input slot
+      if (q + F_NS - 1 < nstages) issue_next((slot + F_NS - 1) % F_NS);
+      // ---------------- stage 2: final rows 2w, 2w+1 from step-1 rows 2w .. 2w+3
+      if (w < F_TY / 2 && cj >= 2) {
+        const double* S = s1buf + (q & 1) * S1B;
+        double x[4][4];
+        load_rows(S + (2 * w) * F_S1W, F_S1W, lane, x);
+        planes2<SG, pm3(I - 1), 0>(x, prm, acc2);
+        // final plane zf = p - 2 complete: ring slot (I - 1 + 1) % 3
+        constexpr int s = pm3(I);
+        const int zf = p - 2;
+        if (cj >= 4 && zf >= Z0 && zf < zend) {
+#pragma unroll
+          for (int y = 0; y < 2; ++y) {
+            const int gy = Y0 + 2 * w + y;
+            if (gy < P1 - 1 && gy < Y0 + F_TY) {
+              double* o = out + (int64_t(zf) * P1 + gy) * P2 + X0;
+#pragma unroll
+              for (int e = 0; e < 2; ++e) {
+                const int cx = X0 + c0 + e;
+                if (c0 + e >= 1 && c0 + e < 63 && cx >= 1 && cx < P2 - 1) o[c0 + e] = acc2[s][y][e];
+              }
+            }
+          }
+        }
+#pragma unroll
+        for (int y = 0; y < 2; ++y) { acc2[s][y][0] = 0.0; acc2[s][y][1] = 0.0; }
+      }
+      if (++slot == F_NS) { slot = 0; phase ^= 1; }
+      if (++cj == SI) { cj = 0; citem += gridDim.x; }
+    };
+    [&]<int... Is>(std::integer_sequence<int, Is...>) {
+      (one(std::integral_constant<int, Is>{}), ...);
+    }(std::make_integer_sequence<int, 3>{});
+  }
+}
+
+bool make_fparams(const Plan& p, FParams& prm) {
+  std::memset(&prm, 0, sizeof(prm));
+  if (p.ndim != 3 || p.R != 1) return false;
+  const int R = 1, n = 3;
+  for (int a0 = 0; a0 < n; ++a0) {
+    std::vector<const Term*> ts;
+    for (const Term& t : p.terms)
+      if (t.plane == a0) ts.push_back(&t);
+    if (ts.empty()) { prm.mode[a0] = PM_NONE; continue; }
+    if (ts.size() == 1 && ts[0]->kind == kPoint && ts[0]->u[R] == 1.0 && ts[0]->u[0] == 0.0 && ts[0]->u[2] == 0.0 &&
+        ts[0]->v[0] == 0.0 && ts[0]->v[2] == 0.0) {
+      prm.mode[a0] = PM_POINT; prm.w[a0] = ts[0]->v[R]; continue;
+    }
+    if (ts.size() == 2 && ts[0]->kind == kArm && ts[1]->kind == kArm && ts[0]->u[R] == 1.0 && ts[1]->v[R] == 1.0 &&
+        ts[0]->u[0] == 0.0 && ts[0]->u[2] == 0.0 && ts[1]->v[0] == 0.0 && ts[1]->v[2] == 0.0) {
+      prm.mode[a0] = PM_STAR;
+      for (int i = 0; i < n; ++i) { prm.v[a0][0][i] = ts[0]->v[i]; prm.u[a0][1][i] = ts[1]->u[i]; }
+      continue;
+    }
+    if (ts.size() == 2 && ts[0]->kind == kChain && ts[0]->r == 1 && ts[1]->kind == kPoint && ts[1]->r == 0 &&
+        ts[1]->u[R] == 1.0 && ts[0]->u[0] == ts[0]->u[2] && ts[0]->v[0] == ts[0]->v[2]) {
+      prm.mode[a0] = PM_PMA1;
+      for (int i = 0; i < n; ++i) { prm.u[a0][0][i] = ts[0]->u[i]; prm.v[a0][0][i] = ts[0]->v[i]; }
+      prm.w[a0] = ts[1]->v[R];
+      continue;
+    }
+    if ((int)ts.size() > F_MAXK) return false;
+    prm.mode[a0] = PM_CHAINS;
+    prm.K[a0] = (int)ts.size();
+    for (size_t k = 0; k < ts.size(); ++k)
+      for (int i = 0; i < n; ++i) { prm.u[a0][k][i] = ts[k]->u[i]; prm.v[a0][k][i] = ts[k]->v[i]; }
+  }
+  bool same = true;
+  for (int e = 0; e < n * n; ++e)
+    if (p.W[e] != p.W[size_t(2) * n * n + e]) { same = false; break; }
+  prm.mirror[0] = same ? 1 : 0;
+  return true;
+}
+
+template <class SG, bool TMA>
+cudaError_t launch_f(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
+                     const FParams& prm) {
+  constexpr int STAGE = ((F_IN * F_BW * 8 + 127) / 128) * 128;
+  const int smem = 128 + F_NS * STAGE + 2 * F_S1 * F_S1W * 8;
+  static int max_grid = 0;
+  if (max_grid == 0) {
+    cudaError_t e = cudaFuncSetAttribute(rdg3df_kernel<SG, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    max_grid = persistent_grid((const void*)rdg3df_kernel<SG, TMA>, F_WARPS * 32, smem, int64_t(1) << 40);
+  }
+  const int nbx = (int)((p.N[2] + F_BS - 1) / F_BS), nby = (int)((p.N[1] + F_TY - 1) / F_TY);
+  int64_t zc = F_ZC;
+  {
+    const int64_t cols = int64_t(nbx) * nby;
+    const int64_t rounds = (cols * ((p.N[0] + zc - 1) / zc) + max_grid - 1) / max_grid;
+    const int64_t nch = std::max<int64_t>(1, rounds * max_grid / cols);
+    const int64_t zc2 = (p.N[0] + nch - 1) / nch;
+    if (zc2 >= 8 && zc2 <= 2 * F_ZC && cols * ((p.N[0] + zc2 - 1) / zc2) <= rounds * max_grid) zc = zc2;
+  }
+  const int ZC = (int)zc;
+  const int SI = ((ZC + 4) + 2) / 3 * 3;
+  const int nbz = (int)((p.N[0] + ZC - 1) / ZC);
+  const int64_t nitems = int64_t(nbx) * nby * nbz;
+  const int grid = (int)std::min<int64_t>(max_grid, nitems);
+  rdg3df_kernel<SG, TMA><<<grid, F_WARPS * 32, smem, s>>>(src, dst, p.N[0], p.N[1], p.N[2], nbx, nby, (int)nitems, ZC, SI,
+                                                     map, prm);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+bool rdg3d_fused_supported(const Plan& p) {
+  FParams prm;
+  return make_fparams(p, prm);
+}
+
+cudaError_t launch_rdg3d_fused2(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  FParams prm;
+  if (!make_fparams(p, prm)) return cudaErrorNotSupported;
+  CUtensorMap map;
+  const int64_t padded[3] = {p.P[0], p.P[1], p.P[2]};
+  const int box[3] = {1, F_IN, F_BW};
+  const bool tma = !p.force_no_tma && encode_tmap(&map, src, 3, padded, box);
+  if (!tma) std::memset(&map, 0, sizeof(map));
+  // specialisations: Box-3D27P-like (PMA planes, z-mirrored) and Heat-3D-like (point / star, mirrored)
+  if (prm.mode[0] == PM_PMA1 && prm.mode[1] == PM_PMA1 && prm.mirror[0])
+    return tma ? launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, true>(p, src, dst, s, map, prm)
+               : launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, false>(p, src, dst, s, map, prm);
+  if (prm.mode[0] == PM_POINT && prm.mode[1] == PM_STAR && prm.mirror[0])
+    return tma ? launch_f<Sig3<PM_POINT, PM_STAR, 1>, true>(p, src, dst, s, map, prm)
+               : launch_f<Sig3<PM_POINT, PM_STAR, 1>, false>(p, src, dst, s, map, prm);
+  return tma ? launch_f<Sig3<-1, -1, -1>, true>(p, src, dst, s, map, prm)
+             : launch_f<Sig3<-1, -1, -1>, false>(p, src, dst, s, map, prm);
+}
+
+}  // namespace lora

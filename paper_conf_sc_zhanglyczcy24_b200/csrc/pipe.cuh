@@ -79,18 +79,9 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
-// Boxes that start at a negative coordinate are filled by the warp with plain loads (zero
-// outside the array) and completed on the same mbarrier with a plain arrive.  (TMA itself faults
-// with "illegal instruction" when the innermost box start is not 16-byte aligned — an odd FP64
-// column — see tools/ubench/tma_probe.cu; every caller keeps that coordinate even.)
-__device__ __forceinline__ void warp_box_fill_sync(double* dst, const double* __restrict__ src, int64_t P0, int64_t P1,
-                                                   int64_t y, int64_t x, int rows, int cols, int lane) {
-  for (int i = lane; i < rows * cols; i += 32) {
-    const int r = i / cols, c = i - r * cols;
-    const int64_t gy = y + r, gx = x + c;
-    dst[i] = (gy >= 0 && gy < P0 && gx >= 0 && gx < P1) ? __ldg(src + gy * P1 + gx) : 0.0;
-  }
-}
+// TMA tile loads fault ("illegal instruction") when the innermost box start is not 16-byte aligned
+// (an odd FP64 column); negative and out-of-range origins are fine and zero-filled
+// (tools/ubench/tma_probe.cu).  Every caller keeps the innermost coordinate even.
 
 // Fallback fill of a rows x cols box at padded coordinate (y, x) of a P0 x P1 array (2D) by all
 // threads of the CTA with LDGSTS; zero outside the array.  Completion: cp_async_wait + barrier.

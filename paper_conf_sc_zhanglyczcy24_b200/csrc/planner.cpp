@@ -310,7 +310,7 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
   if (fk == 0) {
     // default fusion depth (exact temporal blocking): measured on B200
     static const int dflt[5] = {1, 3, 2, 1, 1};  // by radius; tools/quickbench.py, gpurun_out/qb6.jsonl
-    fk = std::min(max_k, dflt[radius]);
+    fk = std::min(max_k, p.ndim == 3 ? 2 : dflt[radius]);
   }
   p.fuse_k = fk;
   {

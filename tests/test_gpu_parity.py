@@ -199,3 +199,27 @@ def test_graph_replay_matches_eager(monkeypatch):
     assert rel_err(outs[0], oracle.run(W, g, 10)) <= 1e-12
     assert rel_err(y.cpu().numpy(), oracle.run(W, 0.5 * g, 10)) <= 1e-12
     torch.cuda.set_stream(torch.cuda.default_stream())
+
+
+@pytest.mark.parametrize("kind", ["rsym", "heat3d", "asym", "star"])
+@pytest.mark.parametrize("shape", [(1, 1, 1), (3, 4, 5), (17, 9, 33), (40, 30, 130), (70, 15, 61)])
+def test_3d_temporal_fusion_exact(kind, shape):
+    """Two fused 3D steps (kernels_rdg3df.cu, halo re-imposed on the step-1 plane) equal two single
+    steps bitwise and the oracle to 1e-12; odd T exercises the remainder launch."""
+    W = synth.preset("heat3d") if kind == "heat3d" else _weights(kind, 3, 1, 21)
+    g = synth.grid(tuple(n + 2 for n in shape), 31)
+    for T in (1, 2, 3, 5):
+        a, info = run_gpu(W, g, T, engine="rdg_cuda", fuse_k=2)
+        assert info["fuse_k"] == 2
+        b, _ = run_gpu(W, g, T, engine="rdg_cuda", fuse_k=1)
+        assert np.array_equal(a, b), (T, float(np.max(np.abs(a - b))))
+        assert rel_err(a, oracle.run(W, g, T)) <= 1e-12
+
+
+def test_3d_fusion_staging_paths_agree(monkeypatch):
+    W = synth.rsym_weights(3, 1, 8)
+    g = synth.grid((34, 20, 66), 12)
+    a, _ = run_gpu(W, g, 4, engine="rdg_cuda", fuse_k=2)
+    monkeypatch.setenv("LORA_NO_TMA", "1")
+    b, _ = run_gpu(W, g, 4, engine="rdg_cuda", fuse_k=2)
+    assert np.array_equal(a, b)
