@@ -1,0 +1,26 @@
+"""compute-sanitizer memcheck / racecheck / synccheck over small runs of every engine, both staging
+paths (TMA and LDGSTS) and the fused kernels (-m gpu, slow)."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
+@pytest.mark.parametrize("no_tma", ["0", "1"])
+def test_compute_sanitizer_clean(tool, no_tma):
+    cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+    if not os.path.exists(cs):
+        pytest.skip("compute-sanitizer not found")
+    env = dict(os.environ, LORA_NO_TMA=no_tma, LORA_NO_GRAPH="1")
+    r = subprocess.run([cs, "--tool", tool, "--error-exitcode", "17", sys.executable, "tools/sanitize_cases.py"],
+                       cwd=ROOT, env=env, capture_output=True, text=True, timeout=1200)
+    out = r.stdout + r.stderr
+    assert r.returncode == 0, out[-4000:]
+    assert "sanitize cases ok" in out
+    assert "ERROR SUMMARY: 0 errors" in out or "0 errors" in out
