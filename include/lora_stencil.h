@@ -2,7 +2,7 @@
  * lora_stencil.h — C-ABI of the B200-native LoRAStencil engine.
  *
  * What the library computes (PAPER.md = /root/reference/PAPER.md, "P:n" = its line n):
- *   A time-iterated d-dimensional FP64 stencil (d = 2, 3): every interior point is replaced,
+ *   A time-iterated d-dimensional FP64 stencil (d = 1, 2, 3): every interior point is replaced,
  *   T times, by the weighted sum of its (2r+1)^d neighbourhood (§I; eq. 2).
  *   The weights are factored on the host into rank-1 terms u_k v_k^T (eq. 8 P:149-153;
  *   Pyramidal Matrix Adaptation, eq. 15) and each term is evaluated as the banded
@@ -89,7 +89,7 @@ typedef struct {               /* filled by lora_stencil_plan_query             
  * (star arms / PMA / complete-pivot elimination, Q6), checks the reconstruction
  * (<= 1e-14 relative, else NULL with LORA_ERR_FACTOR), and picks engine, tile and fusion.
  *   weights    host, (2*radius+1)^ndim doubles, row-major, copied (caller keeps ownership)
- *   ndim       2 or 3
+ *   ndim       1, 2 or 3 (1D: a single banded gather; tensor-core engine 2D/3D only)
  *   radius     1..4
  *   grid_shape host, ndim interior extents (slowest first), each >= 1
  * The plan binds to the CUDA device that is current at its first run call. */

@@ -56,12 +56,12 @@ def max_threads() -> int:
 def run(W: np.ndarray, grid: np.ndarray, T: int, threads: int = 0) -> np.ndarray:
     """T Jacobi steps of the direct stencil on a padded grid; returns a new padded array.
 
-    W has shape (2h+1,)*d, grid has shape (N_i + 2h) per axis (d = 2 or 3)."""
+    W has shape (2h+1,)*d, grid has shape (N_i + 2h) per axis (d = 1, 2 or 3)."""
     W = np.ascontiguousarray(W, dtype=np.float64)
     grid = np.ascontiguousarray(grid, dtype=np.float64)
     d = W.ndim
     h = (W.shape[0] - 1) // 2
-    assert d in (2, 3) and all(s == 2 * h + 1 for s in W.shape) and grid.ndim == d
+    assert d in (1, 2, 3) and all(s == 2 * h + 1 for s in W.shape) and grid.ndim == d
     N = np.array([s - 2 * h for s in grid.shape], dtype=np.int64)
     out = np.empty_like(grid)
     rc = _load().oracle_stencil_run(W.ctypes.data, d, h, N.ctypes.data, grid.ctypes.data, out.ctypes.data,

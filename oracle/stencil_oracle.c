@@ -17,7 +17,7 @@
  * is therefore bitwise independent of the OpenMP thread count (each point is computed by
  * one thread in a fixed order).
  *
- * Layout: `in`/`out` are padded arrays of extent (N_i + 2h) per axis, C order, slowest first.
+ * d = 1, 2, 3.  Layout: `in`/`out` are padded arrays of extent (N_i + 2h) per axis, C order, slowest first.
  */
 #include <stdint.h>
 #include <stdlib.h>
@@ -25,6 +25,19 @@
 #ifdef _OPENMP
 #include <omp.h>
 #endif
+
+static void step1d(const double* W, int h, int64_t N0, const double* A, double* B) {
+  const int n = 2 * h + 1;
+#pragma omp parallel for schedule(static)
+  for (int64_t x0 = h; x0 < h + N0; ++x0) {
+    double s = 0.0;
+    for (int a0 = 0; a0 < n; ++a0) {
+      double p = W[a0] * A[x0 + a0 - h];
+      s = s + p;
+    }
+    B[x0] = s;
+  }
+}
 
 static void step2d(const double* W, int h, int64_t N0, int64_t N1, const double* A, double* B) {
   const int64_t P1 = N1 + 2 * h;
@@ -68,7 +81,7 @@ static void step3d(const double* W, int h, int64_t N0, int64_t N1, int64_t N2, c
  * nthreads <= 0 keeps the OpenMP default.  Returns 0, or -1 on bad arguments / OOM. */
 int oracle_stencil_run(const double* W, int ndim, int h, const int64_t* N, const double* in, double* out,
                        int64_t T, int nthreads) {
-  if ((ndim != 2 && ndim != 3) || h < 1 || T < 0 || !W || !N || !in || !out) return -1;
+  if (ndim < 1 || ndim > 3 || h < 1 || T < 0 || !W || !N || !in || !out) return -1;
   int64_t total = 1;
   for (int i = 0; i < ndim; ++i) {
     if (N[i] < 1) return -1;
@@ -85,7 +98,8 @@ int oracle_stencil_run(const double* W, int ndim, int h, const int64_t* N, const
   memcpy(A, in, (size_t)total * sizeof(double));
   memcpy(B, in, (size_t)total * sizeof(double)); /* halo of both buffers = the fixed boundary */
   for (int64_t t = 0; t < T; ++t) {
-    if (ndim == 2) step2d(W, h, N[0], N[1], A, B);
+    if (ndim == 1) step1d(W, h, N[0], A, B);
+    else if (ndim == 2) step2d(W, h, N[0], N[1], A, B);
     else step3d(W, h, N[0], N[1], N[2], A, B);
     double* tmp = A; A = B; B = tmp;
   }

@@ -40,6 +40,7 @@ int ensure_device(Plan& p, bool want_scratch) {
 
 // One launch advancing `k` time steps (k > 1 only for engines that fuse, see plan.fuse_k).
 cudaError_t step(const Plan& p, const double* src, double* dst, cudaStream_t s, int k = 1) {
+  if (p.ndim == 1) return launch_1d(p, src, dst, s, p.engine == LORA_ENGINE_DIRECT ? 1 : k);
   switch (p.engine) {
     case LORA_ENGINE_TC: return launch_tc2d(p, src, dst, s);
     case LORA_ENGINE_RDG_CUDA: return launch_rdg2d(p, src, dst, s, k);

@@ -28,6 +28,9 @@ cudaError_t launch_rdg3d(const Plan& p, const double* src, double* dst, cudaStre
 cudaError_t launch_tc3d(const Plan& p, const double* src, double* dst, cudaStream_t s);
 bool tc3d_supported(const Plan& p);
 
+// 1D stencils (kernels_1d.cu): one banded pass, k fused steps per launch.
+cudaError_t launch_1d(const Plan& p, const double* src, double* dst, cudaStream_t s, int k);
+
 bool tc2d_supported(const Plan& p);
 bool rdg3d_supported(const Plan& p);
 // Two fused 3D steps (radius 1), kernels_rdg3df.cu.

@@ -145,7 +145,17 @@ __global__ void copy_halo_kernel(const double* __restrict__ in, double* __restri
 
 }  // namespace
 
+__global__ void copy_halo_1d(const double* __restrict__ in, double* __restrict__ dst, int R, int64_t P0) {
+  const int i = threadIdx.x;
+  if (i < R) dst[i] = in[i];
+  else if (i < 2 * R) dst[P0 - 2 * R + i] = in[P0 - 2 * R + i];
+}
+
 cudaError_t launch_copy_halo(const Plan& p, const double* in, double* dst, cudaStream_t s) {
+  if (p.ndim == 1) {
+    copy_halo_1d<<<1, 32, 0, s>>>(in, dst, p.R, p.P[0]);
+    return cudaGetLastError();
+  }
   int64_t rows = p.ndim == 2 ? p.P[0] : p.P[0] * p.P[1];
   dim3 grid((unsigned)std::min<int64_t>(rows, 65535), (unsigned)((rows + 65534) / 65535));
   copy_halo_kernel<<<grid, 128, 0, s>>>(in, dst, p.ndim, p.R, p.P[0], p.P[1], p.P[2]);
@@ -171,6 +181,7 @@ static cudaError_t direct_r(const Plan& p, const double* src, double* dst, cudaS
 }
 
 cudaError_t launch_direct(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  if (p.ndim == 1) return launch_1d(p, src, dst, s, 1);
   switch (p.R) {
     case 1: return direct_r<1>(p, src, dst, s);
     case 2: return direct_r<2>(p, src, dst, s);

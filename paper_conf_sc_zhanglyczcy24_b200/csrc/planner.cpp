@@ -222,13 +222,13 @@ double cuda_fma_per_point(const Plan& p) {
 int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64_t* grid, const lora_plan_opts* o,
                std::string& err) {
   if (!weights || !grid) { err = "weights and grid_shape must be non-NULL"; return LORA_ERR_INVALID_ARG; }
-  if (ndim != 2 && ndim != 3) { err = "ndim must be 2 or 3"; return LORA_ERR_INVALID_ARG; }
+  if (ndim < 1 || ndim > 3) { err = "ndim must be 1, 2 or 3"; return LORA_ERR_INVALID_ARG; }
   if (radius < 1) { err = "radius must be >= 1"; return LORA_ERR_INVALID_ARG; }
   if (radius > kMaxRadius) { err = "radius > 4 is not supported (DESIGN.md Q14)"; return LORA_ERR_UNSUPPORTED; }
   for (int i = 0; i < ndim; ++i)
     if (grid[i] < 1) { err = "grid extents must be >= 1"; return LORA_ERR_INVALID_ARG; }
   const int n = 2 * radius + 1;
-  const size_t nw = ndim == 2 ? size_t(n) * n : size_t(n) * n * n;
+  const size_t nw = ndim == 1 ? size_t(n) : (ndim == 2 ? size_t(n) * n : size_t(n) * n * n);
   for (size_t i = 0; i < nw; ++i)
     if (!std::isfinite(weights[i])) { err = "weights must be finite"; return LORA_ERR_INVALID_ARG; }
   p.ndim = ndim; p.R = radius;
@@ -244,9 +244,20 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
   for (size_t i = 0; i < nw; ++i) { wmax = std::max(wmax, std::fabs(weights[i])); w1 += std::fabs(weights[i]); nnz += weights[i] != 0.0; }
   const double tol = 1e-15 * wmax;
   p.terms.clear();
-  const int nplanes = ndim == 2 ? 1 : n;
+  const int nplanes = ndim == 3 ? n : 1;
   p.z_symmetric = 0; p.n_planes_point = 0;
   for (int q = 0; q < nplanes; ++q) {
+    if (ndim == 1) {  // one banded gather: a horizontal arm u = e_R, v = w; or a point
+      int nz = 0, zj = 0;
+      for (int j = 0; j < n; ++j) if (weights[j] != 0.0) { ++nz; zj = j; }
+      if (nz == 0) break;
+      Term t; t.plane = 0; t.u[radius] = 1.0;
+      for (int j = 0; j < n; ++j) t.v[j] = weights[j];
+      t.kind = nz == 1 ? kPoint : kArm;
+      t.r = nz == 1 ? std::abs(zj - radius) : support_radius(t.v, n);
+      p.terms.push_back(t);
+      break;
+    }
     Mat P(n);
     for (int i = 0; i < n; ++i)
       for (int j = 0; j < n; ++j) P(i, j) = weights[size_t(q) * n * n + size_t(i) * n + j];
@@ -269,6 +280,10 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
     double nu = 0, nv = 0;
     for (int i = 0; i < n; ++i) { nu += std::fabs(t.u[i]); nv += std::fabs(t.v[i]); }
     g += nu * nv;
+    if (ndim == 1) {
+      for (int j = 0; j < n; ++j) Wr[j] += t.u[radius] * t.v[j];
+      continue;
+    }
     for (int i = 0; i < n; ++i)
       for (int j = 0; j < n; ++j) Wr[size_t(t.plane) * n * n + size_t(i) * n + j] += t.u[i] * t.v[j];
   }
@@ -289,10 +304,12 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
   // DMMA 37 TF, DFMA 34 TF, one shared FP64 budget).
   int eng = o ? o->engine : LORA_ENGINE_AUTO;
   if (eng < 0 || eng > LORA_ENGINE_DIRECT) { err = "unknown engine"; return LORA_ERR_INVALID_ARG; }
-  const double dense = p.ndim == 2 ? double(n) * n : double(n) * n * n;  // the direct kernel issues every tap
+  const double dense = p.ndim == 1 ? double(n) : (p.ndim == 2 ? double(n) * n : double(n) * n * n);  // every tap
   const double c_tc = tc_fma_per_point(p) / 37.0, c_rdg = cuda_fma_per_point(p) / 34.0, c_dir = dense / 34.0;
-  const bool ok_tc = tc2d_supported(p), ok_rdg = rdg2d_supported(p);
-  if (eng == LORA_ENGINE_AUTO) {
+  const bool ok_tc = p.ndim >= 2 && tc2d_supported(p), ok_rdg = p.ndim == 1 || rdg2d_supported(p);
+  if (eng == LORA_ENGINE_AUTO && p.ndim == 1) {
+    eng = LORA_ENGINE_RDG_CUDA;  // 1D: the banded pass with temporal fusion (HBM-bound)
+  } else if (eng == LORA_ENGINE_AUTO) {
     eng = LORA_ENGINE_DIRECT;
     double best = c_dir;
     if (ok_tc && c_tc < best) { best = c_tc; eng = LORA_ENGINE_TC; }
@@ -305,12 +322,12 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
   p.fma_issued = eng == LORA_ENGINE_TC ? tc_fma_per_point(p) : eng == LORA_ENGINE_RDG_CUDA ? cuda_fma_per_point(p) : dense;
   int fk = o ? o->fuse_k : 0;
   if (fk < 0) { err = "fuse_k must be >= 0"; return LORA_ERR_INVALID_ARG; }
-  const int max_k = eng == LORA_ENGINE_RDG_CUDA ? rdg2d_max_fuse(p) : 1;
+  const int max_k = eng != LORA_ENGINE_RDG_CUDA ? 1 : (p.ndim == 1 ? 8 : rdg2d_max_fuse(p));
   if (fk > max_k) { err = "fuse_k exceeds what the chosen engine supports for this stencil"; return LORA_ERR_UNSUPPORTED; }
   if (fk == 0) {
     // default fusion depth (exact temporal blocking): measured on B200
     static const int dflt[5] = {1, 3, 2, 1, 1};  // by radius; tools/quickbench.py, gpurun_out/qb6.jsonl
-    fk = std::min(max_k, p.ndim == 3 ? 2 : dflt[radius]);
+    fk = std::min(max_k, p.ndim == 3 ? 2 : (p.ndim == 1 ? 8 : dflt[radius]));
   }
   p.fuse_k = fk;
   {

@@ -114,6 +114,8 @@ def preset(name: str) -> np.ndarray:
     if name == "heat2d":  # 5-point star, c = 0.5, arms 0.125
         W = np.zeros((3, 3)); W[1, 1] = 0.5; W[0, 1] = W[2, 1] = W[1, 0] = W[1, 2] = 0.125
         return W
+    if name == "heat1d":  # 3-point, c = 0.5, arms 0.25
+        return np.array([0.25, 0.5, 0.25])
     if name == "heat3d":  # 7-point star, c = 0.25, arms 0.125
         W = np.zeros((3, 3, 3)); W[1, 1, 1] = 0.25
         for a in range(3):
@@ -180,6 +182,10 @@ CONFIGS = {
     "box3d27p-512": dict(id=4, ndim=3, radius=1, shape=(512, 512, 512), T=100, weights="rsym"),
     "box2d49p-40960": dict(id=5, ndim=2, radius=3, shape=(40960, 40960), T=100, weights="rsym"),
     "box3d27p-1024": dict(id=6, ndim=3, radius=1, shape=(1024, 1024, 1024), T=100, weights="rsym"),
+    # the remaining Table II kernels at BASELINE-like sizes
+    "star2d13p-10240": dict(id=7, ndim=2, radius=3, shape=(10240, 10240), T=100, weights="star"),
+    "heat1d-10240000": dict(id=8, ndim=1, radius=1, shape=(10240000,), T=100, weights="heat1d"),
+    "1d5p-10240000": dict(id=9, ndim=1, radius=2, shape=(10240000,), T=100, weights="rsym"),
 }
 
 
@@ -189,6 +195,8 @@ def config(name: str):
     c["seed"] = 20240101 + c["id"]
     if c["weights"] == "rsym":
         W = rsym_weights(c["ndim"], c["radius"], c["seed"])
+    elif c["weights"] == "star":
+        W = star_weights(c["ndim"], c["radius"], c["seed"])
     else:
         W = preset(c["weights"])
     c["padded"] = tuple(n + 2 * c["radius"] for n in c["shape"])

@@ -223,3 +223,27 @@ def test_3d_fusion_staging_paths_agree(monkeypatch):
     monkeypatch.setenv("LORA_NO_TMA", "1")
     b, _ = run_gpu(W, g, 4, engine="rdg_cuda", fuse_k=2)
     assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("h", [1, 2, 3, 4])
+@pytest.mark.parametrize("n", [1, 7, 1000, 4097, 100001])
+def test_1d_parity_and_fusion(h, n):
+    """1D (Table II Heat-1D / 1D5P): one banded pass; k fused steps per launch (halo
+    re-imposed) equal k single steps bitwise and the oracle to 1e-12."""
+    W = synth.rsym_weights(1, h, 50 + h)
+    g = synth.grid((n + 2 * h,), 60 + h)
+    for T in (1, 3, 8, 11):
+        a, info = run_gpu(W, g, T)               # planner default (fused)
+        b, _ = run_gpu(W, g, T, engine="rdg_cuda", fuse_k=1)
+        c, _ = run_gpu(W, g, T, engine="direct")
+        assert info["engine_name"] == "rdg_cuda" and info["fuse_k"] > 1
+        assert np.array_equal(a, b) and np.array_equal(b, c), T
+        assert rel_err(a, oracle.run(W, g, T)) <= 1e-12
+
+
+def test_star2d13p_arms():
+    W, c = synth.config("star2d13p-10240")
+    g = synth.grid((300 + 6, 257 + 6), 1)
+    for eng in ("auto", "tc", "direct"):
+        out, info = run_gpu(W, g, 4, engine=eng)
+        assert rel_err(out, oracle.run(W, g, 4)) <= 1e-12

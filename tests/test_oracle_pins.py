@@ -267,3 +267,36 @@ def test_rdg_pma_sum_equals_direct_eq9():
         acc += oracle.rdg_tile(u, v, Xs)
     ref = oracle.run(W, X, 1)[h:-h, h:-h]
     assert rel(acc, ref) <= 1e-14
+
+
+# ---------------------------------------------------------------- 1D (Table II Heat-1D / 1D5P)
+def test_1d_sine_eigenmode():
+    """Radius-1 or -2 symmetric 1D stencil with zero halo: A0 = sin(pi p x/(N+1)) (x = padded
+    index, radius-1 halo) is an eigenvector with lambda = sum_a w_a cos(pi p (a-1)/(N+1))."""
+    W = np.array([0.25, 0.5, 0.25]); N, p = 37, 3
+    A0 = np.sin(math.pi * p * np.arange(N + 2) / (N + 1)); A0[0] = A0[-1] = 0.0
+    lam = sum(W[a] * math.cos(math.pi * p * (a - 1) / (N + 1)) for a in range(3))
+    assert rel(oracle.run(W, A0, 20), lam ** 20 * A0) <= 1e-14
+
+
+def test_1d_plane_wave_and_bruteforce():
+    W = np.array([0.1, 0.2, 0.4, 0.2, 0.1])   # 1D5P-like
+    h, T, N = 2, 7, 80
+    theta = 0.13
+    g = np.cos(theta * np.arange(N + 2 * h))
+    lam = sum(W[a] * np.exp(1j * theta * (a - h)) for a in range(5))
+    out = oracle.run(W, g, T)
+    x = np.arange(N + 2 * h)
+    sl = slice(h + T * h, N + h - T * h)
+    assert rel(out[sl], np.real(lam ** T * np.exp(1j * theta * x))[sl]) <= 1e-13
+    g2 = synth.grid((N + 2 * h,), 5)
+    assert rel(oracle.run(W, g2, 3), _slicing_stencil(W, g2, 3)) <= 1e-14
+
+
+def test_1d_integer_exact():
+    W = np.array([1.0, 2.0, 1.0])
+    g = synth.integer_grid((50,), 3)
+    A = g.astype(np.int64)
+    for _ in range(20):
+        B = A.copy(); B[1:-1] = A[:-2] + 2 * A[1:-1] + A[2:]; A = B
+    assert np.array_equal(oracle.run(W, g, 20), A.astype(np.float64))
