@@ -278,7 +278,8 @@ def main():
     per_stencil = None
     if args.per_stencil and rank == 0 and world == 1:
         per_stencil = {}
-        for name in ("heat2d-256", "box2d9p-10240", "box2d49p-10240", "heat3d-512", "box3d27p-512"):
+        for name in ("heat2d-256", "box2d9p-10240", "box2d49p-10240", "heat3d-512", "box3d27p-512",
+                     "star2d13p-10240", "heat1d-10240000", "1d5p-10240000"):
             Wn, cn = synth.config(name)
             s2 = L.Stencil(Wn, cn["shape"], engine=args.engine)
             xa = torch.rand(cn["padded"], dtype=torch.float64, device=dev) + 0.5
