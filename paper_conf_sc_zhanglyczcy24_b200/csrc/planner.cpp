@@ -155,7 +155,7 @@ double tc_fma_per_point(const Plan& p) {
     const double K = 4.0 * std::ceil((8.0 + 2 * r) / 4.0);
     if (t.kind == kPoint) return 1.0;
     if (t.kind == kArm) return K;
-    return K * (8.0 * std::ceil((BN + 2 * r) / 8.0)) / BN + 16.0;
+    return K * (8.0 * std::ceil((BN + 2 * r) / 8.0)) / BN + (r <= 2 ? 12.0 : 16.0);  // grouped BVS for r <= 2
   };
   double f = 0;
   const int nplanes = p.ndim == 2 ? 1 : n;

@@ -46,6 +46,34 @@ __device__ __forceinline__ void chain_term(const double* __restrict__ X, int w, 
   double T[9][2];
 #pragma unroll
   for (int nb = 0; nb < 9; ++nb) { T[nb][0] = 0.0; T[nb][1] = 0.0; }
+  if constexpr (8 + 2 * HR <= 12) {
+    // Column-grouped BVS (HR <= 2): an 8-column output block needs 8 + 2HR <= 12 consecutive T
+    // columns, i.e. three groups of 4.  Stage 1 is free to choose which 8 tile columns form a T
+    // block (they are just the B-fragment addresses), so T block nb holds group 2nb (tile columns
+    // o + 8nb .. +3) in its even accumulator columns (R0) and group 2nb+1 (o + 8nb + 4 .. +7) in
+    // its odd ones (R1).  Output block ob then reads groups 2ob, 2ob+1, 2ob+2 = R0, R1 of block ob
+    // and R0 of block ob+1: 3 DMMAs instead of 4, still with no shuffle.
+    const int gc = (g & 1) ? 4 + (g >> 1) : (g >> 1);   // tile column of T column n = g in its block
+    const double* xr = X + (8 * w + o + t) * TC_PITCH + o + gc;
+#pragma unroll
+    for (int kk = 0; kk < KS; ++kk) {
+#pragma unroll
+      for (int nb = 0; nb < 9; ++nb) dmma(T[nb], a[kk], xr[4 * kk * TC_PITCH + 8 * nb]);
+    }
+    double vg[3];
+#pragma unroll
+    for (int j = 0; j < 3; ++j) {
+      const int c = 4 * j + o + t - g;   // tap of T column (group 2ob+j, slot t) for output column g
+      vg[j] = (c >= 0 && c <= 2 * R) ? tm.v[c] : 0.0;
+    }
+#pragma unroll
+    for (int ob = 0; ob < 8; ++ob) {
+      dmma(P[ob], T[ob][0], vg[0]);
+      dmma(P[ob], T[ob][1], vg[1]);
+      dmma(P[ob], T[ob + 1][0], vg[2]);
+    }
+    return;
+  }
   const double* xr = X + (8 * w + o + t) * TC_PITCH + g;
 #pragma unroll
   for (int kk = 0; kk < KS; ++kk) {
