@@ -16,8 +16,8 @@ __device__ __forceinline__ void tma2d(void* dst, const CUtensorMap* m, int x, in
                ::"r"(sa(dst)), "l"(m), "r"(x), "r"(y), "r"(sa(b)) : "memory"); }
 constexpr int R = 3, NS = 3, RC = 140;
 // W warps per CTA; each warp a 64-col band (BAND = 64) or the CTA a 64*W band read with boxes of width BW
-template <int W, bool COOP, int SROWS>
-__global__ void __launch_bounds__(W * 32) pat(const __grid_constant__ CUtensorMap map, double* out, int P1, int N0, int nbands, int nitems) {
+template <int W, bool COOP, int SROWS, bool TST = false>
+__global__ void __launch_bounds__(W * 32) pat(const __grid_constant__ CUtensorMap map, double* out, int P1, int N0, int nbands, int nitems, const __grid_constant__ CUtensorMap omap) {
   extern __shared__ __align__(128) unsigned char sm[];
   constexpr int BW = COOP ? 136 : 70;        // box width (doubles)
   constexpr int NB = COOP ? W / 2 : 1;       // boxes per stage (coop: one per warp pair)
@@ -61,15 +61,35 @@ __global__ void __launch_bounds__(W * 32) pat(const __grid_constant__ CUtensorMa
     const double* sb = st + (COOP ? (sub / 2) * BOXB / 8 : 0);
     const int cofs = COOP ? (sub % 2) * 64 : 0;
     const int col = (COOP ? band * 64 * W + sub * 64 : band * 64) + 2 * lane;
+    if constexpr (TST) {
+      // stage the 7 output rows (64 cols) in a per-warp smem buffer, then one TMA store
+      double* ob = reinterpret_cast<double*>(sm + 1024 + W * NS * STAGE) + wl * 2 * SROWS * 64 + (q & 1) * SROWS * 64;
+      if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+      __syncwarp();
+      for (int i = 0; i < SROWS; ++i) {
+        double2 v = *reinterpret_cast<const double2*>(sb + i * BW + cofs + 2 * lane + 2);
+        *reinterpret_cast<double2*>(ob + i * 64 + 2 * lane) = v;
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      __syncwarp();
+      const int y = chunk * RC + j * SROWS;
+      if (lane == 0) {
+        asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];"
+                     ::"l"(&omap), "r"(col + R + 1), "r"(y), "r"(sa(ob)) : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      }
+    } else {
     for (int i = 0; i < SROWS; ++i) {
       const int y = chunk * RC + j * SROWS + i - R;   // "output" row
       double2 v = *reinterpret_cast<const double2*>(sb + i * BW + cofs + 2 * lane + 2);
       if (y >= chunk * RC && y < chunk * RC + RC && y < N0)
         *reinterpret_cast<double2*>(out + int64_t(y + R) * P1 + R + col + 1) = v;
     }
+    }
     __syncwarp();
     if (COOP && lane == 0) arrive(&empty[q % NS]);
   }
+  if constexpr (TST) { if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 }
 __global__ void plain_copy(const double2* __restrict__ a, double2* __restrict__ b, size_t n) {
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) b[i] = a[i];
@@ -77,7 +97,7 @@ __global__ void plain_copy(const double2* __restrict__ a, double2* __restrict__ 
 using EncodeFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*, const cuuint64_t*,
                               const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
                               CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-template <int W, bool COOP, int SROWS>
+template <int W, bool COOP, int SROWS, bool TST = false>
 int run(EncodeFn enc, double* a, double* b, int P, const char* name) {
   constexpr int BW = COOP ? 136 : 70;
   CUtensorMap map;
@@ -85,20 +105,24 @@ int run(EncodeFn enc, double* a, double* b, int P, const char* name) {
   cuuint32_t box[2] = {BW, SROWS}, es[2] = {1, 1};
   enc(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, a, dims, str, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
       CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  CUtensorMap omap;
+  cuuint32_t obox[2] = {64, SROWS};
+  enc(&omap, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, b, dims, str, obox, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+      CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   const int N = P - 2 * R;
   const int nbands = (N + (COOP ? 64 * W : 64) - 1) / (COOP ? 64 * W : 64);
   const int nitems = nbands * ((N + RC - 1) / RC);
   constexpr int STAGE = ((SROWS * BW * 8 + 127) / 128) * 128 * (COOP ? W / 2 : 1);
-  const int smem = 1024 + (COOP ? 1 : W) * NS * STAGE;
-  CK(cudaFuncSetAttribute(pat<W, COOP, SROWS>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-  int occ = 0; cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, pat<W, COOP, SROWS>, W * 32, smem);
+  const int smem = 1024 + (COOP ? 1 : W) * NS * STAGE + (TST ? W * 2 * SROWS * 64 * 8 : 0);
+  CK(cudaFuncSetAttribute(pat<W, COOP, SROWS, TST>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  int occ = 0; cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, pat<W, COOP, SROWS, TST>, W * 32, smem);
   const int units = COOP ? nitems : (nitems + W - 1) / W;
   const int grid = std::min(148 * occ, units);
   cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
-  pat<W, COOP, SROWS><<<grid, W * 32, smem>>>(map, b, P, N, nbands, nitems);
+  pat<W, COOP, SROWS, TST><<<grid, W * 32, smem>>>(map, b, P, N, nbands, nitems, omap);
   CK(cudaDeviceSynchronize());
   float best = 1e9;
-  for (int r = 0; r < 5; ++r) { cudaEventRecord(e0); pat<W, COOP, SROWS><<<grid, W * 32, smem>>>(map, b, P, N, nbands, nitems); cudaEventRecord(e1);
+  for (int r = 0; r < 5; ++r) { cudaEventRecord(e0); pat<W, COOP, SROWS, TST><<<grid, W * 32, smem>>>(map, b, P, N, nbands, nitems, omap); cudaEventRecord(e1);
     CK(cudaEventSynchronize(e1)); float ms; cudaEventElapsedTime(&ms, e0, e1); best = std::min(best, ms); }
   printf("{\"pattern\":\"%s\",\"srows\":%d,\"occ\":%d,\"grid\":%d,\"GBps\":%.0f}\n", name, SROWS, occ, grid, 2.0 * double(N) * N * 8 / best / 1e6);
   return 0;
@@ -112,12 +136,9 @@ int main() {
   double *a, *b; CK(cudaMalloc(&a, (size_t)P * P * 8)); CK(cudaMalloc(&b, (size_t)P * P * 8));
   cudaMemset(a, 0, (size_t)P * P * 8);
   run<4, false, 7>(enc, a, b, P, "warp64_x4");
-  run<4, false, 14>(enc, a, b, P, "warp64_x4");
-  run<4, false, 21>(enc, a, b, P, "warp64_x4");
-  run<8, true, 7>(enc, a, b, P, "cta512_w8");
-  run<8, true, 14>(enc, a, b, P, "cta512_w8");
-  run<4, true, 14>(enc, a, b, P, "cta256_w4");
-  run<4, true, 28>(enc, a, b, P, "cta256_w4");
+  run<4, false, 7, true>(enc, a, b, P, "warp64_x4_tmastore");
+  run<4, false, 14, true>(enc, a, b, P, "warp64_x4_tmastore");
+  run<8, false, 7, true>(enc, a, b, P, "warp64_x8_tmastore");
   size_t n = (size_t)P * P / 2;
   cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
   float best = 1e9;
