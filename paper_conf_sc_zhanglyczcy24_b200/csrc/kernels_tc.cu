@@ -35,7 +35,7 @@ using namespace tc;
 
 // Persistent CTAs walk the 64x64 output tiles; tile i+1 is staged (TMA + mbarrier, or LDGSTS when
 // TMA's 16-byte pitch rule fails) while tile i is computed.
-template <int R, bool TMA>
+template <int R, bool TMA, bool NOBVS>
 __global__ void __launch_bounds__(256, 2) tc2d_kernel(const double* __restrict__ in, double* __restrict__ out,
                                                       int64_t N0, int64_t N1, int ntx, int ntiles,
                                                       const __grid_constant__ CUtensorMap tmap,
@@ -84,7 +84,7 @@ __global__ void __launch_bounds__(256, 2) tc2d_kernel(const double* __restrict__
     }
     const double* X = buf0 + b * BUF;
     double P[8][2];
-    tc_tile<R>(X, w, g, t, prm, P);
+    tc_tile<R, NOBVS>(X, w, g, t, prm, P);
     const int64_t y0 = int64_t(tile / ntx) * TC_BM, x0 = int64_t(tile % ntx) * TC_BN;
     const int64_t gy = y0 + 8 * w + g;
     if (gy < N0) {
@@ -123,7 +123,7 @@ TcParams make_params(const Plan& p) {
   return prm;
 }
 
-template <int R, bool TMA>
+template <int R, bool TMA, bool NOBVS>
 cudaError_t tc_launch(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map) {
   constexpr int SH = tc_rows<R>();
   constexpr size_t BUF = ((SH * TC_PITCH * 8 + 127) / 128) * 128;
@@ -132,13 +132,13 @@ cudaError_t tc_launch(const Plan& p, const double* src, double* dst, cudaStream_
   const int64_t ntiles = int64_t(ntx) * nty;
   static int max_grid = 0;
   if (max_grid == 0) {
-    cudaError_t e = cudaFuncSetAttribute(tc2d_kernel<R, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(tc2d_kernel<R, TMA, NOBVS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    max_grid = persistent_grid((const void*)tc2d_kernel<R, TMA>, 256, smem, int64_t(1) << 40);
+    max_grid = persistent_grid((const void*)tc2d_kernel<R, TMA, NOBVS>, 256, smem, int64_t(1) << 40);
   }
   const int grid = (int)std::min<int64_t>(max_grid, ntiles);
   const TcParams prm = make_params(p);
-  tc2d_kernel<R, TMA><<<grid, 256, smem, s>>>(src, dst, p.N[0], p.N[1], ntx, (int)ntiles, map, prm);
+  tc2d_kernel<R, TMA, NOBVS><<<grid, 256, smem, s>>>(src, dst, p.N[0], p.N[1], ntx, (int)ntiles, map, prm);
   return cudaGetLastError();
 }
 
@@ -147,9 +147,11 @@ cudaError_t tc_r(const Plan& p, const double* src, double* dst, cudaStream_t s) 
   CUtensorMap map;
   const int64_t padded[2] = {p.P[0], p.P[1]};
   const int box[2] = {tc_rows<R>(), TC_PITCH};
-  if (!p.force_no_tma && encode_tmap(&map, src, 2, padded, box)) return tc_launch<R, true>(p, src, dst, s, map);
-  std::memset(&map, 0, sizeof(map));
-  return tc_launch<R, false>(p, src, dst, s, map);
+  const bool tma = !p.force_no_tma && encode_tmap(&map, src, 2, padded, box);
+  if (!tma) std::memset(&map, 0, sizeof(map));
+  if (p.tc_no_bvs)  // Fig. 9 ablation only (LORA_TC_NO_BVS=1): separate instantiation, shuffles in stage 2
+    return tma ? tc_launch<R, true, true>(p, src, dst, s, map) : tc_launch<R, false, true>(p, src, dst, s, map);
+  return tma ? tc_launch<R, true, false>(p, src, dst, s, map) : tc_launch<R, false, false>(p, src, dst, s, map);
 }
 
 }  // namespace

@@ -34,7 +34,8 @@ struct Plan {
   int fuse_k = 1;
   int tile_m = 0, tile_n = 0;
   int z_symmetric = 0;
-  int force_no_tma = 0;   // LORA_NO_TMA=1: use the LDGSTS staging path (tests both loaders)
+  int force_no_tma = 0;
+  int tc_no_bvs = 0;      // LORA_TC_NO_BVS=1: the Fig. 9 ablation (shuffle-based stage 2) in the TC engine   // LORA_NO_TMA=1: use the LDGSTS staging path (tests both loaders)
   int n_planes_point = 0;
   double recon_err = 0, growth = 0;
   double fma_issued = 0, fma_direct = 0, fma_separable = 0;

@@ -32,7 +32,7 @@ template <int R>
 __host__ __device__ constexpr int tc_rows() { return TC_BM + 2 * R + 4; }
 
 // u/v are centred length 2R+1; a term of radius HR lives in [R-HR, R+HR].
-template <int R, int HR>
+template <int R, int HR, bool NOBVS = false>
 __device__ __forceinline__ void chain_term(const double* __restrict__ X, int w, int g, int t, const TcTerm& tm,
                                            double (&P)[8][2]) {
   constexpr int K1 = ((8 + 2 * HR + 3) / 4) * 4, KS = K1 / 4;
@@ -46,6 +46,43 @@ __device__ __forceinline__ void chain_term(const double* __restrict__ X, int w, 
   double T[9][2];
 #pragma unroll
   for (int nb = 0; nb < 9; ++nb) { T[nb][0] = 0.0; T[nb][1] = 0.0; }
+  if constexpr (NOBVS) {
+    // Ablation "TC RDG without BVS" (Fig. 9): T keeps its natural column order and
+    // the stage-2 A fragment A[g][t] = T[g][4h + t] is gathered from the C layout of lane
+    // (g, 2h + t/2), register t % 2, with warp shuffles (4 SHFL.32 per fragment).
+    const double* xr = X + (8 * w + o + t) * TC_PITCH + g;
+#pragma unroll
+    for (int kk = 0; kk < KS; ++kk) {
+#pragma unroll
+      for (int nb = 0; nb < 9; ++nb) dmma(T[nb], a[kk], xr[4 * kk * TC_PITCH + 8 * nb]);
+    }
+    double af[9][2];
+#pragma unroll
+    for (int nb = 0; nb < 9; ++nb)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int src = 4 * g + 2 * h + (t >> 1);
+        const double v0 = __shfl_sync(0xffffffffu, T[nb][0], src);
+        const double v1 = __shfl_sync(0xffffffffu, T[nb][1], src);
+        af[nb][h] = (t & 1) ? v1 : v0;
+      }
+    double vn[2][2];
+#pragma unroll
+    for (int j = 0; j < 2; ++j)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int c = 8 * j + 4 * h + t - g;
+        vn[j][h] = (c >= 0 && c <= 2 * R) ? tm.v[c] : 0.0;
+      }
+#pragma unroll
+    for (int ob = 0; ob < 8; ++ob) {
+      dmma(P[ob], af[ob][0], vn[0][0]);
+      dmma(P[ob], af[ob][1], vn[0][1]);
+      dmma(P[ob], af[ob + 1][0], vn[1][0]);
+      dmma(P[ob], af[ob + 1][1], vn[1][1]);
+    }
+    return;
+  }
   if constexpr (8 + 2 * HR <= 12) {
     // Column-grouped BVS (HR <= 2): an 8-column output block needs 8 + 2HR <= 12 consecutive T
     // columns, i.e. three groups of 4.  Stage 1 is free to choose which 8 tile columns form a T
@@ -149,19 +186,19 @@ __device__ __forceinline__ void point_term(const double* __restrict__ X, int w, 
 
 
 // Accumulates terms k0 .. k1-1 of prm into P (eq. 9: the sum of the rank-1 chains).
-template <int R>
+template <int R, bool NOBVS = false>
 __device__ __forceinline__ void apply_terms(const double* __restrict__ X, int w, int g, int t, const TcParams& prm,
                                             int k0, int k1, double (&P)[8][2]) {
   for (int k = k0; k < k1; ++k) {
     const TcTerm& tm = prm.t[k];
     switch (tm.kind) {
       case 0:
-        if (tm.r == 1) chain_term<R, 1>(X, w, g, t, tm, P);
+        if (tm.r == 1) chain_term<R, 1, NOBVS>(X, w, g, t, tm, P);
         else if constexpr (R >= 2) {
-          if (tm.r == 2) chain_term<R, (R >= 2 ? 2 : 1)>(X, w, g, t, tm, P);
+          if (tm.r == 2) chain_term<R, (R >= 2 ? 2 : 1), NOBVS>(X, w, g, t, tm, P);
           else if constexpr (R >= 3) {
-            if (tm.r == 3) chain_term<R, (R >= 3 ? 3 : 1)>(X, w, g, t, tm, P);
-            else if constexpr (R >= 4) chain_term<R, 4>(X, w, g, t, tm, P);
+            if (tm.r == 3) chain_term<R, (R >= 3 ? 3 : 1), NOBVS>(X, w, g, t, tm, P);
+            else if constexpr (R >= 4) chain_term<R, 4, NOBVS>(X, w, g, t, tm, P);
           }
         }
         break;
@@ -192,12 +229,12 @@ __device__ __forceinline__ void apply_terms(const double* __restrict__ X, int w,
 }
 
 
-template <int R>
+template <int R, bool NOBVS = false>
 __device__ __forceinline__ void tc_tile(const double* __restrict__ X, int w, int g, int t, const TcParams& prm,
                                         double (&P)[8][2]) {
 #pragma unroll
   for (int ob = 0; ob < 8; ++ob) { P[ob][0] = 0.0; P[ob][1] = 0.0; }
-  apply_terms<R>(X, w, g, t, prm, 0, prm.nterms, P);
+  apply_terms<R, NOBVS>(X, w, g, t, prm, 0, prm.nterms, P);
 }
 
 }  // namespace tc

@@ -247,3 +247,16 @@ def test_star2d13p_arms():
     for eng in ("auto", "tc", "direct"):
         out, info = run_gpu(W, g, 4, engine=eng)
         assert rel_err(out, oracle.run(W, g, 4)) <= 1e-12
+
+
+@pytest.mark.parametrize("h", [1, 2, 3])
+def test_tc_without_bvs_ablation_parity(h, monkeypatch):
+    """The Fig. 9 ablation variant (stage-2 A fragments gathered with shuffles, no BVS) computes
+    the same chains: matches the oracle and the BVS kernel to rounding."""
+    W = synth.rsym_weights(2, h, 90 + h)
+    g = synth.grid((130 + 2 * h, 70 + 2 * h), 91)
+    a, _ = run_gpu(W, g, 3, engine="tc")
+    monkeypatch.setenv("LORA_TC_NO_BVS", "1")
+    b, _ = run_gpu(W, g, 3, engine="tc")
+    ref = oracle.run(W, g, 3)
+    assert rel_err(b, ref) <= 1e-12 and rel_err(a, b) <= 1e-13
