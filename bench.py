@@ -44,6 +44,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-engines", action="store_true", help="skip the per-engine comparison on the workload")
+    ap.add_argument("--force-dist", action="store_true",
+                    help="use lora_stencil_run_dist even on one rank (exercises the slab path; LORA_DIST_SPLIT=1 "
+                         "additionally forces the overlapped edge/interior split)")
     return ap.parse_args()
 
 
@@ -204,11 +207,15 @@ def main():
     st = L.Stencil(W, shape, engine=args.engine, fuse_k=args.fuse)
     info = st.info()
     comm = None
-    if world > 1:
-        uid = L.lora_stencil_comm_get_id() if rank == 0 else None
-        obj = [uid]
-        dist.broadcast_object_list(obj, src=0)
-        comm = L.lora_stencil_comm_init(world, rank, obj[0])
+    if world > 1 or args.force_dist:
+        if world > 1:
+            uid = L.lora_stencil_comm_get_id() if rank == 0 else None
+            obj = [uid]
+            dist.broadcast_object_list(obj, src=0)
+            uid = obj[0]
+        else:
+            uid = b"\0" * L.lora_stencil_comm_id_size()
+        comm = L.lora_stencil_comm_init(world, rank, uid)
 
     # seeded synthetic input (SplitMix64 over the padded array; each rank its own seed offset)
     g = synth.grid(padded, cfg["seed"] + 1000 * rank)
@@ -336,7 +343,7 @@ def main():
                 "config": {"workload": args.workload, "grid_per_rank": list(shape), "T": T, "radius": h,
                            "ndim": cfg["ndim"], "global_grid": [shape[0] * world] + list(shape[1:]),
                            "engine": info["engine_name"], "fuse_k": fuse, "n_terms": info["n_terms"],
-                           "parallelism": f"slab{world}" if world > 1 else "single",
+                           "parallelism": f"slab{world}" if comm is not None else "single",
                            "l2": "inputs (%.2f GB per buffer) larger than the 126 MB L2" % (8 * np.prod(padded) / 1e9)},
                 "clocks": clk.summary(), "gpu_launches": launches_per_step * args.steps,
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
