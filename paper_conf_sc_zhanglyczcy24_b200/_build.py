@@ -11,10 +11,10 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
-LIB = os.path.join(PKG, "liblora_stencil.so")
+LIB = os.environ.get("LORA_LIB_OUT", os.path.join(PKG, "liblora_stencil.so"))   # experiments: variant builds
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-FLAGS = ["-O3", "-lineinfo", "-std=c++20", "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC,-O2",
+FLAGS = [*os.environ.get("LORA_NVCC_EXTRA", "").split(), "-O3", "-lineinfo", "-std=c++20", "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC,-O2",
          "-I" + INCLUDE, "-I" + CSRC]
 
 
@@ -31,7 +31,7 @@ def _stale(out, deps):
 
 def build(force: bool = False, verbose: bool = False, jobs: int = 8) -> str:
     headers = glob.glob(os.path.join(CSRC, "*.hpp")) + glob.glob(os.path.join(INCLUDE, "*.h"))
-    objdir = os.path.join(PKG, "build")
+    objdir = os.path.join(PKG, os.environ.get("LORA_BUILD_DIR", "build"))
     os.makedirs(objdir, exist_ok=True)
     objs, cmds = [], []
     for src in sources():
