@@ -327,8 +327,15 @@ def main():
             ts = a0.elapsed_time(a1) / 2e3
             gs = float(np.prod(shape)) * T / ts / 1e9
             i3 = s3.info()
+            # issued FP64 rate against the measured FP64 pipe peak (step-0 microbenchmark, DESIGN.md §5:
+            # DMMA 36.9 TF, DFMA 33.8 TF; profiles/r01_step0_fp64_pipes.jsonl)
+            fp64_peak = 36.9e12 if eng == "tc" else 33.8e12
+            issued_tf = gs * 1e9 * i3["fma_per_point_issued"] * 2
             engines[eng] = {"GStencil_s": gs, "frac_hbm_roofline": gs / (peak / BYTES_PER_POINT), "fuse_k": i3["fuse_k"],
-                            "fma_per_point_issued": i3["fma_per_point_issued"], "ms_per_step": ts * 1e3}
+                            "fma_per_point_issued": i3["fma_per_point_issued"], "ms_per_step": ts * 1e3,
+                            "issued_fp64_tflops": issued_tf / 1e12,
+                            "frac_fp64_pipe_peak": issued_tf / fp64_peak,
+                            "fp64_pipe": "DMMA (tensor)" if eng == "tc" else "DFMA"}
             s3.close()
 
     cpu = None

@@ -30,7 +30,8 @@ def _stale(out, deps):
 
 
 def build(force: bool = False, verbose: bool = False, jobs: int = 8) -> str:
-    headers = glob.glob(os.path.join(CSRC, "*.hpp")) + glob.glob(os.path.join(INCLUDE, "*.h"))
+    headers = (glob.glob(os.path.join(CSRC, "*.hpp")) + glob.glob(os.path.join(CSRC, "*.cuh")) +
+               glob.glob(os.path.join(INCLUDE, "*.h")))
     objdir = os.path.join(PKG, os.environ.get("LORA_BUILD_DIR", "build"))
     os.makedirs(objdir, exist_ok=True)
     objs, cmds = [], []

@@ -90,7 +90,10 @@ __device__ __forceinline__ void chain_term(const double* __restrict__ X, int w, 
     // o + 8nb .. +3) in its even accumulator columns (R0) and group 2nb+1 (o + 8nb + 4 .. +7) in
     // its odd ones (R1).  Output block ob then reads groups 2ob, 2ob+1, 2ob+2 = R0, R1 of block ob
     // and R0 of block ob+1: 3 DMMAs instead of 4, still with no shuffle.
-    const int gc = (g & 1) ? 4 + (g >> 1) : (g >> 1);   // tile column of T column n = g in its block
+    // The odd group's slots are additionally rotated, slot t <-> group column (t + 2) mod 4 (another
+    // eq. 17 permutation, undone in V'), so that each half-warp's 16 B-fragment addresses stay distinct
+    // mod 16 doubles with the 76-double pitch: bank-conflict free, like the ungrouped layout.
+    const int gc = (g & 1) ? 4 + (((g >> 1) + 2) & 3) : (g >> 1);   // tile column of T column n = g
     const double* xr = X + (8 * w + o + t) * TC_PITCH + o + gc;
 #pragma unroll
     for (int kk = 0; kk < KS; ++kk) {
@@ -100,7 +103,8 @@ __device__ __forceinline__ void chain_term(const double* __restrict__ X, int w, 
     double vg[3];
 #pragma unroll
     for (int j = 0; j < 3; ++j) {
-      const int c = 4 * j + o + t - g;   // tap of T column (group 2ob+j, slot t) for output column g
+      const int slot = (j == 1) ? ((t + 2) & 3) : t;   // group column held in A slot t
+      const int c = 4 * j + o + slot - g;              // its tap for output column g
       vg[j] = (c >= 0 && c <= 2 * R) ? tm.v[c] : 0.0;
     }
 #pragma unroll
