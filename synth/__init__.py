@@ -25,7 +25,7 @@ import numpy as np
 __all__ = [
     "splitmix64", "uniform_from_index", "grid", "rsym_weights", "star_weights", "preset",
     "CONFIGS", "config", "integer_pyramid_weights", "integer_grid", "asym_weights",
-    "constant_grid", "sine_grid", "plane_wave_grid", "dyadic_box_weights",
+    "constant_grid", "sine_grid", "plane_wave_grid", "dyadic_box_weights", "grid_torch",
 ]
 
 _GAMMA = np.uint64(0x9E3779B97F4A7C15)
@@ -66,6 +66,36 @@ def _classes(ndim: int, radius: int, star: bool):
     if star:
         cls = [c for c in cls if sum(1 for x in c if x) <= 1]
     return cls
+
+
+def grid_torch(padded_shape, seed: int, device="cuda", chunk: int = 1 << 26):
+    """The same SplitMix64 grid as `grid`, generated with torch int64 arithmetic on `device`
+    (bit-identical: int64 multiply wraps like uint64; logical shifts are emulated with masks).
+    For grids too large to build on the host."""
+    import torch
+    n = 1
+    for d in padded_shape:
+        n *= int(d)
+    out = torch.empty(n, dtype=torch.float64, device=device)
+
+    def u64(x):  # python int -> int64 with the same bits
+        x &= (1 << 64) - 1
+        return x - (1 << 64) if x >= 1 << 63 else x
+
+    gamma, m1, m2 = u64(0x9E3779B97F4A7C15), u64(0xBF58476D1CE4E5B9), u64(0x94D049BB133111EB)
+
+    def lsr(z, k):
+        return (z >> k) & ((1 << (64 - k)) - 1)
+
+    for s in range(0, n, chunk):
+        e = min(n, s + chunk)
+        i = torch.arange(s, e, dtype=torch.int64, device=device)
+        z = u64(seed) + (i + 1) * gamma
+        z = (z ^ lsr(z, 30)) * m1
+        z = (z ^ lsr(z, 27)) * m2
+        z = z ^ lsr(z, 31)
+        out[s:e] = 0.5 + lsr(z, 11).to(torch.float64) * (2.0 ** -53)
+    return out.view(*[int(d) for d in padded_shape])
 
 
 def rsym_weights(ndim: int, radius: int, seed: int, star: bool = False) -> np.ndarray:

@@ -36,3 +36,9 @@ def test_rsym_weights_symmetry_and_normalisation():
 
 def test_presets_sum_to_one():
     assert synth.preset("heat2d").sum() == 1.0 and synth.preset("heat3d").sum() == 1.0
+
+
+def test_grid_torch_is_bit_identical():
+    import torch
+    g = synth.grid_torch((37, 41), 20240101, device="cpu", chunk=100).numpy()
+    assert np.array_equal(g, synth.grid((37, 41), 20240101))
