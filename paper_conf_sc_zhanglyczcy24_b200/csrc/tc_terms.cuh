@@ -22,8 +22,10 @@ struct TcParams {
 
 constexpr int TC_BM = 64, TC_BN = 64, TC_PITCH = 76;
 
+// Not `volatile`: the compiler may interleave independent DMMAs (a volatile asm pins program order,
+// which turned the per-block stage-2 accumulation into a dependent chain).
 __device__ __forceinline__ void dmma(double (&c)[2], double a, double b) {
-  asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+  asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
                : "+d"(c[0]), "+d"(c[1])
                : "d"(a), "d"(b));
 }
@@ -75,12 +77,13 @@ __device__ __forceinline__ void chain_term(const double* __restrict__ X, int w, 
         vn[j][h] = (c >= 0 && c <= 2 * R) ? tm.v[c] : 0.0;
       }
 #pragma unroll
-    for (int ob = 0; ob < 8; ++ob) {
-      dmma(P[ob], af[ob][0], vn[0][0]);
-      dmma(P[ob], af[ob][1], vn[0][1]);
-      dmma(P[ob], af[ob + 1][0], vn[1][0]);
-      dmma(P[ob], af[ob + 1][1], vn[1][1]);
-    }
+    for (int ob = 0; ob < 8; ++ob) dmma(P[ob], af[ob][0], vn[0][0]);
+#pragma unroll
+    for (int ob = 0; ob < 8; ++ob) dmma(P[ob], af[ob][1], vn[0][1]);
+#pragma unroll
+    for (int ob = 0; ob < 8; ++ob) dmma(P[ob], af[ob + 1][0], vn[1][0]);
+#pragma unroll
+    for (int ob = 0; ob < 8; ++ob) dmma(P[ob], af[ob + 1][1], vn[1][1]);
     return;
   }
   if constexpr (8 + 2 * HR <= 12) {
@@ -108,11 +111,11 @@ __device__ __forceinline__ void chain_term(const double* __restrict__ X, int w, 
       vg[j] = (c >= 0 && c <= 2 * R) ? tm.v[c] : 0.0;
     }
 #pragma unroll
-    for (int ob = 0; ob < 8; ++ob) {
-      dmma(P[ob], T[ob][0], vg[0]);
-      dmma(P[ob], T[ob][1], vg[1]);
-      dmma(P[ob], T[ob + 1][0], vg[2]);
-    }
+    for (int ob = 0; ob < 8; ++ob) dmma(P[ob], T[ob][0], vg[0]);     // pass-major: consecutive DMMAs
+#pragma unroll                                                       // hit different accumulators
+    for (int ob = 0; ob < 8; ++ob) dmma(P[ob], T[ob][1], vg[1]);
+#pragma unroll
+    for (int ob = 0; ob < 8; ++ob) dmma(P[ob], T[ob + 1][0], vg[2]);
     return;
   }
   const double* xr = X + (8 * w + o + t) * TC_PITCH + g;
@@ -130,12 +133,13 @@ __device__ __forceinline__ void chain_term(const double* __restrict__ X, int w, 
       vb[j][i] = (c >= 0 && c <= 2 * R) ? tm.v[c] : 0.0;
     }
 #pragma unroll
-  for (int ob = 0; ob < 8; ++ob) {
-    dmma(P[ob], T[ob][0], vb[0][0]);
-    dmma(P[ob], T[ob][1], vb[0][1]);
-    dmma(P[ob], T[ob + 1][0], vb[1][0]);
-    dmma(P[ob], T[ob + 1][1], vb[1][1]);
-  }
+  for (int ob = 0; ob < 8; ++ob) dmma(P[ob], T[ob][0], vb[0][0]);
+#pragma unroll
+  for (int ob = 0; ob < 8; ++ob) dmma(P[ob], T[ob][1], vb[0][1]);
+#pragma unroll
+  for (int ob = 0; ob < 8; ++ob) dmma(P[ob], T[ob + 1][0], vb[1][0]);
+#pragma unroll
+  for (int ob = 0; ob < 8; ++ob) dmma(P[ob], T[ob + 1][1], vb[1][1]);
 }
 
 // Horizontal arm (u = e_R): P[g][n] += sum_c X[8w+g+R][8ob+c] v[c-n]; A from smem, B = band of v.
@@ -152,9 +156,9 @@ __device__ __forceinline__ void harm_term(const double* __restrict__ X, int w, i
   }
   const double* xr = X + (8 * w + g + R) * TC_PITCH + o + t;
 #pragma unroll
-  for (int ob = 0; ob < 8; ++ob)
+  for (int kk = 0; kk < KS; ++kk)
 #pragma unroll
-    for (int kk = 0; kk < KS; ++kk) dmma(P[ob], xr[8 * ob + 4 * kk], b[kk]);
+    for (int ob = 0; ob < 8; ++ob) dmma(P[ob], xr[8 * ob + 4 * kk], b[kk]);
 }
 
 // Vertical arm (v = e_R): P[g][n] += sum_k U[g][k] X[8w+o+k][8ob+n+R].
@@ -171,9 +175,9 @@ __device__ __forceinline__ void varm_term(const double* __restrict__ X, int w, i
   }
   const double* xr = X + (8 * w + o + t) * TC_PITCH + g + R;
 #pragma unroll
-  for (int ob = 0; ob < 8; ++ob)
+  for (int kk = 0; kk < KS; ++kk)
 #pragma unroll
-    for (int kk = 0; kk < KS; ++kk) dmma(P[ob], a[kk], xr[4 * kk * TC_PITCH + 8 * ob]);
+    for (int ob = 0; ob < 8; ++ob) dmma(P[ob], a[kk], xr[4 * kk * TC_PITCH + 8 * ob]);
 }
 
 template <int R>
