@@ -162,7 +162,7 @@ struct LaneCtx {
 
 template <int R, int SIG, int K, int I0, int I, int S>
 __device__ __forceinline__ void fused_stage(const double* __restrict__ src, int p, double (&acc)[K][2 * R + 1][2],
-                                            const RdgParams& P, double* const* __restrict__ bufs, int par,
+                                            const RdgParams& P, double* __restrict__ bufs, int par,
                                             const double* __restrict__ in, double* __restrict__ out, int64_t P1,
                                             const StageCtx<K>& sc, const LaneCtx& lc) {
   constexpr int n = 2 * R + 1;
@@ -186,7 +186,8 @@ __device__ __forceinline__ void fused_stage(const double* __restrict__ src, int 
       if (!lc.inside0) v0 = 0.0;
       if (!lc.inside1) v1 = 0.0;
     }
-    double* b = bufs[2 * (S - 1) + par];
+    constexpr int BUFD = ((Geom<R>::BW + 15) / 16) * 16;
+    double* b = bufs + (2 * (S - 1) + par) * BUFD;   // [stage][parity] row buffers (no local-memory pointer table)
     b[R + 2 * p] = v0;
     b[R + 2 * p + 1] = v1;
     __syncwarp();
@@ -206,7 +207,7 @@ __device__ __forceinline__ void fused_stage(const double* __restrict__ src, int 
 
 template <int R, int SIG, int K, int I>
 __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p, double (&acc)[K][2 * R + 1][2],
-                                           const RdgParams& P, double* const* __restrict__ bufs,
+                                           const RdgParams& P, double* __restrict__ bufs,
                                            const double* __restrict__ in, double* __restrict__ out, int64_t P1,
                                            const StageCtx<K>& sc, const LaneCtx& lc, int par0) {
   constexpr int n = 2 * R + 1;
@@ -233,9 +234,7 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (K == 1 || R == 1) ? 4 : 3) rd
   unsigned char* wbase = smem_raw + 128 + wl * (G::WARP_BYTES + 2 * (K - 1) * BUFD * 8);
   unsigned char* ring = wbase;
   double* bufmem = reinterpret_cast<double*>(wbase + G::WARP_BYTES);
-  double* bufs[2 * K];                          // [stage][parity]
-#pragma unroll
-  for (int i = 0; i < 2 * (K - 1); ++i) bufs[i] = bufmem + i * BUFD;
+  double* bufs = bufmem;                        // [stage][parity] rows of BUFD doubles
   for (int i = lane; i < 2 * (K - 1) * BUFD; i += 32) bufmem[i] = 0.0;  // margins stay zero
   const int64_t P1 = N1 + 2 * R;
   const int P0 = (int)(N0 + 2 * R);
