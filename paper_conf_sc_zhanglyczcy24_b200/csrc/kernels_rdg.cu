@@ -219,8 +219,14 @@ __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p,
   }
 }
 
+#ifndef RDG_MINB_ALL
+#define RDG_MINB_ALL 0   // experiments: force resident CTAs per SM for every instantiation
+#endif
+template <int R, int K>
+constexpr int rdg_minb() { return (RDG_MINB_ALL > 0) ? RDG_MINB_ALL : ((K == 1 || R == 1) ? 4 : 3); }
+
 template <int R, int SIG, int K, bool TMA>
-__global__ void __launch_bounds__(RDG_WARPS * 32, (K == 1 || R == 1) ? 4 : 3) rdg2d_kernel(const double* __restrict__ in, double* __restrict__ out,
+__global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, K>())) rdg2d_kernel(const double* __restrict__ in, double* __restrict__ out,
                                                               int64_t N0, int64_t N1, int nbands, int nitems, int RC,
                                                               int SI, const __grid_constant__ CUtensorMap tmap,
                                                               const __grid_constant__ RdgParams prm) {

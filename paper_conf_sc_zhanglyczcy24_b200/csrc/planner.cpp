@@ -325,9 +325,16 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
   const int max_k = eng != LORA_ENGINE_RDG_CUDA ? 1 : (p.ndim == 1 ? 8 : rdg2d_max_fuse(p));
   if (fk > max_k) { err = "fuse_k exceeds what the chosen engine supports for this stencil"; return LORA_ERR_UNSUPPORTED; }
   if (fk == 0) {
-    // default fusion depth (exact temporal blocking): measured on B200
-    static const int dflt[5] = {1, 3, 2, 1, 1};  // by radius; tools/quickbench.py, gpurun_out/qb6.jsonl
-    fk = std::min(max_k, p.ndim == 3 ? 2 : (p.ndim == 1 ? 8 : dflt[radius]));
+    // default fusion depth (exact temporal blocking), from B200 measurements
+    // (profiles/r01_quickbench_*.jsonl): fusing pays while the CUDA-core engine is HBM-bound, i.e.
+    // for light stencils (<= 20 issued FMA per point: Box-2D9P, Star-2D13P, 3D, 1D); the radius-3
+    // box (31 FMA/pt) is faster unfused.
+    const double work = cuda_fma_per_point(p);
+    if (p.ndim == 1) fk = 8;
+    else if (p.ndim == 3) fk = 2;
+    else if (work > 20.0) fk = 1;
+    else fk = radius == 1 ? 3 : 2;
+    fk = std::min(max_k, fk);
   }
   p.fuse_k = fk;
   {
