@@ -33,8 +33,8 @@ cudaError_t launch_1d(const Plan& p, const double* src, double* dst, cudaStream_
 
 bool tc2d_supported(const Plan& p);
 bool rdg3d_supported(const Plan& p);
-// Two fused 3D steps (radius 1), kernels_rdg3df.cu.
-cudaError_t launch_rdg3d_fused2(const Plan& p, const double* src, double* dst, cudaStream_t s);
+// k = 2, 3 fused 3D steps (radius 1), kernels_rdg3df.cu.
+cudaError_t launch_rdg3d_fused(const Plan& p, const double* src, double* dst, cudaStream_t s, int k);
 bool rdg3d_fused_supported(const Plan& p);
 bool rdg2d_supported(const Plan& p);
 

@@ -470,7 +470,7 @@ bool rdg2d_supported(const Plan& p) {
 }
 
 int rdg2d_max_fuse(const Plan& p) {
-  if (p.ndim == 3) return rdg3d_fused_supported(p) ? 2 : 1;
+  if (p.ndim == 3) return rdg3d_fused_supported(p) ? 3 : 1;
   if (p.ndim != 2) return 1;
   RdgParams prm;
   const int sig = signature(p, prm);
@@ -479,7 +479,7 @@ int rdg2d_max_fuse(const Plan& p) {
 }
 
 cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s, int k) {
-  if (p.ndim == 3) return k == 1 ? launch_rdg3d(p, src, dst, s) : (k == 2 ? launch_rdg3d_fused2(p, src, dst, s) : cudaErrorNotSupported);
+  if (p.ndim == 3) return k == 1 ? launch_rdg3d(p, src, dst, s) : launch_rdg3d_fused(p, src, dst, s, k);
   switch (p.R) {
     case 1: return rdg_r<1>(p, src, dst, s, k);
     case 2: return rdg_r<2>(p, src, dst, s, k);

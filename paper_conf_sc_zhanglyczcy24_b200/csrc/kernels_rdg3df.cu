@@ -1,4 +1,4 @@
-// Exact temporal fusion of two 3D time steps (SURVEY NEXT-2 "2.5D blocking") for the
+// Exact temporal fusion of K = 2 or 3 3D time steps (SURVEY NEXT-2 "2.5D blocking") for the
 // radius-1 Alg. 2 CUDA-core engine.
 //
 // A CTA (8 warps) owns a column of the domain: 64 lane columns x 16 step-1 rows (14 final rows),
@@ -30,11 +30,9 @@ namespace {
 
 constexpr int F_NS = 3;              // TMA ring stages
 constexpr int F_WARPS = 8;
-constexpr int F_S1 = 16;             // step-1 rows per CTA column (2 per warp)
-constexpr int F_TY = 14;             // final rows per CTA column
+constexpr int F_S1 = 16;             // stage-1 rows per CTA column (2 per warp); stage s: 16 - 2(s-1)
 constexpr int F_IN = 18;             // staged input rows
 constexpr int F_BW = 66;             // staged columns (64 + 2R)
-constexpr int F_BS = 60;             // x band stride (valid final columns per band, even TMA origin)
 constexpr int F_S1W = 72;            // step-1 plane buffer row pitch (doubles): data at [1, 65)
 constexpr int F_ZC = 64;
 
@@ -155,21 +153,52 @@ __device__ __forceinline__ void load_rows(const double* __restrict__ base, int p
   }
 }
 
-template <class SG, bool TMA>
+// Intermediate stage S (1 <= S < K): the stage-S plane just completed in acc[S-1] (ring slot CS)
+// gets the fixed Dirichlet halo re-imposed and is published to its shared plane buffer.
+template <int K, int S, int CS>
+__device__ __forceinline__ void publish(double (&acc)[K][3][2][2], double* __restrict__ buf, int w, int lane,
+                                        int Y0, int X0, int zs, int P0, int P1, int P2,
+                                        const double* __restrict__ in) {
+  const int c0 = 2 * lane;
+#pragma unroll
+  for (int y = 0; y < 2; ++y) {
+    double v[2] = {acc[S - 1][CS][y][0], acc[S - 1][CS][y][1]};
+    acc[S - 1][CS][y][0] = 0.0; acc[S - 1][CS][y][1] = 0.0;
+    const int gy = Y0 - (K - S) + 2 * w + y;  // padded row of this stage-S row
+    const bool zin = zs >= 0 && zs < P0, yin = gy >= 0 && gy < P1;
+    const bool zh = zs < 1 || zs >= P0 - 1, yh = gy < 1 || gy >= P1 - 1;
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {
+      const int cx = X0 + c0 + e;
+      const bool xin = cx >= 0 && cx < P2, xh = cx < 1 || cx >= P2 - 1;
+      double t = v[e];
+      if (!(zin && yin && xin)) t = 0.0;
+      else if (zh || yh || xh) t = in[(int64_t(zs) * P1 + gy) * P2 + cx];
+      buf[(2 * w + y) * F_S1W + 1 + c0 + e] = t;
+    }
+  }
+}
+
+// K fused steps (K = 2, 3).  Stage s computes 16 - 2(s-1) rows (warps w < 8 - (s-1)); final rows
+// TY = 16 - 2(K-1); one __syncthreads per stage boundary per plane.
+template <class SG, int K, bool TMA>
 __global__ void __launch_bounds__(F_WARPS * 32, 2) rdg3df_kernel(const double* __restrict__ in, double* __restrict__ out,
                                                                  int64_t N0, int64_t N1, int64_t N2, int nbx, int nby,
                                                                  int nitems, int ZC, int SI,
                                                                  const __grid_constant__ CUtensorMap tmap,
                                                                  const __grid_constant__ FParams prm) {
   constexpr int STAGE = ((F_IN * F_BW * 8 + 127) / 128) * 128;
-  constexpr int S1B = F_S1 * F_S1W;  // doubles per step-1 plane buffer
+  constexpr int S1B = F_S1 * F_S1W;          // doubles per intermediate plane buffer
+  constexpr int TY = F_S1 - 2 * (K - 1);     // final rows per CTA column
+  constexpr int SG1 = (K - 1) & 1;           // keeps the staged x origin even
+  constexpr int BS = 64 - 2 * (K - 1) - 2 * SG1;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw);
   unsigned char* ring = smem_raw + 128;
-  double* s1buf = reinterpret_cast<double*>(smem_raw + 128 + F_NS * STAGE);  // [2][F_S1][F_S1W]
+  double* sbuf = reinterpret_cast<double*>(smem_raw + 128 + F_NS * STAGE);  // [K-1][2][F_S1][F_S1W]
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   const int P0 = (int)(N0 + 2), P1 = (int)(N1 + 2), P2 = (int)(N2 + 2);
-  for (int i = tid; i < 2 * S1B; i += blockDim.x) s1buf[i] = 0.0;   // margins stay zero
+  for (int i = tid; i < 2 * (K - 1) * S1B; i += blockDim.x) sbuf[i] = 0.0;   // margins stay zero
   const int my_items = blockIdx.x < nitems ? (nitems - 1 - blockIdx.x) / gridDim.x + 1 : 0;
   const int nstages = my_items * SI;
   if (TMA && tid == 0) {
@@ -180,15 +209,15 @@ __global__ void __launch_bounds__(F_WARPS * 32, 2) rdg3df_kernel(const double* _
   // item -> lane column 0 at padded X0, final rows from padded Y0, final planes from padded Z0
   auto geom = [&](int item, int& X0, int& Y0, int& Z0) {
     const int bx = item % nbx, rest = item / nbx, by = rest % nby, bz = rest / nby;
-    X0 = 1 + bx * F_BS - 1 - 1;        // R + b*BS - R(K-1) - SG   (X0 - R even)
-    Y0 = 1 + by * F_TY;
+    X0 = 1 + bx * BS - (K - 1) - SG1;   // R + b*BS - R(K-1) - SG   (X0 - R even)
+    Y0 = 1 + by * TY;
     Z0 = 1 + bz * ZC;
   };
   int pitem = blockIdx.x, pj = 0, pX = 0, pY = 0, pZ = 0;
   if (pitem < nitems) geom(pitem, pX, pY, pZ);
   auto issue_next = [&](int slot) {
     double* dst = reinterpret_cast<double*>(ring + slot * STAGE);
-    const int x = pX - 1, y = pY - 2, z = pZ - 2 + pj;
+    const int x = pX - 1, y = pY - K, z = pZ - K + pj;
     if constexpr (TMA) {  // x even by construction; negative origins are zero-filled by TMA
       if (tid == 0) {
         fence_proxy_async();
@@ -213,7 +242,7 @@ __global__ void __launch_bounds__(F_WARPS * 32, 2) rdg3df_kernel(const double* _
   // prologue (uniform across the CTA: issue_next may contain __syncthreads)
   for (int q = 0; q < F_NS - 1; ++q)
     if (q < nstages) issue_next(q);
-  double acc1[3][2][2], acc2[3][2][2];
+  double acc[K][3][2][2];
   int citem = blockIdx.x, cj = 0, slot = 0, phase = 0;
   int X0 = 0, Y0 = 0, Z0 = 0, zend = 0;
   const int c0 = 2 * lane;  // lane's first column (relative to X0)
@@ -227,71 +256,64 @@ __global__ void __launch_bounds__(F_WARPS * 32, 2) rdg3df_kernel(const double* _
         geom(citem, X0, Y0, Z0);
         zend = min(Z0 + ZC, P0 - 1);
 #pragma unroll
-        for (int s = 0; s < 3; ++s)
+        for (int k = 0; k < K; ++k)
 #pragma unroll
-          for (int y = 0; y < 2; ++y) { acc1[s][y][0] = acc1[s][y][1] = 0.0; acc2[s][y][0] = acc2[s][y][1] = 0.0; }
+          for (int s = 0; s < 3; ++s)
+#pragma unroll
+            for (int y = 0; y < 2; ++y) { acc[k][s][y][0] = 0.0; acc[k][s][y][1] = 0.0; }
       }
-      const int p = Z0 - 2 + cj;  // padded input plane
-      // ---------------- stage 1: step-1 rows 2w, 2w+1 from input tile rows 2w .. 2w+3
+      const int p = Z0 - K + cj;  // padded input plane
+      const int par = q & 1;
+      // ---------------- stage 1: rows 2w, 2w+1 (16 rows) from input tile rows 2w .. 2w+3
       {
         const double* st = reinterpret_cast<const double*>(ring + slot * STAGE);
         double x[4][4];
         load_rows(st + (2 * w) * F_BW, F_BW, lane, x);
-        planes2<SG, I, 0>(x, prm, acc1);
+        planes2<SG, I, 0>(x, prm, acc[0]);
+        publish<K, 1, (I + 1) % 3>(acc, sbuf + (0 * 2 + par) * S1B, w, lane, Y0, X0, p - 1, P0, P1, P2, in);
       }
-      // step-1 plane z1 = p - 1 is complete (ring slot (I + 1) % 3); re-impose the halo, publish it
-      {
-        constexpr int s = (I + 1) % 3;
-        const int z1 = p - 1;
-        const int par = q & 1;
-        double* S = s1buf + par * S1B;
-#pragma unroll
-        for (int y = 0; y < 2; ++y) {
-          double v0 = acc1[s][y][0], v1 = acc1[s][y][1];
-          acc1[s][y][0] = 0.0; acc1[s][y][1] = 0.0;
-          const int gy = Y0 - 1 + 2 * w + y;  // padded row of this step-1 row
-          const int gx = X0 + c0;
-          const bool zin = z1 >= 0 && z1 < P0, yin = gy >= 0 && gy < P1;
-          const bool zh = z1 < 1 || z1 >= P0 - 1, yh = gy < 1 || gy >= P1 - 1;
-#pragma unroll
-          for (int e = 0; e < 2; ++e) {
-            const int cx = gx + e;
-            const bool xin = cx >= 0 && cx < P2, xh = cx < 1 || cx >= P2 - 1;
-            double v = e ? v1 : v0;
-            if (!(zin && yin && xin)) v = 0.0;
-            else if (zh || yh || xh) v = in[(int64_t(z1) * P1 + gy) * P2 + cx];
-            S[(2 * w + y) * F_S1W + 1 + c0 + e] = v;
-          }
-        }
-      }
-      __syncthreads();  // step-1 plane visible; every warp is done with the input slot
+      __syncthreads();  // stage-1 plane visible; every warp is done with the input slot
       if (q + F_NS - 1 < nstages) issue_next((slot + F_NS - 1) % F_NS);
-      // ---------------- stage 2: final rows 2w, 2w+1 from step-1 rows 2w .. 2w+3
-      if (w < F_TY / 2 && cj >= 2) {
-        const double* S = s1buf + (q & 1) * S1B;
-        double x[4][4];
-        load_rows(S + (2 * w) * F_S1W, F_S1W, lane, x);
-        planes2<SG, pm3(I - 1), 0>(x, prm, acc2);
-        // final plane zf = p - 2 complete: ring slot (I - 1 + 1) % 3
-        constexpr int s = pm3(I);
-        const int zf = p - 2;
-        if (cj >= 4 && zf >= Z0 && zf < zend) {
+      // ---------------- stages 2 .. K
+      auto stage = [&](auto Sc) {
+        constexpr int S = decltype(Sc)::value;
+        constexpr int IS = pm3(I - (S - 1));       // ring position of the stage-(S-1) plane consumed
+        const bool active = w < F_S1 / 2 - (S - 1) && cj >= 2 * (S - 1);
+        if (active) {
+          const double* Sb = sbuf + ((S - 2) * 2 + par) * S1B;
+          double x[4][4];
+          load_rows(Sb + (2 * w) * F_S1W, F_S1W, lane, x);
+          planes2<SG, IS, 0>(x, prm, acc[S - 1]);
+        }
+        if constexpr (S < K) {
+          if (active) publish<K, S, (IS + 1) % 3>(acc, sbuf + ((S - 1) * 2 + par) * S1B, w, lane, Y0, X0, p - S, P0, P1,
+                                                  P2, in);
+          __syncthreads();
+        } else if (active) {
+          // final plane zf = p - K complete: ring slot (IS + 1) % 3
+          constexpr int s = (IS + 1) % 3;
+          const int zf = p - K;
+          if (cj >= 2 * K && zf >= Z0 && zf < zend) {
 #pragma unroll
-          for (int y = 0; y < 2; ++y) {
-            const int gy = Y0 + 2 * w + y;
-            if (gy < P1 - 1 && gy < Y0 + F_TY) {
-              double* o = out + (int64_t(zf) * P1 + gy) * P2 + X0;
+            for (int y = 0; y < 2; ++y) {
+              const int gy = Y0 + 2 * w + y;
+              if (gy < P1 - 1 && gy < Y0 + TY) {
+                double* o = out + (int64_t(zf) * P1 + gy) * P2 + X0;
 #pragma unroll
-              for (int e = 0; e < 2; ++e) {
-                const int cx = X0 + c0 + e;
-                if (c0 + e >= 1 && c0 + e < 63 && cx >= 1 && cx < P2 - 1) o[c0 + e] = acc2[s][y][e];
+                for (int e = 0; e < 2; ++e) {
+                  const int cx = X0 + c0 + e;
+                  if (c0 + e >= K - 1 && c0 + e < 65 - K && cx >= 1 && cx < P2 - 1) o[c0 + e] = acc[K - 1][s][y][e];
+                }
               }
             }
           }
-        }
 #pragma unroll
-        for (int y = 0; y < 2; ++y) { acc2[s][y][0] = 0.0; acc2[s][y][1] = 0.0; }
-      }
+          for (int y = 0; y < 2; ++y) { acc[K - 1][s][y][0] = 0.0; acc[K - 1][s][y][1] = 0.0; }
+        }
+      };
+      [&]<int... Ss>(std::integer_sequence<int, Ss...>) {
+        (stage(std::integral_constant<int, Ss + 2>{}), ...);
+      }(std::make_integer_sequence<int, K - 1>{});
       if (++slot == F_NS) { slot = 0; phase ^= 1; }
       if (++cj == SI) { cj = 0; citem += gridDim.x; }
     };
@@ -340,18 +362,19 @@ bool make_fparams(const Plan& p, FParams& prm) {
   return true;
 }
 
-template <class SG, bool TMA>
+template <class SG, int K, bool TMA>
 cudaError_t launch_f(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
                      const FParams& prm) {
   constexpr int STAGE = ((F_IN * F_BW * 8 + 127) / 128) * 128;
-  const int smem = 128 + F_NS * STAGE + 2 * F_S1 * F_S1W * 8;
+  const int smem = 128 + F_NS * STAGE + 2 * (K - 1) * F_S1 * F_S1W * 8;
   static int max_grid = 0;
   if (max_grid == 0) {
-    cudaError_t e = cudaFuncSetAttribute(rdg3df_kernel<SG, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaError_t e = cudaFuncSetAttribute(rdg3df_kernel<SG, K, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
-    max_grid = persistent_grid((const void*)rdg3df_kernel<SG, TMA>, F_WARPS * 32, smem, int64_t(1) << 40);
+    max_grid = persistent_grid((const void*)rdg3df_kernel<SG, K, TMA>, F_WARPS * 32, smem, int64_t(1) << 40);
   }
-  const int nbx = (int)((p.N[2] + F_BS - 1) / F_BS), nby = (int)((p.N[1] + F_TY - 1) / F_TY);
+  constexpr int TY = F_S1 - 2 * (K - 1), BS = 64 - 2 * (K - 1) - 2 * ((K - 1) & 1);
+  const int nbx = (int)((p.N[2] + BS - 1) / BS), nby = (int)((p.N[1] + TY - 1) / TY);
   int64_t zc = F_ZC;
   {
     const int64_t cols = int64_t(nbx) * nby;
@@ -361,13 +384,31 @@ cudaError_t launch_f(const Plan& p, const double* src, double* dst, cudaStream_t
     if (zc2 >= 8 && zc2 <= 2 * F_ZC && cols * ((p.N[0] + zc2 - 1) / zc2) <= rounds * max_grid) zc = zc2;
   }
   const int ZC = (int)zc;
-  const int SI = ((ZC + 4) + 2) / 3 * 3;
+  const int SI = ((ZC + 2 * K) + 2) / 3 * 3;
   const int nbz = (int)((p.N[0] + ZC - 1) / ZC);
   const int64_t nitems = int64_t(nbx) * nby * nbz;
   const int grid = (int)std::min<int64_t>(max_grid, nitems);
-  rdg3df_kernel<SG, TMA><<<grid, F_WARPS * 32, smem, s>>>(src, dst, p.N[0], p.N[1], p.N[2], nbx, nby, (int)nitems, ZC, SI,
+  rdg3df_kernel<SG, K, TMA><<<grid, F_WARPS * 32, smem, s>>>(src, dst, p.N[0], p.N[1], p.N[2], nbx, nby, (int)nitems, ZC, SI,
                                                      map, prm);
   return cudaGetLastError();
+}
+
+template <int K>
+cudaError_t launch_fk(const Plan& p, const double* src, double* dst, cudaStream_t s, const FParams& prm) {
+  CUtensorMap map;
+  const int64_t padded[3] = {p.P[0], p.P[1], p.P[2]};
+  const int box[3] = {1, F_IN, F_BW};
+  const bool tma = !p.force_no_tma && encode_tmap(&map, src, 3, padded, box);
+  if (!tma) std::memset(&map, 0, sizeof(map));
+  // specialisations: Box-3D27P-like (PMA planes, z-mirrored) and Heat-3D-like (point / star, mirrored)
+  if (prm.mode[0] == PM_PMA1 && prm.mode[1] == PM_PMA1 && prm.mirror[0])
+    return tma ? launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, K, true>(p, src, dst, s, map, prm)
+               : launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, K, false>(p, src, dst, s, map, prm);
+  if (prm.mode[0] == PM_POINT && prm.mode[1] == PM_STAR && prm.mirror[0])
+    return tma ? launch_f<Sig3<PM_POINT, PM_STAR, 1>, K, true>(p, src, dst, s, map, prm)
+               : launch_f<Sig3<PM_POINT, PM_STAR, 1>, K, false>(p, src, dst, s, map, prm);
+  return tma ? launch_f<Sig3<-1, -1, -1>, K, true>(p, src, dst, s, map, prm)
+             : launch_f<Sig3<-1, -1, -1>, K, false>(p, src, dst, s, map, prm);
 }
 
 }  // namespace
@@ -377,23 +418,12 @@ bool rdg3d_fused_supported(const Plan& p) {
   return make_fparams(p, prm);
 }
 
-cudaError_t launch_rdg3d_fused2(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+cudaError_t launch_rdg3d_fused(const Plan& p, const double* src, double* dst, cudaStream_t s, int k) {
   FParams prm;
   if (!make_fparams(p, prm)) return cudaErrorNotSupported;
-  CUtensorMap map;
-  const int64_t padded[3] = {p.P[0], p.P[1], p.P[2]};
-  const int box[3] = {1, F_IN, F_BW};
-  const bool tma = !p.force_no_tma && encode_tmap(&map, src, 3, padded, box);
-  if (!tma) std::memset(&map, 0, sizeof(map));
-  // specialisations: Box-3D27P-like (PMA planes, z-mirrored) and Heat-3D-like (point / star, mirrored)
-  if (prm.mode[0] == PM_PMA1 && prm.mode[1] == PM_PMA1 && prm.mirror[0])
-    return tma ? launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, true>(p, src, dst, s, map, prm)
-               : launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, false>(p, src, dst, s, map, prm);
-  if (prm.mode[0] == PM_POINT && prm.mode[1] == PM_STAR && prm.mirror[0])
-    return tma ? launch_f<Sig3<PM_POINT, PM_STAR, 1>, true>(p, src, dst, s, map, prm)
-               : launch_f<Sig3<PM_POINT, PM_STAR, 1>, false>(p, src, dst, s, map, prm);
-  return tma ? launch_f<Sig3<-1, -1, -1>, true>(p, src, dst, s, map, prm)
-             : launch_f<Sig3<-1, -1, -1>, false>(p, src, dst, s, map, prm);
+  if (k == 2) return launch_fk<2>(p, src, dst, s, prm);
+  if (k == 3) return launch_fk<3>(p, src, dst, s, prm);
+  return cudaErrorNotSupported;
 }
 
 }  // namespace lora
