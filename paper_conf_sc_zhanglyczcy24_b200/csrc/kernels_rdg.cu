@@ -222,11 +222,17 @@ __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p,
 #ifndef RDG_MINB_ALL
 #define RDG_MINB_ALL 0   // experiments: force resident CTAs per SM for every instantiation
 #endif
-template <int R, int K>
-constexpr int rdg_minb() { return (RDG_MINB_ALL > 0) ? RDG_MINB_ALL : ((K == 1 || R == 1) ? 4 : 3); }
+// Resident CTAs per SM (register budget 512 / minb per thread x 128 threads), measured on B200
+// (profiles/r01_rdg_occupancy.txt): the heavy radius >= 3 PMA pass wants registers for ILP more
+// than warps (2 CTAs: 338 GS/s vs 305 at 4 for Box-2D49P); light passes want 4; fused radius >= 2 3.
+template <int R, int SIG, int K>
+constexpr int rdg_minb() {
+  return (RDG_MINB_ALL > 0) ? RDG_MINB_ALL
+                            : ((SIG == SIG_PMA && R >= 3 && K == 1) ? 2 : ((K == 1 || R == 1) ? 4 : 3));
+}
 
 template <int R, int SIG, int K, bool TMA>
-__global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, K>())) rdg2d_kernel(const double* __restrict__ in, double* __restrict__ out,
+__global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d_kernel(const double* __restrict__ in, double* __restrict__ out,
                                                               int64_t N0, int64_t N1, int nbands, int nitems, int RC,
                                                               int SI, const __grid_constant__ CUtensorMap tmap,
                                                               const __grid_constant__ RdgParams prm) {
