@@ -169,7 +169,10 @@ __device__ __forceinline__ void apply_all(const double (&x)[BY<R> + 2 * R][2 * R
 }
 
 template <int R, class SG, bool TMA>
-__global__ void __launch_bounds__(R3_WARPS * 32, 3) rdg3d_kernel(const double* __restrict__ in, double* __restrict__ out,
+#ifndef RDG3_MINB
+#define RDG3_MINB 2   // 2 CTAs x 4 warps: registers for ILP beat occupancy (Box-3D27P 291 -> 368 GS/s)
+#endif
+__global__ void __launch_bounds__(R3_WARPS * 32, RDG3_MINB) rdg3d_kernel(const double* __restrict__ in, double* __restrict__ out,
                                                                  int64_t N0, int64_t N1, int64_t N2, int nbx, int nby,
                                                                  int nitems, int ZC, int SI, const __grid_constant__ CUtensorMap tmap,
                                                                  const __grid_constant__ R3Params prm) {

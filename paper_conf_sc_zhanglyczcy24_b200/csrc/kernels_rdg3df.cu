@@ -182,7 +182,10 @@ __device__ __forceinline__ void publish(double (&acc)[K][3][2][2], double* __res
 // K fused steps (K = 2, 3).  Stage s computes 16 - 2(s-1) rows (warps w < 8 - (s-1)); final rows
 // TY = 16 - 2(K-1); one __syncthreads per stage boundary per plane.
 template <class SG, int K, bool TMA>
-__global__ void __launch_bounds__(F_WARPS * 32, 2) rdg3df_kernel(const double* __restrict__ in, double* __restrict__ out,
+#ifndef RDG3F_MINB
+#define RDG3F_MINB 2
+#endif
+__global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const double* __restrict__ in, double* __restrict__ out,
                                                                  int64_t N0, int64_t N1, int64_t N2, int nbx, int nby,
                                                                  int nitems, int ZC, int SI,
                                                                  const __grid_constant__ CUtensorMap tmap,

@@ -327,11 +327,11 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
   if (fk == 0) {
     // default fusion depth (exact temporal blocking), from B200 measurements
     // (profiles/r01_quickbench_*.jsonl): fusing pays while the CUDA-core engine is HBM-bound, i.e.
-    // for light stencils (<= 20 issued FMA per point: Box-2D9P, Star-2D13P, 3D, 1D); the radius-3
-    // box (31 FMA/pt) is faster unfused.
+    // for light stencils (2D <= 20, 3D <= 12 issued FMA per point: Box-2D9P, Star-2D13P, Heat-3D,
+    // 1D); Box-2D49P (31 FMA/pt) and Box-3D27P (18) are faster unfused.
     const double work = cuda_fma_per_point(p);
     if (p.ndim == 1) fk = 8;
-    else if (p.ndim == 3) fk = 2;
+    else if (p.ndim == 3) fk = work <= 12.0 ? 2 : 1;   // Heat-3D fuses; Box-3D27P is faster unfused
     else if (work > 20.0) fk = 1;
     else fk = radius == 1 ? 3 : 2;
     fk = std::min(max_k, fk);
