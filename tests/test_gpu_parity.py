@@ -263,3 +263,28 @@ def test_tc_without_bvs_ablation_parity(h, monkeypatch):
     b, _ = run_gpu(W, g, 3, engine="tc")
     ref = oracle.run(W, g, 3)
     assert rel_err(b, ref) <= 1e-12 and rel_err(a, b) <= 1e-13
+
+
+@pytest.mark.parametrize("name", ["box2d49p", "box3d27p", "heat1d"])
+def test_run_host_matches_device_run(name):
+    """lora_stencil_run_host (host buffers, the e2e path) == lora_stencil_run on device buffers."""
+    import torch
+    import paper_conf_sc_zhanglyczcy24_b200 as L
+    if name == "box2d49p":
+        W, shape = synth.rsym_weights(2, 3, 1), (300, 257)
+    elif name == "box3d27p":
+        W, shape = synth.rsym_weights(3, 1, 1), (40, 33, 66)
+    else:
+        W, shape = synth.preset("heat1d"), (100003,)
+    h = (W.shape[0] - 1) // 2
+    g = synth.grid(tuple(n + 2 * h for n in shape), 5)
+    dev, _ = run_gpu(W, g, 9)
+    st = L.Stencil(W, shape)
+    hin = torch.from_numpy(g).pin_memory()
+    hout = torch.empty_like(hin).pin_memory()
+    st.run_host(hin, hout, 9)
+    assert np.array_equal(hout.numpy(), dev)
+    out2 = np.empty_like(g)            # pageable numpy buffers work too
+    st.run_host(g, out2, 9)
+    assert np.array_equal(out2, dev)
+    st.close()

@@ -163,3 +163,28 @@ def test_cost_model_reproduces_paper_counts():
     conv = 2 * math.ceil((2 * h + 1) ** 2 / 4)                             # eq. 13 per 8(2h+2) points ... per same block
     assert lora == gold["eq16_mma_ratio_h3"]["lora"] and conv == gold["eq16_mma_ratio_h3"]["convstencil"]
     assert gold["fusion_fragment_waste"]["saved"] / gold["fusion_fragment_waste"]["total"] == pytest.approx(0.6154, abs=1e-4)
+
+
+def test_default_engine_and_fusion_choices(L):
+    """The planner's defaults follow the measured B200 costs: CUDA-core RDG,
+    fused only where the pass is HBM-bound."""
+    expect = {"heat2d-256": 3, "box2d9p-10240": 3, "box2d49p-10240": 1, "star2d13p-10240": 2,
+              "heat3d-512": 2, "box3d27p-512": 1, "heat1d-10240000": 8, "1d5p-10240000": 8}
+    for name, k in expect.items():
+        W, c = synth.config(name)
+        info = L.Stencil(W, c["shape"]).info()
+        assert info["engine_name"] == "rdg_cuda" and info["fuse_k"] == k, (name, info["fuse_k"])
+        assert info["halo_depth"] == k * c["radius"]
+
+
+def test_plan_query_fields(L):
+    W = synth.rsym_weights(2, 3, 4)
+    info = L.Stencil(W, (100, 200), engine="tc").info()
+    assert info["ndim"] == 2 and info["radius"] == 3 and info["grid"][:2] == [100, 200]
+    assert info["n_terms"] == 4 and info["n_tc_chain"] == 3 and info["n_cuda"] == 1
+    assert info["fma_per_point_direct"] == 49 and info["fma_per_point_separable"] == 31
+    assert 80 <= info["fma_per_point_issued"] <= 100 and info["tile_m"] == 64
+    with pytest.raises(L.LoraError):
+        L.Stencil(W, (100, 200), engine="rdg_cuda", fuse_k=3)   # exceeds the radius-3 maximum
+    with pytest.raises(L.LoraError):
+        L.Stencil(synth.preset("heat1d"), (100,), engine="tc")   # no tensor-core 1D engine
