@@ -263,10 +263,14 @@ def main():
     per_launch_bytes = BYTES_PER_POINT * float(np.prod(shape))      # per launch: one (fused) superstep
     avg_launch_s = t / args.steps / (-(-T // fuse))
     achieved = per_launch_bytes / avg_launch_s / 1e9
+    tr = ncu_traffic(args.workload, info["engine_name"])
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-            "traffic": ncu_traffic(args.workload, info["engine_name"]), "peak_source": peak_src,
+            "traffic": tr["bytes"] if tr else None,       # dram read+write bytes per launch (ncu --set full)
+            "traffic_source": ({k: tr[k] for k in ("kernel", "source", "fuse")} if tr else None),
+            "peak_source": peak_src,
             "kernel": f"{info['engine_name']} stencil step", "algorithmic_bytes_per_launch": per_launch_bytes,
             "avg_launch_ms": avg_launch_s * 1e3,
+            "avg_launch_note": "timed step / stencil launches per step (the 2 halo-copy launches per run, ~0.1%, included)",
             "gstencil_roofline": peak / BYTES_PER_POINT * world}
 
     # e2e: through the C-ABI with HOST buffers (H2D of the input + D2H of the result inside the region)
