@@ -7,7 +7,9 @@
 #include <cstdlib>
 #include <cstring>
 #include <new>
+#include <algorithm>
 #include <string>
+#include <vector>
 
 #include "kernels.hpp"
 #include "plan.hpp"
@@ -42,7 +44,7 @@ int ensure_device(Plan& p, bool want_scratch) {
 cudaError_t step(const Plan& p, const double* src, double* dst, cudaStream_t s, int k = 1) {
   if (p.ndim == 1) return launch_1d(p, src, dst, s, p.engine == LORA_ENGINE_DIRECT ? 1 : k);
   switch (p.engine) {
-    case LORA_ENGINE_TC: return launch_tc2d(p, src, dst, s);
+    case LORA_ENGINE_TC: return launch_tc2d(p, src, dst, s, k);
     case LORA_ENGINE_RDG_CUDA: return launch_rdg2d(p, src, dst, s, k);
     default: return launch_direct(p, src, dst, s);
   }
@@ -54,6 +56,21 @@ int copy_halo_launch(const Plan& p, const double* in, double* dst, void* stream)
   return (int)launch_copy_halo(p, in, dst, static_cast<cudaStream_t>(stream));
 }
 
+// Steps advanced by each launch of the time loop: ceil(T/k) launches of k fused steps, the last one
+// taking the remainder — except that the tensor-core engine's composed kernel exists only for k
+// itself, so a remainder other than 1 runs as single steps.
+std::vector<int> launch_plan(const Plan& p, int64_t T) {
+  const int64_t k = p.fuse_k < 1 ? 1 : p.fuse_k;
+  std::vector<int> v;
+  for (int64_t done = 0; done < T;) {
+    int64_t st = std::min<int64_t>(k, T - done);
+    if (p.engine == LORA_ENGINE_TC && st != k) st = 1;
+    v.push_back((int)st);
+    done += st;
+  }
+  return v;
+}
+
 // Enqueues the whole time loop on stream s (no synchronisation).
 cudaError_t enqueue(Plan& p, const double* in, double* out, int64_t T, bool two, cudaStream_t s) {
   cudaError_t e = launch_copy_halo(p, in, out, s);
@@ -62,15 +79,13 @@ cudaError_t enqueue(Plan& p, const double* in, double* out, int64_t T, bool two,
     e = launch_copy_halo(p, in, p.scratch, s);
     if (e != cudaSuccess) return e;
   }
-  // ceil(T / k) launches of k fused steps (the last one takes the remainder); launch i writes
-  // `out` when (L - 1 - i) is even, else the scratch buffer, so the last lands in `out`.
-  const int64_t k = p.fuse_k < 1 ? 1 : p.fuse_k;
-  const int64_t L = (T + k - 1) / k;
+  // launch i writes `out` when (L - 1 - i) is even, else the scratch buffer, so the last lands in `out`
+  const std::vector<int> steps = launch_plan(p, T);
+  const int64_t L = (int64_t)steps.size();
   const double* src = in;
   for (int64_t i = 0; i < L; ++i) {
-    const int64_t steps = (i == L - 1) ? T - k * (L - 1) : k;
     double* dst = ((L - 1 - i) % 2 == 0) ? out : p.scratch;
-    e = step(p, src, dst, s, (int)steps);
+    e = step(p, src, dst, s, steps[i]);
     if (e != cudaSuccess) return e;
     src = dst;
   }
@@ -92,8 +107,7 @@ int run_device(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s
     cudaError_t e = cudaMemcpyAsync(out, in, bytes, cudaMemcpyDeviceToDevice, s);
     return e == cudaSuccess ? LORA_OK : cuda_fail(e, "cudaMemcpyAsync");
   }
-  const int64_t k = p.fuse_k < 1 ? 1 : p.fuse_k;
-  const int64_t L = (T + k - 1) / k;
+  const int64_t L = (int64_t)launch_plan(p, T).size();
   const bool two = L >= 2;
   int rc = ensure_device(p, two);
   if (rc) return rc;

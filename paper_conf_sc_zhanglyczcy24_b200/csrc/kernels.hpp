@@ -13,8 +13,10 @@ cudaError_t launch_copy_halo(const Plan& p, const double* in, double* dst, cudaS
 // K11: CUDA-core direct (2R+1)^d-point stencil, one time step src -> dst (interior only).
 cudaError_t launch_direct(const Plan& p, const double* src, double* dst, cudaStream_t s);
 
-// K1 (2D): RDG chains U_k X V_k on FP64 tensor cores (DMMA m8n8k4) with BVS, one step.
-cudaError_t launch_tc2d(const Plan& p, const double* src, double* dst, cudaStream_t s);
+// K1 (2D): RDG chains U_k X V_k on FP64 tensor cores (DMMA m8n8k4) with BVS, one step; k > 1: the
+// composed k-step kernel (§IV-A) on the points farther than (k-1)R from the halo plus an
+// exact stepwise recomputation of the band next to it.
+cudaError_t launch_tc2d(const Plan& p, const double* src, double* dst, cudaStream_t s, int k = 1);
 
 // K6 (2D): RDG chains as banded passes on the FP64 CUDA-core pipe, k fused steps (exact temporal
 // blocking, halo re-imposed every sub-step); 3D dispatches to launch_rdg3d (k = 1).

@@ -161,9 +161,110 @@ bool tc2d_supported(const Plan& p) {
   return p.ndim == 2 && (int)p.terms.size() <= TC_MAXT;
 }
 
-cudaError_t launch_tc2d(const Plan& p, const double* src, double* dst, cudaStream_t s) {
-  if (p.ndim == 3) return launch_tc3d(p, src, dst, s);
+namespace {
+// Exact k-step values on the band of interior points within (k-1)R of the Dirichlet halo, where the
+// composed kernel is not equal to k steps (the intermediate steps would read updated halo cells):
+// one thread per band point re-runs the k Jacobi steps on its (2kR+1)^2 window with the halo fixed.
+struct WB { double w[kMaxN * kMaxN]; };
+
+template <int R, int K>
+__global__ void band_kernel(const double* __restrict__ in, double* __restrict__ out, int64_t N0, int64_t N1,
+                            int64_t nband, const __grid_constant__ WB W) {
+  constexpr int n = 2 * R + 1, H = K * R, M = 2 * H + 1, B = (K - 1) * R;
+  const int64_t id = blockIdx.x * int64_t(blockDim.x) + threadIdx.x;
+  if (id >= nband) return;
+  const int64_t P0 = N0 + 2 * R, P1 = N1 + 2 * R;
+  const int64_t bt = std::min<int64_t>(B, N0), mid = std::max<int64_t>(0, N0 - 2 * B);
+  const int64_t bw = std::min<int64_t>(B, N1);
+  int64_t y, x;  // interior coordinates of this band point
+  const int64_t top = bt * N1;
+  if (id < top) { y = id / N1; x = id % N1; }
+  else if (id < top + mid * (N1 > 2 * B ? 2 * bw : N1)) {
+    const int64_t j = id - top, per = N1 > 2 * B ? 2 * bw : N1;
+    y = B + j / per;
+    const int64_t c = j % per;
+    x = N1 > 2 * B ? (c < bw ? c : N1 - 2 * bw + c) : c;
+  } else {
+    const int64_t j = id - top - mid * (N1 > 2 * B ? 2 * bw : N1);
+    y = std::max<int64_t>(B, N0 - B) + j / N1;
+    x = j % N1;
+  }
+  const int64_t cy = y + R, cx = x + R;  // padded
+  double a[M][M], b[M][M];
+#pragma unroll
+  for (int i = 0; i < M; ++i)
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      const int64_t gy = cy - H + i, gx = cx - H + j;
+      a[i][j] = (gy >= 0 && gy < P0 && gx >= 0 && gx < P1) ? in[gy * P1 + gx] : 0.0;
+    }
+#pragma unroll
+  for (int s = 1; s <= K; ++s) {
+    const int r = (K - s) * R;  // cells within r of the centre are needed after step s
+#pragma unroll
+    for (int i = H - r; i <= H + r; ++i)
+#pragma unroll
+      for (int j = H - r; j <= H + r; ++j) {
+        const int64_t gy = cy - H + i, gx = cx - H + j;
+        const bool halo = gy < R || gy >= P0 - R || gx < R || gx >= P1 - R;
+        double v = a[i][j];
+        if (!halo) {
+          v = 0.0;
+#pragma unroll
+          for (int p = 0; p < n; ++p)
+#pragma unroll
+            for (int q = 0; q < n; ++q) v = fma(W.w[p * n + q], a[i + p - R][j + q - R], v);
+        }
+        b[i][j] = v;
+      }
+#pragma unroll
+    for (int i = H - r; i <= H + r; ++i)
+#pragma unroll
+      for (int j = H - r; j <= H + r; ++j) a[i][j] = b[i][j];
+  }
+  out[cy * P1 + cx] = a[H][H];
+}
+
+template <int R, int K>
+cudaError_t band_launch(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  constexpr int B = (K - 1) * R;
+  const int64_t N0 = p.N[0], N1 = p.N[1];
+  const int64_t inner = std::max<int64_t>(0, N0 - 2 * B) * std::max<int64_t>(0, N1 - 2 * B);
+  const int64_t nband = N0 * N1 - inner;
+  if (nband == 0) return cudaSuccess;
+  WB w{};
+  for (int i = 0; i < (2 * R + 1) * (2 * R + 1); ++i) w.w[i] = p.W[i];
+  band_kernel<R, K><<<(unsigned)((nband + 127) / 128), 128, 0, s>>>(src, dst, N0, N1, nband, w);
+  return cudaGetLastError();
+}
+
+cudaError_t band_dispatch(const Plan& p, const double* src, double* dst, cudaStream_t s, int k) {
+  if (p.R == 1 && k == 2) return band_launch<1, 2>(p, src, dst, s);
+  if (p.R == 1 && k == 3) return band_launch<1, 3>(p, src, dst, s);
+  if (p.R == 1 && k == 4) return band_launch<1, 4>(p, src, dst, s);
+  if (p.R == 2 && k == 2) return band_launch<2, 2>(p, src, dst, s);
+  return cudaErrorNotSupported;
+}
+}  // namespace
+
+cudaError_t launch_tc2d(const Plan& p, const double* src, double* dst, cudaStream_t s, int k) {
+  if (p.ndim == 3) return k == 1 ? launch_tc3d(p, src, dst, s) : cudaErrorNotSupported;
   if (!tc2d_supported(p)) return cudaErrorInvalidValue;
+  if (k > 1) {
+    // composed kernel on the view whose halo is kR wide (same memory: N' + 2kR = N + 2R) ...
+    if (k != p.fuse_k || p.cR != k * p.R) return cudaErrorInvalidValue;
+    const int64_t B = int64_t(k - 1) * p.R;
+    if (p.N[0] > 2 * B && p.N[1] > 2 * B) {
+      Plan v = p;
+      v.R = p.cR; v.W = p.cW; v.terms = p.cterms;
+      v.N[0] = p.N[0] - 2 * B; v.N[1] = p.N[1] - 2 * B;
+      v.graph_exec = nullptr;
+      cudaError_t e = launch_tc2d(v, src, dst, s, 1);
+      if (e != cudaSuccess) return e;
+    }
+    // ... and the exact band next to the Dirichlet halo
+    return band_dispatch(p, src, dst, s, k);
+  }
   switch (p.R) {
     case 1: return tc_r<1>(p, src, dst, s);
     case 2: return tc_r<2>(p, src, dst, s);

@@ -30,12 +30,17 @@ struct Plan {
   int64_t N[3] = {1, 1, 1};
   std::vector<double> W;  // (2R+1)^ndim, row-major copy
   std::vector<Term> terms;
+  // Composed-kernel fusion for the tensor-core engine (§IV-A): k steps of W are
+  // the single (2kR+1)^2 stencil W * ... * W, factored like any other plane (radius cR = kR <= 4).
+  int cR = 0;
+  std::vector<double> cW;
+  std::vector<Term> cterms;
   int engine = LORA_ENGINE_AUTO;
   int fuse_k = 1;
   int tile_m = 0, tile_n = 0;
   int z_symmetric = 0;
-  int force_no_tma = 0;
-  int tc_no_bvs = 0;      // LORA_TC_NO_BVS=1: the Fig. 9 ablation (shuffle-based stage 2) in the TC engine   // LORA_NO_TMA=1: use the LDGSTS staging path (tests both loaders)
+  int force_no_tma = 0;   // LORA_NO_TMA=1: use the LDGSTS staging path (tests both loaders)
+  int tc_no_bvs = 0;      // LORA_TC_NO_BVS=1: the Fig. 9 ablation (shuffle-based stage 2) in the TC engine
   int n_planes_point = 0;
   double recon_err = 0, growth = 0;
   double fma_issued = 0, fma_direct = 0, fma_separable = 0;

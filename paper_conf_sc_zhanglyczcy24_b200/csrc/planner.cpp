@@ -322,7 +322,8 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
   p.fma_issued = eng == LORA_ENGINE_TC ? tc_fma_per_point(p) : eng == LORA_ENGINE_RDG_CUDA ? cuda_fma_per_point(p) : dense;
   int fk = o ? o->fuse_k : 0;
   if (fk < 0) { err = "fuse_k must be >= 0"; return LORA_ERR_INVALID_ARG; }
-  const int max_k = eng != LORA_ENGINE_RDG_CUDA ? 1 : (p.ndim == 1 ? 8 : rdg2d_max_fuse(p));
+  const int max_k = eng == LORA_ENGINE_RDG_CUDA ? (p.ndim == 1 ? 8 : rdg2d_max_fuse(p))
+                   : (eng == LORA_ENGINE_TC && p.ndim == 2 ? kMaxRadius / radius : 1);
   if (fk > max_k) { err = "fuse_k exceeds what the chosen engine supports for this stencil"; return LORA_ERR_UNSUPPORTED; }
   if (fk == 0) {
     // default fusion depth (exact temporal blocking), from B200 measurements
@@ -337,6 +338,45 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
     fk = std::min(max_k, fk);
   }
   p.fuse_k = fk;
+  if (eng == LORA_ENGINE_TC && fk == 0) p.fuse_k = 1;   // composed fusion on tensor cores is opt-in
+  if (eng == LORA_ENGINE_TC && p.fuse_k > 1) {
+    // composed kernel: W_k = W (*) W_{k-1} (full 2D convolution of the offset weights: applying the
+    // correlation twice adds the offsets), radius kR; factored by the same planner (PMA / arms /
+    // elimination).  Exact on points farther than (k-1)R from the Dirichlet halo; the band next
+    // to it is recomputed stepwise by the launcher (reading Q5).
+    const int k = p.fuse_k, cR = k * radius, cn = 2 * cR + 1;
+    std::vector<double> Wk(p.W.begin(), p.W.end());
+    int rk = radius;
+    for (int step = 2; step <= k; ++step) {
+      const int m = 2 * rk + 1, r2 = rk + radius, m2 = 2 * r2 + 1;
+      std::vector<double> Wn(size_t(m2) * m2, 0.0);
+      for (int a0 = 0; a0 < n; ++a0)
+        for (int a1 = 0; a1 < n; ++a1)
+          for (int b0 = 0; b0 < m; ++b0)
+            for (int b1 = 0; b1 < m; ++b1) Wn[size_t(a0 + b0) * m2 + (a1 + b1)] += p.W[size_t(a0) * n + a1] * Wk[size_t(b0) * m + b1];
+      Wk.swap(Wn);
+      rk = r2;
+    }
+    p.cR = cR;
+    p.cW = Wk;
+    p.cterms.clear();
+    Mat C(cn);
+    double cmax = 0;
+    for (int i = 0; i < cn * cn; ++i) { C.a[i] = Wk[i]; cmax = std::max(cmax, std::fabs(Wk[i])); }
+    factor_plane(C, cR, 0, 1e-15 * cmax, p.cterms);
+    double ce = 0;
+    for (int i = 0; i < cn; ++i)
+      for (int j = 0; j < cn; ++j) {
+        double acc = 0;
+        for (const Term& t : p.cterms) acc += t.u[i] * t.v[j];
+        ce = std::max(ce, std::fabs(acc - C(i, j)));
+      }
+    if (cmax > 0 && ce / cmax > 1e-13) { err = "composed kernel does not factor to 1e-13"; return LORA_ERR_FACTOR; }
+    if ((int)p.cterms.size() > 16) { err = "composed kernel has too many rank-1 terms for the TC engine"; return LORA_ERR_UNSUPPORTED; }
+    lora::Plan cv = p;
+    cv.R = cR; cv.W = Wk; cv.terms = p.cterms;
+    p.fma_issued = tc_fma_per_point(cv) / k;
+  }
   {
     const char* e = std::getenv("LORA_NO_TMA");
     p.force_no_tma = (e && e[0] == '1') ? 1 : 0;

@@ -288,3 +288,18 @@ def test_run_host_matches_device_run(name):
     st.run_host(g, out2, 9)
     assert np.array_equal(out2, dev)
     st.close()
+
+
+@pytest.mark.parametrize("h,k", [(1, 2), (1, 3), (1, 4), (2, 2)])
+@pytest.mark.parametrize("kind", ["rsym", "star", "asym"])
+@pytest.mark.parametrize("shape", [(1, 1), (3, 5), (7, 13), (67, 129), (130, 70)])
+def test_tc_composed_fusion(h, k, kind, shape):
+    """The paper's kernel fusion (§IV-A) on the tensor-core engine, made exact: the
+    composed (2kh+1)^2 kernel on points farther than (k-1)h from the Dirichlet halo, the band next
+    to it recomputed stepwise (Q5).  Matches the oracle for T = 1, k, k+1, 2k+1."""
+    W = _weights(kind, 2, h, 70 + h)
+    g = synth.grid(tuple(n + 2 * h for n in shape), 71)
+    for T in sorted({1, 2, k, k + 1, 2 * k - 1, 2 * k + 1}):
+        out, info = run_gpu(W, g, T, engine="tc", fuse_k=k)
+        assert info["fuse_k"] == k
+        assert rel_err(out, oracle.run(W, g, T)) <= 1e-12, (T, rel_err(out, oracle.run(W, g, T)))
