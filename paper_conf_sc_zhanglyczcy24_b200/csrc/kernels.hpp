@@ -10,7 +10,11 @@ namespace lora {
 // Copies the Dirichlet halo ring of `in` into `dst` (both padded arrays of the plan's shape).
 cudaError_t launch_copy_halo(const Plan& p, const double* in, double* dst, cudaStream_t s);
 
-// K11: CUDA-core direct (2R+1)^d-point stencil, one time step src -> dst (interior only).
+// K11: CUDA-core direct (2R+1)^d-point stencil, one time step src -> dst (interior only).  2D runs on
+// the RDG warp-streaming machinery (launch_direct2d_stream, kernels_rdg.cu) so that the comparison
+// with the rank-1 engines is like for like.
+cudaError_t launch_direct2d_stream(const Plan& p, const double* src, double* dst, cudaStream_t s);
+cudaError_t launch_direct3d_stream(const Plan& p, const double* src, double* dst, cudaStream_t s);  // R <= 2
 cudaError_t launch_direct(const Plan& p, const double* src, double* dst, cudaStream_t s);
 
 // K1 (2D): RDG chains U_k X V_k on FP64 tensor cores (DMMA m8n8k4) with BVS, one step; k > 1: the

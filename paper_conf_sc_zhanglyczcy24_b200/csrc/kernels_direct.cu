@@ -1,5 +1,8 @@
 // K11 — CUDA-core FP64 direct stencil (the in-tree comparison kernel, north star (c)), and the
 // halo-copy helper.  out(x) = sum_a W[a] in(x + a - R) (eq. 2), interior only.
+// 1D, 2D and 3D with R <= 2 run the direct sum on the same warp-streaming machinery as the RDG
+// engines (kernels_1d.cu, kernels_rdg.cu SIG_DIRECT, kernels_rdg3d.cu PM_DIRECT) so that the
+// comparison is like for like; this file keeps the 3D R = 3, 4 tile kernel and the halo copy.
 //
 // Weights travel as kernel parameters (constant bank 0), so every DFMA takes its weight as a
 // c[0x0][..] operand: no load instruction per weight.
@@ -10,57 +13,7 @@
 namespace lora {
 namespace {
 
-struct W2 { double w[kMaxN * kMaxN]; };
 template <int R> struct W3 { double w[(2 * R + 1) * (2 * R + 1) * (2 * R + 1)]; };
-
-// ---------------------------------------------------------------- 2D
-// CTA = 32 x 8 threads; tile = 64 rows x 32 columns of outputs; each thread a column strip of
-// RY = 8 rows.  The (64+2R) x (32+2R) input tile is staged in shared memory with coalesced
-// loads; each staged input row feeds the (up to 2R+1) output rows it touches (register
-// sliding window), so each thread reads (RY+2R)(2R+1) doubles from smem per RY outputs.
-constexpr int D2_BX = 32, D2_TY = 8, D2_RY = 8, D2_BY = D2_TY * D2_RY;
-
-template <int R>
-__global__ void __launch_bounds__(256) direct2d(const double* __restrict__ in, double* __restrict__ out,
-                                                int64_t N0, int64_t N1, const W2 W) {
-  constexpr int n = 2 * R + 1;
-  constexpr int SH = D2_BY + 2 * R, SW = D2_BX + 2 * R;
-  __shared__ double tile[SH][SW + 1];
-  const int64_t P1 = N1 + 2 * R;
-  const int64_t y0 = int64_t(blockIdx.y) * D2_BY, x0 = int64_t(blockIdx.x) * D2_BX;  // interior coords
-  const int tid = threadIdx.y * D2_BX + threadIdx.x;
-  for (int i = tid; i < SH * SW; i += 256) {
-    int r = i / SW, c = i % SW;
-    int64_t gy = y0 + r, gx = x0 + c;  // padded coords
-    tile[r][c] = (gy < N0 + 2 * R && gx < P1) ? in[gy * P1 + gx] : 0.0;
-  }
-  __syncthreads();
-  const int tx = threadIdx.x, ty = threadIdx.y;
-  double acc[D2_RY];
-#pragma unroll
-  for (int j = 0; j < D2_RY; ++j) acc[j] = 0.0;
-#pragma unroll
-  for (int rr = 0; rr < D2_RY + 2 * R; ++rr) {
-    double x[n];
-#pragma unroll
-    for (int b = 0; b < n; ++b) x[b] = tile[ty * D2_RY + rr][tx + b];
-#pragma unroll
-    for (int j = 0; j < D2_RY; ++j) {
-      const int a = rr - j;
-      if (a >= 0 && a < n) {
-#pragma unroll
-        for (int b = 0; b < n; ++b) acc[j] = fma(W.w[a * n + b], x[b], acc[j]);
-      }
-    }
-  }
-  const int64_t gx = x0 + tx;
-  if (gx >= N1) return;
-#pragma unroll
-  for (int j = 0; j < D2_RY; ++j) {
-    const int64_t gy = y0 + ty * D2_RY + j;
-    if (gy < N0) out[(gy + R) * P1 + gx + R] = acc[j];
-  }
-}
 
 // ---------------------------------------------------------------- 3D
 // z-streaming: CTA = 32 x 8 threads owns a 32 x 8 (x, y) column of outputs over a z-chunk.
@@ -165,12 +118,7 @@ cudaError_t launch_copy_halo(const Plan& p, const double* in, double* dst, cudaS
 template <int R>
 static cudaError_t direct_r(const Plan& p, const double* src, double* dst, cudaStream_t s) {
   constexpr int n = 2 * R + 1;
-  if (p.ndim == 2) {
-    W2 w{};
-    for (int i = 0; i < n * n; ++i) w.w[i] = p.W[i];
-    dim3 grid((unsigned)((p.N[1] + D2_BX - 1) / D2_BX), (unsigned)((p.N[0] + D2_BY - 1) / D2_BY));
-    direct2d<R><<<grid, dim3(D2_BX, D2_TY), 0, s>>>(src, dst, p.N[0], p.N[1], w);
-  } else {
+  {
     W3<R> w{};
     for (int i = 0; i < n * n * n; ++i) w.w[i] = p.W[i];
     dim3 grid((unsigned)((p.N[2] + D3_BX - 1) / D3_BX), (unsigned)((p.N[1] + D3_BY - 1) / D3_BY),
@@ -182,6 +130,8 @@ static cudaError_t direct_r(const Plan& p, const double* src, double* dst, cudaS
 
 cudaError_t launch_direct(const Plan& p, const double* src, double* dst, cudaStream_t s) {
   if (p.ndim == 1) return launch_1d(p, src, dst, s, 1);
+  if (p.ndim == 2) return launch_direct2d_stream(p, src, dst, s);
+  if (p.ndim == 3 && p.R <= 2) return launch_direct3d_stream(p, src, dst, s);
   switch (p.R) {
     case 1: return direct_r<1>(p, src, dst, s);
     case 2: return direct_r<2>(p, src, dst, s);

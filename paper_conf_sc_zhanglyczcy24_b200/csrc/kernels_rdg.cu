@@ -30,7 +30,7 @@ constexpr int RDG_RC = 128;     // output rows per work item (chunk)
 constexpr int RDG_WARPS = 4;    // warps per CTA (independent streams)
 constexpr int RDG_NS = 3;       // ring stages per warp (3 keeps 4 CTAs = 16 warps per SM)
 
-enum { SIG_PMA = 0, SIG_STAR = 1, SIG_FULL = 2 };
+enum { SIG_PMA = 0, SIG_STAR = 1, SIG_FULL = 2, SIG_DIRECT = 3 };   // DIRECT: W itself in u[][] (K11)
 
 struct RdgParams {
   int K;                     // number of (u, v) chain terms used by the signature
@@ -111,6 +111,18 @@ __device__ __forceinline__ void row_body(const double* __restrict__ xs, int p, d
       const int s = pmod(I - R - a, n);
       acc[s][0] = fma(P.u[1][R + a], x[R], acc[s][0]);
       acc[s][1] = fma(P.u[1][R + a], x[R + 1], acc[s][1]);
+    }
+  } else if constexpr (SIG == SIG_DIRECT) {
+    // the in-tree comparison (north star (c)): the unfactored (2R+1)^2 sum on the same stream —
+    // input row r adds sum_b W[R+a][R+b] x[r][x+b] to output row r - R - a.
+#pragma unroll
+    for (int a = -R; a <= R; ++a) {
+      const int s = pmod(I - R - a, n);
+#pragma unroll
+      for (int b = -R; b <= R; ++b) {
+        acc[s][0] = fma(P.u[R + a][R + b], x[R + b], acc[s][0]);
+        acc[s][1] = fma(P.u[R + a][R + b], x[R + b + 1], acc[s][1]);
+      }
     }
   } else {
     // general: K <= 2R+1 full-radius rank-1 terms (complete-pivot elimination, Q6)
@@ -228,7 +240,8 @@ __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p,
 template <int R, int SIG, int K>
 constexpr int rdg_minb() {
   return (RDG_MINB_ALL > 0) ? RDG_MINB_ALL
-                            : ((SIG == SIG_PMA && R >= 3 && K == 1) ? 2 : ((K == 1 || R == 1) ? 4 : 3));
+                            : (((SIG == SIG_PMA || SIG == SIG_DIRECT) && R >= 3 && K == 1) ? 2
+                                                                                         : ((K == 1 || R == 1) ? 4 : 3));
 }
 
 template <int R, int SIG, int K, bool TMA>
@@ -442,7 +455,7 @@ constexpr int max_fuse(int R) { return R == 1 ? 4 : (R == 2 ? 3 : 2); }
 
 template <int R, int SIG>
 cudaError_t rdg_k(const Plan& p, const double* src, double* dst, cudaStream_t s, const RdgParams& prm, int k) {
-  if constexpr (SIG == SIG_FULL) {
+  if constexpr (SIG == SIG_FULL || SIG == SIG_DIRECT) {
     if (k != 1) return cudaErrorNotSupported;
     return rdg_sig<R, SIG, 1>(p, src, dst, s, prm);
   } else {
@@ -473,6 +486,22 @@ bool rdg2d_supported(const Plan& p) {
   if (p.ndim != 2) return false;
   RdgParams prm;
   return signature(p, prm) >= 0;
+}
+
+cudaError_t launch_direct2d_stream(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  if (p.ndim != 2) return cudaErrorInvalidValue;
+  RdgParams prm;
+  std::memset(&prm, 0, sizeof(prm));
+  const int n = 2 * p.R + 1;
+  for (int i = 0; i < n; ++i)
+    for (int j = 0; j < n; ++j) prm.u[i][j] = p.W[size_t(i) * n + j];
+  switch (p.R) {
+    case 1: return rdg_sig<1, SIG_DIRECT, 1>(p, src, dst, s, prm);
+    case 2: return rdg_sig<2, SIG_DIRECT, 1>(p, src, dst, s, prm);
+    case 3: return rdg_sig<3, SIG_DIRECT, 1>(p, src, dst, s, prm);
+    case 4: return rdg_sig<4, SIG_DIRECT, 1>(p, src, dst, s, prm);
+  }
+  return cudaErrorInvalidValue;
 }
 
 int rdg2d_max_fuse(const Plan& p) {

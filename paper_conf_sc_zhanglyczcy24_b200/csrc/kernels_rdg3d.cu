@@ -31,7 +31,7 @@ template <int R> constexpr int BY = (R == 1 ? 4 : 2);
 constexpr int R3_ZC = 64;
 constexpr int R3_MAXK = 5;   // rank-1 terms per plane (<= 2R+1 for R <= 2)
 
-enum { PM_NONE = 0, PM_POINT = 1, PM_CHAINS = 2, PM_STAR = 3, PM_PMA1 = 4 };
+enum { PM_NONE = 0, PM_POINT = 1, PM_CHAINS = 2, PM_STAR = 3, PM_PMA1 = 4, PM_DIRECT = 5 };
 
 struct R3Params {
   int mode[5];               // per plane a0
@@ -91,6 +91,21 @@ __device__ __forceinline__ void apply_plane(const double (&x)[BY<R> + 2 * R][2 *
         t0 = fma(P.u[A0][1][R + a], x[y + R + a][R], t0);
         t1 = fma(P.u[A0][1][R + a], x[y + R + a][R + 1], t1);
       }
+      d[y][0] = t0;
+      d[y][1] = t1;
+    }
+  } else if (mode == PM_DIRECT) {
+    // the in-tree comparison (north star (c)): the plane's unfactored (2R+1)^2 sum, W_a0 in u[a0][][]
+#pragma unroll
+    for (int y = 0; y < BY<R>; ++y) {
+      double t0 = 0.0, t1 = 0.0;
+#pragma unroll
+      for (int a = -R; a <= R; ++a)
+#pragma unroll
+        for (int b = -R; b <= R; ++b) {
+          t0 = fma(P.u[A0][R + a][R + b], x[y + R + a][R + b], t0);
+          t1 = fma(P.u[A0][R + a][R + b], x[y + R + a][R + b + 1], t1);
+        }
       d[y][0] = t0;
       d[y][1] = t1;
     }
@@ -306,10 +321,22 @@ __global__ void __launch_bounds__(R3_WARPS * 32, RDG3_MINB) rdg3d_kernel(const d
   }
 }
 
-bool make_params3(const Plan& p, R3Params& prm) {
+bool make_params3(const Plan& p, R3Params& prm, bool direct = false) {
   std::memset(&prm, 0, sizeof(prm));
   const int R = p.R, n = 2 * R + 1;
   if (p.ndim != 3 || R > 2) return false;
+  if (direct) {  // every plane as its plain (2R+1)^2 sum, no plane sharing
+    for (int a0 = 0; a0 < n; ++a0) {
+      bool any = false;
+      for (int i = 0; i < n; ++i)
+        for (int j = 0; j < n; ++j) {
+          prm.u[a0][i][j] = p.W[(size_t(a0) * n + i) * n + j];
+          any = any || prm.u[a0][i][j] != 0.0;
+        }
+      prm.mode[a0] = any ? PM_DIRECT : PM_NONE;
+    }
+    return true;
+  }
   for (int a0 = 0; a0 < n; ++a0) {
     std::vector<const Term*> ts;
     for (const Term& t : p.terms)
@@ -386,10 +413,10 @@ cudaError_t rdg3d_launch(const Plan& p, const double* src, double* dst, cudaStre
 }
 
 template <int R>
-cudaError_t rdg3d_r(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+cudaError_t rdg3d_r(const Plan& p, const double* src, double* dst, cudaStream_t s, bool direct = false) {
   using G = G3<R>;
   R3Params prm;
-  if (!make_params3(p, prm)) return cudaErrorNotSupported;
+  if (!make_params3(p, prm, direct)) return cudaErrorNotSupported;
   CUtensorMap map;
   const int64_t padded[3] = {p.P[0], p.P[1], p.P[2]};
   const int box[3] = {1, G::ROWS, G::BW};
@@ -408,6 +435,14 @@ cudaError_t rdg3d_r(const Plan& p, const double* src, double* dst, cudaStream_t 
 }
 
 }  // namespace
+
+cudaError_t launch_direct3d_stream(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  switch (p.R) {
+    case 1: return rdg3d_r<1>(p, src, dst, s, true);
+    case 2: return rdg3d_r<2>(p, src, dst, s, true);
+  }
+  return cudaErrorNotSupported;
+}
 
 bool rdg3d_supported(const Plan& p) {
   R3Params prm;
