@@ -113,3 +113,25 @@ def test_run_dist_two_ranks_nccl_bitwise(case):
     ref = y.cpu().numpy()
     for r, s, a in res:
         assert np.array_equal(a, ref[h + s:h + s + a.shape[0]])
+
+
+def test_nccl_binding_one_rank_communicator(monkeypatch):
+    """Exercises the run-time NCCL binding on one GPU: dlopen of libnccl.so.2, ncclGetUniqueId,
+    ncclCommInitRank with the 128-byte id passed by value, and ncclCommDestroy (LORA_FORCE_NCCL=1
+    builds a real 1-rank communicator); a dist run on it equals the plain run."""
+    import torch
+    import paper_conf_sc_zhanglyczcy24_b200 as L
+    monkeypatch.setenv("LORA_FORCE_NCCL", "1")
+    uid = L.lora_stencil_comm_get_id()
+    assert len(uid) == 128 and any(uid)
+    comm = L.lora_stencil_comm_init(1, 0, uid)
+    W = synth.rsym_weights(2, 1, 2)
+    g = synth.grid((130, 66), 3)
+    st = L.Stencil(W, (128, 64))
+    x = torch.from_numpy(g).cuda()
+    a = torch.empty_like(x); b = torch.empty_like(x)
+    st.run(x, a, 3)
+    L.lora_stencil_run_dist(st.plan, comm, x.data_ptr(), b.data_ptr(), 3, torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    assert torch.equal(a, b)
+    L.lora_stencil_comm_destroy(comm)
