@@ -303,3 +303,30 @@ def test_tc_composed_fusion(h, k, kind, shape):
         out, info = run_gpu(W, g, T, engine="tc", fuse_k=k)
         assert info["fuse_k"] == k
         assert rel_err(out, oracle.run(W, g, T)) <= 1e-12, (T, rel_err(out, oracle.run(W, g, T)))
+
+
+@pytest.mark.parametrize("engine", ["auto", "tc", "rdg_cuda", "direct"])
+@pytest.mark.parametrize("d", [2, 3])
+def test_identity_shift_zero_weights(engine, d):
+    """P7 on the GPU: W = delta copies bitwise for any T; a single off-centre weight 1 shifts exactly
+    (bitwise, halo inflow included); W = 0 gives a zero interior and the untouched halo."""
+    if engine == "tc" and d == 3:
+        pytest.skip("TC 3D needs a multi-point plane")
+    h = 1
+    shape = (20, 17) if d == 2 else (9, 8, 7)
+    g = synth.grid(tuple(n + 2 * h for n in shape), 8)
+    I = np.zeros((3,) * d); I[(1,) * d] = 1.0
+    out, _ = run_gpu(I, g, 5, engine=engine)
+    assert np.array_equal(out, g)
+    S = np.zeros((3,) * d); S[(2,) + (0,) * (d - 1)] = 1.0      # in[x + (1, -1, ...)]
+    out, _ = run_gpu(S, g, 3, engine=engine)
+    assert np.array_equal(out, oracle.run(S, g, 3))
+    Z = np.zeros((3,) * d)
+    try:
+        out, _ = run_gpu(Z, g, 2, engine=engine)
+    except Exception as e:   # the tensor-core engine has no terms to run for W = 0
+        assert engine == "tc", e
+        return
+    ref = g.copy()
+    ref[tuple(slice(1, -1) for _ in range(d))] = 0.0
+    assert np.array_equal(out, ref)
