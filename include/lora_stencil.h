@@ -112,6 +112,16 @@ int lora_stencil_run(lora_plan* p, const double* in, double* out, int64_t timest
  * PCIe/C2C bandwidth; pageable buffers work but are staged by the driver. */
 int lora_stencil_run_host(lora_plan* p, const double* in_host, double* out_host, int64_t timesteps, void* stream);
 
+/* As lora_stencil_run_host but returns once the H2D copy, the run and the D2H copy are
+ * ENQUEUED on `stream` (which must not be the legacy NULL stream: LORA_ERR_INVALID_ARG).
+ * The caller synchronises `stream` before reading out_host or writing in_host, and must not
+ * enqueue another call on the same plan from a different stream before then (the plan's
+ * device buffers are reused).  Host buffers should be pinned, else the copies are
+ * synchronous.  Independent problems on two plans and two streams overlap one problem's
+ * copies with the other's stencil steps (bench.py e2e). */
+int lora_stencil_run_host_async(lora_plan* p, const double* in_host, double* out_host, int64_t timesteps,
+                                void* stream);
+
 /* Fills *info from the plan (host-only). */
 int lora_stencil_plan_query(const lora_plan* p, lora_plan_info* info);
 

@@ -65,6 +65,7 @@ _sig = {
     "lora_stencil_plan_ex": (_P, [_P, ctypes.c_int, ctypes.c_int, _P, _P]),
     "lora_stencil_run": (ctypes.c_int, [_P, _P, _P, ctypes.c_int64, _P]),
     "lora_stencil_run_host": (ctypes.c_int, [_P, _P, _P, ctypes.c_int64, _P]),
+    "lora_stencil_run_host_async": (ctypes.c_int, [_P, _P, _P, ctypes.c_int64, _P]),
     "lora_stencil_plan_query": (ctypes.c_int, [_P, _P]),
     "lora_stencil_plan_terms": (ctypes.c_int, [_P, ctypes.c_int, _P, _P, _P, _P, _P, _P]),
     "lora_stencil_plan_destroy": (None, [_P]),
@@ -154,6 +155,13 @@ def lora_stencil_run_host(plan, in_host: np.ndarray, out_host: np.ndarray, times
     ip = in_host.ctypes.data if isinstance(in_host, np.ndarray) else in_host.data_ptr()
     op = out_host.ctypes.data if isinstance(out_host, np.ndarray) else out_host.data_ptr()
     _check(_lib.lora_stencil_run_host(plan, ip, op, int(timesteps), stream or None))
+
+
+def lora_stencil_run_host_async(plan, in_host, out_host, timesteps: int, stream: int) -> None:
+    """Host buffers (pinned); enqueued on `stream` (not 0), the caller synchronises it."""
+    ip = in_host.ctypes.data if isinstance(in_host, np.ndarray) else in_host.data_ptr()
+    op = out_host.ctypes.data if isinstance(out_host, np.ndarray) else out_host.data_ptr()
+    _check(_lib.lora_stencil_run_host_async(plan, ip, op, int(timesteps), stream or None))
 
 
 def lora_stencil_comm_id_size() -> int:

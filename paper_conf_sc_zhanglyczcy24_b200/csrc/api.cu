@@ -241,9 +241,8 @@ int lora_stencil_run(lora_plan* p, const double* in, double* out, int64_t timest
   return rc;
 }
 
-int lora_stencil_run_host(lora_plan* p, const double* in_host, double* out_host, int64_t timesteps, void* stream) {
-  if (!p || !in_host || !out_host) return fail(LORA_ERR_INVALID_ARG, "NULL plan, in or out");
-  if (timesteps < 0) return fail(LORA_ERR_INVALID_ARG, "timesteps must be >= 0");
+static int run_host_enqueue(lora_plan* p, const double* in_host, double* out_host, int64_t timesteps,
+                            cudaStream_t s) {
   int rc = ensure_device(*p, false);
   if (rc) return rc;
   const size_t bytes = p->elems * sizeof(double);
@@ -253,13 +252,33 @@ int lora_stencil_run_host(lora_plan* p, const double* in_host, double* out_host,
   if (!p->dev_out) {
     if (cudaMalloc(&p->dev_out, bytes) != cudaSuccess) { cudaGetLastError(); p->dev_out = nullptr; return fail(LORA_ERR_OOM, "cudaMalloc(dev_out)"); }
   }
-  cudaStream_t s = static_cast<cudaStream_t>(stream);
   cudaError_t e = cudaMemcpyAsync(p->dev_in, in_host, bytes, cudaMemcpyHostToDevice, s);
   if (e != cudaSuccess) return cuda_fail(e, "H2D copy");
   rc = run_device(*p, p->dev_in, p->dev_out, timesteps, s);
   if (rc) return rc;
   e = cudaMemcpyAsync(out_host, p->dev_out, bytes, cudaMemcpyDeviceToHost, s);
   if (e != cudaSuccess) return cuda_fail(e, "D2H copy");
+  return LORA_OK;
+}
+
+int lora_stencil_run_host_async(lora_plan* p, const double* in_host, double* out_host, int64_t timesteps,
+                                void* stream) {
+  if (!p || !in_host || !out_host) return fail(LORA_ERR_INVALID_ARG, "NULL plan, in or out");
+  if (timesteps < 0) return fail(LORA_ERR_INVALID_ARG, "timesteps must be >= 0");
+  if (stream == nullptr) return fail(LORA_ERR_INVALID_ARG, "run_host_async needs an explicit stream");
+  int rc = run_host_enqueue(p, in_host, out_host, timesteps, static_cast<cudaStream_t>(stream));
+  if (rc) return rc;
+  g_err.clear();
+  return LORA_OK;
+}
+
+int lora_stencil_run_host(lora_plan* p, const double* in_host, double* out_host, int64_t timesteps, void* stream) {
+  if (!p || !in_host || !out_host) return fail(LORA_ERR_INVALID_ARG, "NULL plan, in or out");
+  if (timesteps < 0) return fail(LORA_ERR_INVALID_ARG, "timesteps must be >= 0");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  int rc = run_host_enqueue(p, in_host, out_host, timesteps, s);
+  if (rc) return rc;
+  cudaError_t e;
   e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return cuda_fail(e, "stream sync");
   g_err.clear();

@@ -287,7 +287,23 @@ def test_run_host_matches_device_run(name):
     out2 = np.empty_like(g)            # pageable numpy buffers work too
     st.run_host(g, out2, 9)
     assert np.array_equal(out2, dev)
+    # async form: two plans on two streams in flight at once (the bench e2e pipeline)
+    st2 = L.Stencil(W, shape)
+    g2 = synth.grid(g.shape, 6)
+    dev2, _ = run_gpu(W, g2, 9)
+    hin2 = torch.from_numpy(g2).pin_memory()
+    outs = [torch.zeros_like(hin).pin_memory(), torch.zeros_like(hin).pin_memory()]
+    ss = [torch.cuda.Stream(), torch.cuda.Stream()]
+    for _ in range(2):
+        L.lora_stencil_run_host_async(st.plan, hin, outs[0], 9, ss[0].cuda_stream)
+        L.lora_stencil_run_host_async(st2.plan, hin2, outs[1], 9, ss[1].cuda_stream)
+    for s in ss:
+        s.synchronize()
+    assert np.array_equal(outs[0].numpy(), dev) and np.array_equal(outs[1].numpy(), dev2)
+    with pytest.raises(L.LoraError):
+        L.lora_stencil_run_host_async(st.plan, hin, outs[0], 9, 0)   # the legacy stream is refused
     st.close()
+    st2.close()
 
 
 @pytest.mark.parametrize("h,k", [(1, 2), (1, 3), (1, 4), (2, 2)])
