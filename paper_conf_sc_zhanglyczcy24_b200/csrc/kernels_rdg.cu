@@ -30,7 +30,7 @@ constexpr int RDG_RC = 128;     // output rows per work item (chunk)
 constexpr int RDG_WARPS = 4;    // warps per CTA (independent streams)
 constexpr int RDG_NS = 3;       // ring stages per warp (3 keeps 4 CTAs = 16 warps per SM)
 
-enum { SIG_PMA = 0, SIG_STAR = 1, SIG_FULL = 2, SIG_DIRECT = 3 };   // DIRECT: W itself in u[][] (K11)
+enum { SIG_PMA = 0, SIG_STAR = 1, SIG_FULL = 2, SIG_DIRECT = 3, SIG_ROWS = 4 };   // DIRECT: W itself in u[][] (K11)
 
 struct RdgParams {
   int K;                     // number of (u, v) chain terms used by the signature
@@ -95,6 +95,34 @@ __device__ __forceinline__ void row_body(const double* __restrict__ xs, int p, d
     constexpr int s0 = pmod(I - R, n);
     acc[s0][0] = fma(P.c, x[R], acc[s0][0]);
     acc[s0][1] = fma(P.c, x[R + 1], acc[s0][1]);
+  } else if constexpr (SIG == SIG_ROWS) {
+    // row-pair rank-1 split of a doubly reflection-symmetric W (Plan::rdg_rows): term a has
+    // u_a = e_{R+a} + e_{R-a} and v_a = W[R+a,:] (palindromic), so the horizontal gather is
+    // v_a[0] x_0 + sum_b v_a[b] (x_{-b} + x_{+b}) on the shared pair sums and the vertical gather
+    // is one add into each of the (at most two) output rows R+a, R-a away.
+    double sp0[R + 1], sp1[R + 1];
+#pragma unroll
+    for (int b = 1; b <= R; ++b) {
+      sp0[b] = x[R - b] + x[R + b];
+      sp1[b] = x[R - b + 1] + x[R + b + 1];
+    }
+#pragma unroll
+    for (int a = 0; a <= R; ++a) {
+      double t0 = P.v[a][R] * x[R], t1 = P.v[a][R] * x[R + 1];
+#pragma unroll
+      for (int b = 1; b <= R; ++b) {
+        t0 = fma(P.v[a][R + b], sp0[b], t0);
+        t1 = fma(P.v[a][R + b], sp1[b], t1);
+      }
+      const int s = pmod(I - R - a, n);
+      acc[s][0] += t0;
+      acc[s][1] += t1;
+      if (a > 0) {
+        const int s2 = pmod(I - R + a, n);
+        acc[s2][0] += t0;
+        acc[s2][1] += t1;
+      }
+    }
   } else if constexpr (SIG == SIG_STAR) {
     // star arms: horizontal arm (u = e_R) lands on the centre row; vertical arm (v = e_R) is X itself.
     double t0 = 0.0, t1 = 0.0;
@@ -240,7 +268,7 @@ __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p,
 template <int R, int SIG, int K>
 constexpr int rdg_minb() {
   return (RDG_MINB_ALL > 0) ? RDG_MINB_ALL
-                            : (((SIG == SIG_PMA || SIG == SIG_DIRECT) && R >= 3 && K == 1) ? 2
+                            : (((SIG == SIG_PMA || SIG == SIG_ROWS || SIG == SIG_DIRECT) && R >= 3 && K == 1) ? 2
                                                                                          : ((K == 1 || R == 1) ? 4 : 3));
 }
 
@@ -367,6 +395,12 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
 int signature(const Plan& p, RdgParams& prm) {
   std::memset(&prm, 0, sizeof(prm));
   const int R = p.R, n = 2 * R + 1;
+  if (p.rdg_rows && p.ndim == 2) {
+    prm.K = R + 1;
+    for (int a = 0; a <= R; ++a)
+      for (int j = 0; j < n; ++j) prm.v[a][j] = p.W[size_t(R + a) * n + j];
+    return SIG_ROWS;
+  }
   // PMA pyramid: chains of radius R, R-1, ..., 1 (in that order) + centre scalar
   bool pma = (int)p.terms.size() == R + 1;
   for (int k = 0; pma && k < R; ++k) pma = p.terms[k].kind == kChain && p.terms[k].r == R - k;
@@ -474,6 +508,9 @@ cudaError_t rdg_r(const Plan& p, const double* src, double* dst, cudaStream_t s,
   RdgParams prm;
   const int sig = signature(p, prm);
   if (sig == SIG_PMA) return rdg_k<R, SIG_PMA>(p, src, dst, s, prm, k);
+  if constexpr (R >= 3) {
+    if (sig == SIG_ROWS) return rdg_k<R, SIG_ROWS>(p, src, dst, s, prm, k);
+  }
   if (sig == SIG_STAR) return rdg_k<R, SIG_STAR>(p, src, dst, s, prm, k);
   if (sig == SIG_FULL) return rdg_k<R, SIG_FULL>(p, src, dst, s, prm, k);
   return cudaErrorNotSupported;

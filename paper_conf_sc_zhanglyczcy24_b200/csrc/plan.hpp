@@ -42,6 +42,11 @@ struct Plan {
   int force_no_tma = 0;   // LORA_NO_TMA=1: use the LDGSTS staging path (tests both loaders)
   int tc_no_bvs = 0;      // LORA_TC_NO_BVS=1: the Fig. 9 ablation (shuffle-based stage 2) in the TC engine
   int n_planes_point = 0;
+  // CUDA-core engine, 2D, radius >= 3, W reflection-symmetric in both axes: evaluate W as the
+  // row-pair rank-1 split u_a = e_{R+a} + e_{R-a}, v_a = W[R+a,:] (a = 0..R; exact, growth 1),
+  // which issues R + (R+1)^2 + 2R+1 FP64 ops per point against PMA's (28 vs 26 at R = 3).
+  // LORA_RDG_PMA=1 keeps the PMA factors on that engine (ablation).
+  int rdg_rows = 0;
   double recon_err = 0, growth = 0;
   double fma_issued = 0, fma_direct = 0, fma_separable = 0;
   // device state (lazily created at first run)

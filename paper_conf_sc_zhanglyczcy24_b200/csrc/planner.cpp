@@ -201,8 +201,19 @@ double cuda_fma_per_point(const Plan& p) {
     return f;
   };
   if (p.ndim == 2) {
-    double f = plane_cost(0);
-    return f;
+    const int R = p.R;
+    if (p.rdg_rows) return R + (R + 1) * (R + 1) + (2 * R + 1);   // SIG_ROWS (kernels_rdg.cu)
+    // PMA pyramid (SIG_PMA): R shared tap-pair sums, then per chain of radius H a palindromic
+    // horizontal gather (H+1) and a vertical scatter (2H+1), plus the scalar C_{h+1}
+    bool pma = (int)p.terms.size() == R + 1;
+    for (int k = 0; pma && k < R; ++k) pma = p.terms[k].kind == kChain && p.terms[k].r == R - k;
+    if (pma) pma = p.terms[R].kind == kPoint && p.terms[R].r == 0;
+    if (pma) {
+      double f = R + 1;
+      for (int k = 0; k < R; ++k) f += (R - k + 1) + (2 * (R - k) + 1);
+      return f;
+    }
+    return plane_cost(0);
   }
   double f = 0;
   for (int q = 0; q < n; ++q) {
@@ -293,6 +304,21 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
   p.growth = w1 > 0 ? g / w1 : 0.0;
   if (p.recon_err > 1e-14) { err = "factorisation does not reconstruct W to 1e-14"; return LORA_ERR_FACTOR; }
 
+  {  // row-pair split for the CUDA-core engine (Plan::rdg_rows)
+    bool rows = ndim == 2 && radius >= 3;
+    for (int i = 0; rows && i < n; ++i)
+      for (int j = 0; j < n; ++j)
+        if (weights[size_t(i) * n + j] != weights[size_t(n - 1 - i) * n + j] ||
+            weights[size_t(i) * n + j] != weights[size_t(i) * n + (n - 1 - j)]) { rows = false; break; }
+    const char* e = std::getenv("LORA_RDG_PMA");
+    if (e && e[0] == '1') rows = false;
+    p.rdg_rows = 0;
+    if (rows) {  // only where it issues less than the planner's own factors (not for star arms)
+      const double f_terms = cuda_fma_per_point(p);
+      p.rdg_rows = 1;
+      if (cuda_fma_per_point(p) >= f_terms) p.rdg_rows = 0;
+    }
+  }
   p.fma_direct = nnz;
   p.fma_separable = 0;
   for (const Term& t : p.terms) {

@@ -159,6 +159,26 @@ def test_2d_temporal_fusion_exact(h, kind, shape):
             assert rel_err(a, oracle.run(W, g, T)) <= 1e-12
 
 
+@pytest.mark.parametrize("h", [3, 4])
+@pytest.mark.parametrize("shape", [(3, 5), (67, 129), (300, 200)])
+def test_rows_and_pma_forms(h, shape, monkeypatch):
+    """The CUDA-core engine's two rank-1 splits of a doubly reflection-symmetric W (row pairs,
+    Plan::rdg_rows, the default at radius >= 3; PMA with LORA_RDG_PMA=1) both match the oracle,
+    unfused and fused, and the fused form equals the unfused one bitwise."""
+    W = synth.rsym_weights(2, h, 60 + h)
+    g = synth.grid(tuple(n + 2 * h for n in shape), 91 + h)
+    for pma in ("0", "1"):
+        monkeypatch.setenv("LORA_RDG_PMA", pma)
+        for T in (1, 2, 5):
+            a, info = run_gpu(W, g, T, engine="rdg_cuda", fuse_k=1)
+            n = h + 1
+            want = (h + n * n + 2 * h + 1) if pma == "0" else (h + 1 + sum((h - k + 1) + (2 * (h - k) + 1) for k in range(h)))
+            assert info["fma_per_point_issued"] == want
+            assert rel_err(a, oracle.run(W, g, T)) <= 1e-12
+            b, _ = run_gpu(W, g, T, engine="rdg_cuda", fuse_k=2)
+            assert np.array_equal(a, b)
+
+
 def test_fusion_staging_paths_agree(monkeypatch):
     W = synth.rsym_weights(2, 3, 5)
     g = synth.grid((206, 136), 11)
