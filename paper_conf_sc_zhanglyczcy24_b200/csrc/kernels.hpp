@@ -7,6 +7,31 @@
 
 namespace lora {
 
+// Device-initiated halo exchange (csrc/dist_p2p.cu): the slab's boundary work items
+// store their edge rows/planes straight into the neighbour's halo over peer memory (NVLink P2P /
+// CUDA IPC) and publish a per-unit step counter there; the neighbour's boundary items wait on it
+// before staging their halo.  Interior items neither wait nor signal, so the exchange overlaps the
+// interior tile by tile.  A "unit" is a 64-column band (2D) or a 64 x BY column (3D); a boundary
+// item of unit b waits for the neighbour's units b-1..b+1 (2D) / the 3 x 3 around b (3D), whose
+// staged tiles overlap the columns it reads and writes.
+struct P2PArgs {
+  int active = 0;                  // 0: ordinary single-GPU launch
+  int nunits = 0;                  // flag units per side
+  int nux = 0;                     // 3D: units per y row (unit = bx + nux * by)
+  int pad_ = 0;
+  const unsigned long long* wait_lo = nullptr;   // my flags written by the lower neighbour (null: none)
+  const unsigned long long* wait_hi = nullptr;   // my flags written by the upper neighbour
+  unsigned long long* sig_lo = nullptr;          // the lower neighbour's flags for me
+  unsigned long long* sig_hi = nullptr;          // the upper neighbour's flags for me
+  double* dst_lo = nullptr;        // the lower neighbour's destination buffer of this step
+  double* dst_hi = nullptr;
+  long long off_lo = 0;            // my padded element index + off_lo = its index (n0_lo * row)
+  long long off_hi = 0;            // -(n0 * row)
+  unsigned long long wait_val = 0; // boundary items wait until flags >= wait_val
+  unsigned long long sig_val = 0;  // and publish sig_val when their stores are done
+  int* err = nullptr;              // device error word (spin timeout => 1)
+};
+
 // Copies the Dirichlet halo ring of `in` into `dst` (both padded arrays of the plan's shape).
 cudaError_t launch_copy_halo(const Plan& p, const double* in, double* dst, cudaStream_t s);
 
@@ -25,6 +50,10 @@ cudaError_t launch_tc2d(const Plan& p, const double* src, double* dst, cudaStrea
 // K6 (2D): RDG chains as banded passes on the FP64 CUDA-core pipe, k fused steps (exact temporal
 // blocking, halo re-imposed every sub-step); 3D dispatches to launch_rdg3d (k = 1).
 cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s, int k);
+// One unfused step of the 2D CUDA-core engine (any signature incl. the direct comparison kernel) or
+// of the 3D one, with the device-initiated halo exchange of `d` (d.active = 1).
+cudaError_t launch_step_p2p(const Plan& p, const double* src, double* dst, cudaStream_t s, const P2PArgs& d);
+int p2p_units(const Plan& p, int* nux);   // flag units per side, 0 if the plan's engine has no P2P path
 int rdg2d_max_fuse(const Plan& p);
 
 // K2 on CUDA cores (3D, Alg. 2 with RDG per plane), one step.

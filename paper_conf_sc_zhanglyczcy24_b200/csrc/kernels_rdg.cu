@@ -39,12 +39,17 @@ struct RdgParams {
   double c;                  // PMA scalar C_{h+1}
 };
 
-template <int R>
+// NH = 64-column halves per warp: lane p owns columns 64h + 2p, 64h + 2p + 1 (h < NH), so each
+// staged row is read with the conflict-free 16-byte lane pattern of one half at a time; NH = 2
+// halves the band-edge recomputation of the fused kernels and gives every warp two independent
+// row pipelines (ILP for the 8-cycle DFMA latency).
+template <int R, int NH = 1>
 struct Geom {
   static constexpr int n = 2 * R + 1;
   static constexpr int m = n >= 6 ? 1 : 2;
   static constexpr int SROWS = n * m;                                  // rows per stage (multiple of n)
-  static constexpr int BW = 64 + 2 * R;                                // staged columns
+  static constexpr int BW = 64 * NH + 2 * R;                           // staged columns
+  static constexpr int BUFD = ((BW + 15) / 16) * 16;                   // doubles per intermediate row buffer
   static constexpr int STAGE = ((SROWS * BW * 8 + 127) / 128) * 128;   // bytes per stage
   static constexpr int SI = (RDG_RC + 2 * R + SROWS - 1) / SROWS;      // stages per work item
   static constexpr int WARP_BYTES = RDG_NS * STAGE;
@@ -117,7 +122,10 @@ __device__ __forceinline__ void row_body(const double* __restrict__ xs, int p, d
       const int s = pmod(I - R - a, n);
       acc[s][0] += t0;
       acc[s][1] += t1;
-      if (a > 0) {
+      if (a == R) {   // slot I mod n was emptied after the previous row: this is its first term
+        acc[pmod(I, n)][0] = t0;
+        acc[pmod(I, n)][1] = t1;
+      } else if (a > 0) {
         const int s2 = pmod(I - R + a, n);
         acc[s2][0] += t0;
         acc[s2][1] += t1;
@@ -195,67 +203,101 @@ struct StageCtx {
   int64_t ioff[K];          //                     element offset of (row for I = 0, column 0) in `in`
 };
 
+template <int NH>
 struct LaneCtx {
-  int c0;                   // padded column of the lane's first column (may be < 0)
-  bool inside0, inside1, colhalo0, colhalo1, valid0, valid1, vec;
+  int c0;                   // padded column of the lane's first column (may be < 0); half h adds 64h
+  bool inside[NH][2], colhalo[NH][2], valid[NH][2], vec[NH];
+  bool edge;                // some column of the lane is a column halo or outside the array
 };
 
-template <int R, int SIG, int K, int I0, int I, int S>
-__device__ __forceinline__ void fused_stage(const double* __restrict__ src, int p, double (&acc)[K][2 * R + 1][2],
-                                            const RdgParams& P, double* __restrict__ bufs, int par,
-                                            const double* __restrict__ in, double* __restrict__ out, int64_t P1,
-                                            const StageCtx<K>& sc, const LaneCtx& lc) {
+// One iteration of the fused pipeline (input row I of the staged tile), stages S = K down to 1.
+// Stage S >= 2 consumes the row stage S-1 produced in the PREVIOUS iteration (row buffer of the
+// other parity), so within an iteration every stage reads before any stage writes and the stages
+// are independent instruction streams (ILP for the 8-cycle DFMA latency); one __syncwarp per
+// iteration orders the buffer writes against the next iteration's reads.  Stage S therefore lags
+// stage 1 by (S-1)(R+1) rows (StageCtx row offsets include the extra (S-1) rows).
+// FULL: every row of the stage is interior for every intermediate step, every final row is stored
+// and every lane stores a 16-byte pair (decided per stage, warp-uniform): no per-row checks.
+template <int R, int SIG, int K, int NH, bool FULL, int I0, int I, int S>
+__device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, int p,
+                                           double (&acc)[K][NH][2 * R + 1][2], const RdgParams& P,
+                                           double* __restrict__ bufs, int par, const double* __restrict__ in,
+                                           double* __restrict__ out, int64_t P1, const StageCtx<K>& sc,
+                                           const LaneCtx<NH>& lc) {
   constexpr int n = 2 * R + 1;
-  constexpr int Is = pmod(I0 - (S - 1) * R, n);   // row index mod n of stage S's input row
-  row_body<R, SIG, Is>(src, p, acc[S - 1], P);
+  constexpr int BUFD = Geom<R, NH>::BUFD;
+  constexpr int Is = pmod(I0 - (S - 1) * (R + 1), n);   // ring index of stage S's input row (any per-stage constant)
+  const double* src = S == 1 ? st_row : bufs + (2 * (S - 2) + (par ^ 1)) * BUFD;
+#pragma unroll
+  for (int h = 0; h < NH; ++h) row_body<R, SIG, Is>(src + 64 * h, p, acc[S - 1][h], P);
   constexpr int cs = (Is + 1) % n;                // slot of the row this stage just completed
-  double v0 = acc[S - 1][cs][0], v1 = acc[S - 1][cs][1];
-  acc[S - 1][cs][0] = 0.0;
-  acc[S - 1][cs][1] = 0.0;
+  double v[NH][2];
+#pragma unroll
+  for (int h = 0; h < NH; ++h) {
+    v[h][0] = acc[S - 1][h][cs][0];
+    v[h][1] = acc[S - 1][h][cs][1];
+    acc[S - 1][h][cs][0] = 0.0;
+    acc[S - 1][h][cs][1] = 0.0;
+  }
   if constexpr (S < K) {
     // re-impose the fixed Dirichlet halo on the intermediate row (exact temporal blocking)
-    if (I < sc.hlo[S - 1] || I >= sc.hhi[S - 1]) {
+    if (FULL) {
+    } else if (I < sc.hlo[S - 1] || I >= sc.hhi[S - 1]) {
       const bool row_in = I >= sc.rlo[S - 1] && I < sc.rhi[S - 1];
       const double* ir = in + sc.ioff[S - 1] + int64_t(I) * P1 + lc.c0;
-      v0 = (row_in && lc.inside0) ? ir[0] : 0.0;
-      v1 = (row_in && lc.inside1) ? ir[1] : 0.0;
-    } else if (lc.colhalo0 | lc.colhalo1 | !lc.inside0 | !lc.inside1) {
+#pragma unroll
+      for (int h = 0; h < NH; ++h)
+#pragma unroll
+        for (int j = 0; j < 2; ++j) v[h][j] = (row_in && lc.inside[h][j]) ? ir[64 * h + j] : 0.0;
+    } else if (lc.edge) {
       const double* ir = in + sc.ioff[S - 1] + int64_t(I) * P1 + lc.c0;
-      if (lc.colhalo0) v0 = ir[0];
-      if (lc.colhalo1) v1 = ir[1];
-      if (!lc.inside0) v0 = 0.0;
-      if (!lc.inside1) v1 = 0.0;
+#pragma unroll
+      for (int h = 0; h < NH; ++h)
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          if (lc.colhalo[h][j]) v[h][j] = ir[64 * h + j];
+          if (!lc.inside[h][j]) v[h][j] = 0.0;
+        }
     }
-    constexpr int BUFD = ((Geom<R>::BW + 15) / 16) * 16;
-    double* b = bufs + (2 * (S - 1) + par) * BUFD;   // [stage][parity] row buffers (no local-memory pointer table)
-    b[R + 2 * p] = v0;
-    b[R + 2 * p + 1] = v1;
-    __syncwarp();
-    fused_stage<R, SIG, K, I0, I, S + 1>(b, p, acc, P, bufs, par, in, out, P1, sc, lc);
+    double* b = bufs + (2 * (S - 1) + par) * BUFD;   // [stage][parity] row buffers
+#pragma unroll
+    for (int h = 0; h < NH; ++h) {   // 8-byte stores: R + 2p is odd for odd R
+      b[R + 64 * h + 2 * p] = v[h][0];
+      b[R + 64 * h + 2 * p + 1] = v[h][1];
+    }
+  } else if constexpr (FULL) {
+    double* o = out + sc.ooff + int64_t(I) * P1;
+#pragma unroll
+    for (int h = 0; h < NH; ++h) *reinterpret_cast<double2*>(o + 64 * h) = make_double2(v[h][0], v[h][1]);
   } else {
     if (I >= sc.lo && I < sc.hi) {
       double* o = out + sc.ooff + int64_t(I) * P1;
-      if (lc.vec) {
-        *reinterpret_cast<double2*>(o) = make_double2(v0, v1);
-      } else {
-        if (lc.valid0) o[0] = v0;
-        if (lc.valid1) o[1] = v1;
+#pragma unroll
+      for (int h = 0; h < NH; ++h) {
+        if (lc.vec[h]) {
+          *reinterpret_cast<double2*>(o + 64 * h) = make_double2(v[h][0], v[h][1]);
+        } else {
+          if (lc.valid[h][0]) o[64 * h] = v[h][0];
+          if (lc.valid[h][1]) o[64 * h + 1] = v[h][1];
+        }
       }
     }
   }
+  if constexpr (S > 1) fused_iter<R, SIG, K, NH, FULL, I0, I, S - 1>(st_row, p, acc, P, bufs, par, in, out, P1, sc, lc);
 }
 
-template <int R, int SIG, int K, int I>
-__device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p, double (&acc)[K][2 * R + 1][2],
+template <int R, int SIG, int K, int NH, bool FULL, int I>
+__device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p, double (&acc)[K][NH][2 * R + 1][2],
                                            const RdgParams& P, double* __restrict__ bufs,
                                            const double* __restrict__ in, double* __restrict__ out, int64_t P1,
-                                           const StageCtx<K>& sc, const LaneCtx& lc, int par0) {
+                                           const StageCtx<K>& sc, const LaneCtx<NH>& lc, int par0) {
   constexpr int n = 2 * R + 1;
-  if constexpr (I < Geom<R>::SROWS) {
+  if constexpr (I < Geom<R, NH>::SROWS) {
     constexpr int OFF = pmod(R - K * R, n);  // q0 mod n (RC is a multiple of n)
-    fused_stage<R, SIG, K, pmod(I + OFF, n), I, 1>(st + I * Geom<R>::BW, p, acc, P, bufs, (par0 + I) & 1, in, out, P1,
-                                                   sc, lc);
-    fused_rows<R, SIG, K, I + 1>(st, p, acc, P, bufs, in, out, P1, sc, lc, par0);
+    fused_iter<R, SIG, K, NH, FULL, pmod(I + OFF, n), I, K>(st + I * Geom<R, NH>::BW, p, acc, P, bufs, (par0 + I) & 1,
+                                                            in, out, P1, sc, lc);
+    if constexpr (K > 1) __syncwarp();
+    fused_rows<R, SIG, K, NH, FULL, I + 1>(st, p, acc, P, bufs, in, out, P1, sc, lc, par0);
   }
 }
 
@@ -265,11 +307,24 @@ __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p,
 // Resident CTAs per SM (register budget 512 / minb per thread x 128 threads), measured on B200
 // (profiles/r01_rdg_occupancy.txt): the heavy radius >= 3 PMA pass wants registers for ILP more
 // than warps (2 CTAs: 338 GS/s vs 305 at 4 for Box-2D49P); light passes want 4; fused radius >= 2 3.
+#ifndef RDG_NH_FUSED
+#define RDG_NH_FUSED 2   // 64-column halves per warp in the fused (K >= 2) kernels
+#endif
+template <int R, int K>
+constexpr int rdg_cta_smem(int nh) {   // must match rdg_launch
+  return nh == 1 ? 128 + RDG_WARPS * (Geom<R, 1>::WARP_BYTES + 2 * (K - 1) * Geom<R, 1>::BUFD * 8)
+                 : 128 + RDG_WARPS * (Geom<R, 2>::WARP_BYTES + 2 * (K - 1) * Geom<R, 2>::BUFD * 8);
+}
+// NH = 2 where two CTAs of it still fit the 228 KB of shared memory per SM (R = 1, 3, 4)
+template <int R, int SIG, int K>
+constexpr int rdg_nh() { return (K >= 2 && RDG_NH_FUSED == 2 && 2 * (rdg_cta_smem<R, K>(2) + 1024) <= 228 * 1024) ? 2 : 1; }
+
 template <int R, int SIG, int K>
 constexpr int rdg_minb() {
   return (RDG_MINB_ALL > 0) ? RDG_MINB_ALL
-                            : (((SIG == SIG_PMA || SIG == SIG_ROWS || SIG == SIG_DIRECT) && R >= 3 && K == 1) ? 2
-                                                                                         : ((K == 1 || R == 1) ? 4 : 3));
+         : (rdg_nh<R, SIG, K>() == 2 ? 2
+            : (((SIG == SIG_PMA || SIG == SIG_ROWS || SIG == SIG_DIRECT) && R >= 3 && K == 1) ? 2
+                                                                                        : ((K == 1 || R == 1) ? 4 : 3)));
 }
 
 template <int R, int SIG, int K, bool TMA>
@@ -277,10 +332,11 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
                                                               int64_t N0, int64_t N1, int nbands, int nitems, int RC,
                                                               int SI, const __grid_constant__ CUtensorMap tmap,
                                                               const __grid_constant__ RdgParams prm) {
-  using G = Geom<R>;
+  constexpr int NH = rdg_nh<R, SIG, K>();
+  using G = Geom<R, NH>;
   constexpr int SG = (R * (K - 1)) & 1;           // shift keeping the staged origin even (TMA: 16-B aligned start)
-  constexpr int BS = 64 - 2 * R * (K - 1) - 2 * SG;  // band stride (valid final columns per band)
-  constexpr int BUFD = ((G::BW + 15) / 16) * 16;  // doubles per intermediate row buffer
+  constexpr int BS = 64 * NH - 2 * R * (K - 1) - 2 * SG;  // band stride (valid final columns per band)
+  constexpr int BUFD = G::BUFD;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw) + wl * RDG_NS;
@@ -336,10 +392,11 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
     if (q < nstages) issue_next(q);
     else if constexpr (!TMA) cp_async_commit();  // empty group: keeps wait_group<NS-1> exact
   }
-  double acc[K][2 * R + 1][2];
-  LaneCtx lc{};
+  double acc[K][NH][2 * R + 1][2];
+  LaneCtx<NH> lc{};
   StageCtx<K> sc{};
   int citem = gw, cj = 0, X0 = 0, A = 0, rows_valid_end = 0;
+  bool all_fast = false;   // every lane of the item: 16-byte stores, no column halo / outside column
   int slot = 0, phase = 0;
   for (int q = 0; q < nstages; ++q) {
     if (q + RDG_NS - 1 < nstages) issue_next((slot + RDG_NS - 1) % RDG_NS);
@@ -355,28 +412,40 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
 #pragma unroll
       for (int k = 0; k < K; ++k)
 #pragma unroll
-        for (int s = 0; s < 2 * R + 1; ++s) { acc[k][s][0] = 0.0; acc[k][s][1] = 0.0; }
-      const int c0 = X0 + 2 * lane, c1 = c0 + 1;
-      lc.c0 = c0;
-      lc.inside0 = c0 >= 0 && c0 < P1;
-      lc.inside1 = c1 >= 0 && c1 < P1;
-      lc.colhalo0 = lc.inside0 && (c0 < R || c0 >= P1 - R);
-      lc.colhalo1 = lc.inside1 && (c1 < R || c1 >= P1 - R);
-      lc.valid0 = c0 >= X0 + R * (K - 1) && c0 < X0 + 64 - R * (K - 1) && c0 >= R && c0 < P1 - R;
-      lc.valid1 = c1 >= X0 + R * (K - 1) && c1 < X0 + 64 - R * (K - 1) && c1 >= R && c1 < P1 - R;
-      lc.vec = lc.valid0 && lc.valid1 && ((reinterpret_cast<uintptr_t>(out + c0) & 15) == 0) && ((P1 & 1) == 0);
+        for (int h = 0; h < NH; ++h)
+#pragma unroll
+          for (int s = 0; s < 2 * R + 1; ++s) { acc[k][h][s][0] = 0.0; acc[k][h][s][1] = 0.0; }
+      lc.c0 = X0 + 2 * lane;
+      lc.edge = false;
+#pragma unroll
+      for (int h = 0; h < NH; ++h) {
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          const int c = lc.c0 + 64 * h + j;
+          lc.inside[h][j] = c >= 0 && c < P1;
+          lc.colhalo[h][j] = lc.inside[h][j] && (c < R || c >= P1 - R);
+          lc.valid[h][j] = c >= X0 + R * (K - 1) && c < X0 + 64 * NH - R * (K - 1) && c >= R && c < P1 - R;
+          lc.edge = lc.edge || lc.colhalo[h][j] || !lc.inside[h][j];
+        }
+        lc.vec[h] = lc.valid[h][0] && lc.valid[h][1] &&
+                    ((reinterpret_cast<uintptr_t>(out + lc.c0 + 64 * h) & 15) == 0) && ((P1 & 1) == 0);
+      }
       rows_valid_end = min(A + RC, P0 - R);
+      bool mine = !lc.edge;
+#pragma unroll
+      for (int h = 0; h < NH; ++h) mine = mine && lc.vec[h];
+      all_fast = __all_sync(0xffffffffu, mine);
     }
     // stage bookkeeping: input row I of this stage is padded row yb + I
     const int yb = A - K * R + cj * G::SROWS;
     {
-      const int yf = yb - K * R;  // final row produced by input row I = 0
+      const int yf = yb - K * R - (K - 1);  // final row produced by input row I = 0 (one-row lag per stage)
       sc.lo = A - yf;
       sc.hi = rows_valid_end - yf;
       sc.ooff = int64_t(yf) * P1 + lc.c0;
 #pragma unroll
       for (int S = 1; S < K; ++S) {
-        const int ys = yb - S * R;  // stage-S row produced by input row I = 0
+        const int ys = yb - S * R - (S - 1);  // stage-S row produced by input row I = 0
         sc.hlo[S - 1] = R - ys;
         sc.hhi[S - 1] = P0 - R - ys;
         sc.rlo[S - 1] = -ys;
@@ -385,7 +454,11 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
       }
     }
     const double* st = reinterpret_cast<const double*>(ring + slot * G::STAGE);
-    fused_rows<R, SIG, K, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1);
+    bool full = all_fast && sc.lo <= 0 && sc.hi >= G::SROWS;
+#pragma unroll
+    for (int S = 1; S < K; ++S) full = full && sc.hlo[S - 1] <= 0 && sc.hhi[S - 1] >= G::SROWS;
+    if (full) fused_rows<R, SIG, K, NH, true, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1);
+    else fused_rows<R, SIG, K, NH, false, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1);
     __syncwarp();  // every lane is done with this slot before it is refilled
     if (++slot == RDG_NS) { slot = 0; phase ^= 1; }
     if (++cj == SI) { cj = 0; citem += TW; }
@@ -435,10 +508,11 @@ int signature(const Plan& p, RdgParams& prm) {
 template <int R, int SIG, int K, bool TMA>
 cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
                        const RdgParams& prm) {
-  using G = Geom<R>;
+  constexpr int NH = rdg_nh<R, SIG, K>();
+  using G = Geom<R, NH>;
   constexpr int n = 2 * R + 1;
-  constexpr int BS = 64 - 2 * R * (K - 1) - 2 * ((R * (K - 1)) & 1);
-  constexpr int BUFD = ((G::BW + 15) / 16) * 16;
+  constexpr int BS = 64 * NH - 2 * R * (K - 1) - 2 * ((R * (K - 1)) & 1);
+  constexpr int BUFD = G::BUFD;
   const int smem = 128 + RDG_WARPS * (G::WARP_BYTES + 2 * (K - 1) * BUFD * 8);
   static int max_grid = 0;
   if (max_grid == 0) {
@@ -464,7 +538,7 @@ cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream
     if (rc2 <= RDG_RC + n && rc2 >= 4 * K * R && nbands * ((p.N[0] + rc2 - 1) / rc2) <= rounds * TWmax) rc = rc2;
   }
   const int RC = (int)rc;
-  const int SI = (RC + 2 * K * R + G::SROWS - 1) / G::SROWS;
+  const int SI = (RC + 2 * K * R + (K - 1) + G::SROWS - 1) / G::SROWS;
   const int nchunks = (int)((p.N[0] + RC - 1) / RC);
   const int nitems = nbands * nchunks;
   const int grid = (int)std::min<int64_t>(max_grid, (nitems + RDG_WARPS - 1) / RDG_WARPS);
@@ -475,7 +549,7 @@ cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream
 
 template <int R, int SIG, int K>
 cudaError_t rdg_sig(const Plan& p, const double* src, double* dst, cudaStream_t s, const RdgParams& prm) {
-  using G = Geom<R>;
+  using G = Geom<R, rdg_nh<R, SIG, K>()>;
   CUtensorMap map;
   const int64_t padded[2] = {p.P[0], p.P[1]};
   const int box[2] = {G::SROWS, G::BW};
