@@ -163,6 +163,55 @@ void lora_stencil_comm_destroy(lora_comm* c);
 int lora_stencil_dist_exchange_plan(const lora_plan* p, int rank, int nranks, int64_t* kind, int64_t* peer,
                                     int64_t* offset, int64_t* count);
 
+/* ---- multi-GPU: the same slab decomposition with a DEVICE-INITIATED halo exchange ----
+ * (north star (d) "halo exchange over NVLink ... overlapped with interior
+ * compute").  Instead of host-issued ncclSend/ncclRecv after every step, the stencil kernel's
+ * boundary work items store the slab's first/last r interior rows (2D) or planes (3D) straight
+ * into the neighbour's halo through peer memory (NVLink P2P via CUDA IPC, or plain device
+ * pointers within one process) and then publish a per-tile step counter in the neighbour's
+ * memory; the neighbour's boundary items wait for that counter before staging their halo.
+ * Interior tiles never wait, so the exchange overlaps the interior tile by tile and there is no
+ * collective call per step at all.  Results are bitwise equal to lora_stencil_run_dist and to a
+ * single-GPU run of the global grid (same kernels, same per-point arithmetic).
+ *
+ * Engines: the CUDA-core engine (2D, 3D radius <= 2) and the direct comparison kernel, unfused
+ * (one step per launch); other plans return LORA_ERR_UNSUPPORTED.  Every rank's plan has the
+ * same trailing extents and radius (the local n0 may differ).
+ *
+ * Exchange buffers: the communicator owns two padded slabs of the plan's local shape (the
+ * ping-pong pair the neighbours write into) plus the flag words, allocated with cudaMalloc on
+ * the current device (IPC-exportable).  lora_stencil_p2p_buffer exposes them: a caller that
+ * fills buffer 0 directly and passes it as `in_local` (and buffer T%2 as `out_local`) avoids the
+ * copy-in / copy-out.
+ *
+ * A spin-wait that sees no progress for 20 s (a neighbour that never runs) gives up instead of
+ * hanging the GPU and sets a device error word: lora_stencil_p2p_status reports it. */
+typedef struct lora_p2p lora_p2p;
+
+/* Creates this rank's endpoint for plan p (LOCAL shape) on the current device. */
+int lora_stencil_p2p_create(lora_p2p** c, const lora_plan* p, int nranks, int rank);
+/* Size of the opaque exchange handle (128 bytes: a cudaIpcMemHandle_t plus the slab layout). */
+size_t lora_stencil_p2p_handle_size(void);
+/* Writes this endpoint's handle (host bytes) for the neighbours, e.g. via
+ * torch.distributed.all_gather_object. */
+int lora_stencil_p2p_get_handle(const lora_p2p* c, void* handle_out);
+/* Opens the neighbours' handles (rank-1's as lo_handle, rank+1's as hi_handle; NULL where there
+ * is no neighbour) with cudaIpcOpenMemHandle.  Neighbours must live in OTHER processes. */
+int lora_stencil_p2p_connect(lora_p2p* c, const void* lo_handle, const void* hi_handle);
+/* Same-process wiring (one process driving several slabs, on one or several devices; peer
+ * access is enabled where the devices differ).  lo / hi may be NULL. */
+int lora_stencil_p2p_connect_local(lora_p2p* c, const lora_p2p* lo, const lora_p2p* hi);
+/* Device pointer of exchange buffer i (0 or 1), or NULL. */
+double* lora_stencil_p2p_buffer(const lora_p2p* c, int i);
+/* Collective over the connected ranks (every rank calls with the same timesteps), ordered on
+ * `stream`: copy-in (skipped if in_local is buffer 0), T steps with the in-kernel exchange, a
+ * final wait for the neighbours' last rows, copy-out (skipped if out_local is buffer T%2). */
+int lora_stencil_run_dist_p2p(lora_plan* p, lora_p2p* c, const double* in_local, double* out_local,
+                              int64_t timesteps, void* stream);
+/* Synchronises the device and reports a spin-wait timeout (LORA_ERR_CUDA) if one occurred. */
+int lora_stencil_p2p_status(lora_p2p* c);
+void lora_stencil_p2p_destroy(lora_p2p* c);
+
 /* Thread-local message for the last failure on this thread ("" if none). */
 const char* lora_stencil_last_error(void);
 /* Library version string. */

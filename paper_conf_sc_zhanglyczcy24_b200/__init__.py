@@ -75,6 +75,15 @@ _sig = {
     "lora_stencil_run_dist": (ctypes.c_int, [_P, _P, _P, _P, ctypes.c_int64, _P]),
     "lora_stencil_comm_destroy": (None, [_P]),
     "lora_stencil_dist_exchange_plan": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_int, _P, _P, _P, _P]),
+    "lora_stencil_p2p_create": (ctypes.c_int, [_P, _P, ctypes.c_int, ctypes.c_int]),
+    "lora_stencil_p2p_handle_size": (ctypes.c_size_t, []),
+    "lora_stencil_p2p_get_handle": (ctypes.c_int, [_P, _P]),
+    "lora_stencil_p2p_connect": (ctypes.c_int, [_P, _P, _P]),
+    "lora_stencil_p2p_connect_local": (ctypes.c_int, [_P, _P, _P]),
+    "lora_stencil_p2p_buffer": (_P, [_P, ctypes.c_int]),
+    "lora_stencil_run_dist_p2p": (ctypes.c_int, [_P, _P, _P, _P, ctypes.c_int64, _P]),
+    "lora_stencil_p2p_status": (ctypes.c_int, [_P]),
+    "lora_stencil_p2p_destroy": (None, [_P]),
     "lora_stencil_last_error": (ctypes.c_char_p, []),
     "lora_stencil_version": (ctypes.c_char_p, []),
 }
@@ -187,6 +196,51 @@ def lora_stencil_run_dist(plan, comm, in_ptr: int, out_ptr: int, timesteps: int,
 
 def lora_stencil_comm_destroy(comm) -> None:
     _lib.lora_stencil_comm_destroy(comm)
+
+
+def lora_stencil_p2p_create(plan, nranks: int, rank: int):
+    """Device-initiated halo exchange endpoint for `plan` (local slab) on the current device."""
+    c = ctypes.c_void_p(0)
+    _check(_lib.lora_stencil_p2p_create(ctypes.byref(c), plan, int(nranks), int(rank)))
+    return c.value
+
+
+def lora_stencil_p2p_handle_size() -> int:
+    return int(_lib.lora_stencil_p2p_handle_size())
+
+
+def lora_stencil_p2p_get_handle(c) -> bytes:
+    buf = ctypes.create_string_buffer(lora_stencil_p2p_handle_size())
+    _check(_lib.lora_stencil_p2p_get_handle(c, buf))
+    return buf.raw
+
+
+def lora_stencil_p2p_connect(c, lo_handle, hi_handle) -> None:
+    """Other-process neighbours: their handles (bytes) or None where there is no neighbour."""
+    lo = ctypes.create_string_buffer(lo_handle, len(lo_handle)) if lo_handle is not None else None
+    hi = ctypes.create_string_buffer(hi_handle, len(hi_handle)) if hi_handle is not None else None
+    _check(_lib.lora_stencil_p2p_connect(c, lo, hi))
+
+
+def lora_stencil_p2p_connect_local(c, lo, hi) -> None:
+    """Same-process neighbours (endpoint handles or None)."""
+    _check(_lib.lora_stencil_p2p_connect_local(c, lo, hi))
+
+
+def lora_stencil_p2p_buffer(c, i: int) -> int:
+    return int(_lib.lora_stencil_p2p_buffer(c, int(i)) or 0)
+
+
+def lora_stencil_run_dist_p2p(plan, c, in_ptr: int, out_ptr: int, timesteps: int, stream: int = 0) -> None:
+    _check(_lib.lora_stencil_run_dist_p2p(plan, c, in_ptr, out_ptr, int(timesteps), stream or None))
+
+
+def lora_stencil_p2p_status(c) -> None:
+    _check(_lib.lora_stencil_p2p_status(c))
+
+
+def lora_stencil_p2p_destroy(c) -> None:
+    _lib.lora_stencil_p2p_destroy(c)
 
 
 def lora_stencil_dist_exchange_plan(plan, rank: int, nranks: int):

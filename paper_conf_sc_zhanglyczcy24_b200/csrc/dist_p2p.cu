@@ -1,0 +1,333 @@
+// Multi-GPU slab decomposition with a DEVICE-INITIATED halo exchange (
+// include/lora_stencil.h "lora_stencil_p2p_*").  The paper is single-GPU; the exchange
+// step is the north star's (d).
+//
+// Protocol (per run, `base` = the endpoint's epoch, identical on every rank because every rank
+// runs the same sequence of collective calls):
+//   init      copy `in` into buffer 0, the Dirichlet ring of `in` into buffer 1 (its slab-edge
+//             halo rows are rewritten by the neighbour every other step), then publish base + 1 in
+//             every flag unit of each neighbour ("my buffers are ready to be written").
+//   step t    one launch of the unfused stencil kernel buf[(t-1)%2] -> buf[t%2] with P2PArgs:
+//             boundary items wait until the neighbour's flags of the units around them reach
+//             base + t (the neighbour finished step t-1: its edge rows are in my halo, and its own
+//             step t-1 halo reads are done, so I may overwrite its buf[t%2] halo), stage, compute,
+//             store their edge rows locally AND into the neighbour's buf[t%2] halo, then publish
+//             base + 1 + t in the neighbour's flag of their unit.
+//   final     wait until my flags reach base + 1 + T (the neighbours' step-T rows are in my
+//             halo), copy buf[T%2] out; epoch = base + T + 2.
+// Flags are monotonic, so no reset is ever needed.  Every write into a peer's buffer happens
+// after the peer published a value that orders it after the peer's last read of that region.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <climits>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "kernels.hpp"
+#include "lora_stencil.h"
+#include "p2p.cuh"
+#include "plan.hpp"
+
+namespace {
+
+constexpr uint32_t kMagic = 0x4c503250u;  // "LP2P"
+constexpr uint32_t kVersion = 1;
+
+struct Blob {                     // the 128-byte exchange handle
+  uint32_t magic, version;
+  cudaIpcMemHandle_t ipc;         // 64 bytes
+  int64_t n0, row;                // local interior extent along the slab axis, elements per padded row/plane
+  int32_t nunits, R;
+  uint64_t off_buf0, off_buf1, off_flags;   // byte offsets inside the allocation
+};
+static_assert(sizeof(Blob) <= 128, "exchange handle must fit 128 bytes");
+
+struct Peer {
+  bool present = false;
+  double* buf[2] = {nullptr, nullptr};
+  unsigned long long* flags = nullptr;   // the peer's flag array [2][nunits]
+  int64_t n0 = 0;
+  void* ipc_base = nullptr;              // cudaIpcOpenMemHandle mapping to close
+};
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+__global__ void p2p_publish_kernel(unsigned long long* flags, int n, unsigned long long val) {
+  __threadfence_system();
+  for (int i = threadIdx.x; i < n; i += blockDim.x) lora::p2p_st_release(flags + i, val);
+}
+
+__global__ void p2p_wait_kernel(const unsigned long long* flags, int n, unsigned long long val, int* err) {
+  if (threadIdx.x == 0) lora::p2p_wait_units(flags, 0, n - 1, val, err);
+  __syncthreads();
+}
+
+}  // namespace
+
+struct lora_p2p {
+  int rank = 0, nranks = 1, device = -1;
+  int ndim = 2, R = 1, engine = 0;
+  int64_t N[3] = {1, 1, 1};
+  int64_t row = 0;                 // elements per padded row (2D) / plane (3D)
+  size_t elems = 0;
+  int nunits = 0, nux = 0;
+  char* mem = nullptr;
+  size_t bytes = 0;
+  uint64_t off_buf[2] = {0, 0}, off_flags = 0, off_err = 0;
+  double* buf[2] = {nullptr, nullptr};
+  unsigned long long* flags = nullptr;   // [0][u]: written by rank-1, [1][u]: written by rank+1
+  int* err = nullptr;
+  Peer lo, hi;
+  unsigned long long epoch = 0;
+};
+
+namespace {
+
+Peer local_peer(const lora_p2p* o) {
+  Peer q;
+  q.present = true;
+  q.buf[0] = o->buf[0];
+  q.buf[1] = o->buf[1];
+  q.flags = o->flags;
+  q.n0 = o->N[0];
+  return q;
+}
+
+int check_layout(const lora_p2p* c, int64_t row, int nunits, int R, const char* who) {
+  if (row != c->row || nunits != c->nunits || R != c->R)
+    return lora::fail(LORA_ERR_INVALID_ARG, std::string(who) + " neighbour's slab layout (trailing extents / radius) differs");
+  return LORA_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+size_t lora_stencil_p2p_handle_size(void) { return 128; }
+
+int lora_stencil_p2p_create(lora_p2p** out, const lora_plan* p, int nranks, int rank) {
+  using namespace lora;
+  if (!out || !p || nranks < 1 || rank < 0 || rank >= nranks) return fail(LORA_ERR_INVALID_ARG, "bad p2p arguments");
+  *out = nullptr;
+  int nux = 0;
+  const int nunits = p2p_units(*p, &nux);
+  if (nunits <= 0)
+    return fail(LORA_ERR_UNSUPPORTED, "device-initiated exchange: needs the CUDA-core engine (2D, 3D radius <= 2) or the direct kernel");
+  if (nranks > 1 && p->N[0] < p->R) return fail(LORA_ERR_INVALID_ARG, "each slab needs >= radius rows/planes");
+  lora_p2p* c = new (std::nothrow) lora_p2p();
+  if (!c) return fail(LORA_ERR_OOM, "out of host memory");
+  c->rank = rank;
+  c->nranks = nranks;
+  c->ndim = p->ndim;
+  c->R = p->R;
+  c->engine = p->engine;
+  for (int i = 0; i < 3; ++i) c->N[i] = p->N[i];
+  c->row = p->ndim == 2 ? p->P[1] : p->P[1] * p->P[2];
+  c->elems = p->elems;
+  c->nunits = nunits;
+  c->nux = nux;
+  const size_t bb = align_up(p->elems * sizeof(double), 256);
+  c->off_buf[0] = 0;
+  c->off_buf[1] = bb;
+  c->off_flags = 2 * bb;
+  c->off_err = c->off_flags + align_up(2 * size_t(nunits) * sizeof(unsigned long long), 256);
+  c->bytes = c->off_err + 256;
+  cudaGetDevice(&c->device);
+  cudaError_t e = cudaMalloc(&c->mem, c->bytes);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    delete c;
+    return fail(LORA_ERR_OOM, "cudaMalloc(p2p exchange buffers) failed");
+  }
+  c->buf[0] = reinterpret_cast<double*>(c->mem + c->off_buf[0]);
+  c->buf[1] = reinterpret_cast<double*>(c->mem + c->off_buf[1]);
+  c->flags = reinterpret_cast<unsigned long long*>(c->mem + c->off_flags);
+  c->err = reinterpret_cast<int*>(c->mem + c->off_err);
+  {  // load the helper kernels now: with lazy module loading a first launch while a neighbour's
+     // kernel spins on this process's signals could otherwise wait on a context-wide load
+    cudaFuncAttributes fa;
+    cudaFuncGetAttributes(&fa, p2p_publish_kernel);
+    cudaFuncGetAttributes(&fa, p2p_wait_kernel);
+  }
+  e = cudaMemset(c->mem + c->off_flags, 0, c->bytes - c->off_flags);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) {
+    cudaFree(c->mem);
+    delete c;
+    return cuda_fail(e, "p2p flag initialisation");
+  }
+  *out = c;
+  return LORA_OK;
+}
+
+int lora_stencil_p2p_get_handle(const lora_p2p* c, void* handle_out) {
+  using namespace lora;
+  if (!c || !handle_out) return fail(LORA_ERR_INVALID_ARG, "NULL endpoint or handle buffer");
+  Blob b;
+  std::memset(&b, 0, sizeof(b));
+  b.magic = kMagic;
+  b.version = kVersion;
+  cudaError_t e = cudaIpcGetMemHandle(&b.ipc, c->mem);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaIpcGetMemHandle");
+  b.n0 = c->N[0];
+  b.row = c->row;
+  b.nunits = c->nunits;
+  b.R = c->R;
+  b.off_buf0 = c->off_buf[0];
+  b.off_buf1 = c->off_buf[1];
+  b.off_flags = c->off_flags;
+  std::memset(handle_out, 0, 128);
+  std::memcpy(handle_out, &b, sizeof(b));
+  return LORA_OK;
+}
+
+int lora_stencil_p2p_connect(lora_p2p* c, const void* lo_handle, const void* hi_handle) {
+  using namespace lora;
+  if (!c) return fail(LORA_ERR_INVALID_ARG, "NULL endpoint");
+  if ((c->rank > 0) != (lo_handle != nullptr) || (c->rank < c->nranks - 1) != (hi_handle != nullptr))
+    return fail(LORA_ERR_INVALID_ARG, "a handle is needed exactly for each existing neighbour (rank-1, rank+1)");
+  const void* hs[2] = {lo_handle, hi_handle};
+  Peer* ps[2] = {&c->lo, &c->hi};
+  for (int k = 0; k < 2; ++k) {
+    if (!hs[k]) continue;
+    Blob b;
+    std::memcpy(&b, hs[k], sizeof(b));
+    if (b.magic != kMagic || b.version != kVersion) return fail(LORA_ERR_INVALID_ARG, "not a lora p2p handle");
+    int rc = check_layout(c, b.row, b.nunits, b.R, k == 0 ? "lower" : "upper");
+    if (rc) return rc;
+    void* base = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&base, b.ipc, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaIpcOpenMemHandle (neighbour in this process? use p2p_connect_local)");
+    Peer& q = *ps[k];
+    if (q.ipc_base) cudaIpcCloseMemHandle(q.ipc_base);
+    q.present = true;
+    q.ipc_base = base;
+    q.buf[0] = reinterpret_cast<double*>(static_cast<char*>(base) + b.off_buf0);
+    q.buf[1] = reinterpret_cast<double*>(static_cast<char*>(base) + b.off_buf1);
+    q.flags = reinterpret_cast<unsigned long long*>(static_cast<char*>(base) + b.off_flags);
+    q.n0 = b.n0;
+  }
+  return LORA_OK;
+}
+
+int lora_stencil_p2p_connect_local(lora_p2p* c, const lora_p2p* lo, const lora_p2p* hi) {
+  using namespace lora;
+  if (!c) return fail(LORA_ERR_INVALID_ARG, "NULL endpoint");
+  const lora_p2p* os[2] = {lo, hi};
+  Peer* ps[2] = {&c->lo, &c->hi};
+  for (int k = 0; k < 2; ++k) {
+    if (!os[k]) { *ps[k] = Peer(); continue; }
+    int rc = check_layout(c, os[k]->row, os[k]->nunits, os[k]->R, k == 0 ? "lower" : "upper");
+    if (rc) return rc;
+    if (os[k]->device != c->device) {
+      int ok = 0;
+      cudaDeviceCanAccessPeer(&ok, c->device, os[k]->device);
+      if (!ok) return fail(LORA_ERR_UNSUPPORTED, "no peer access between the two devices");
+      cudaError_t e = cudaDeviceEnablePeerAccess(os[k]->device, 0);
+      if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return cuda_fail(e, "cudaDeviceEnablePeerAccess");
+      cudaGetLastError();
+    }
+    *ps[k] = local_peer(os[k]);
+  }
+  return LORA_OK;
+}
+
+double* lora_stencil_p2p_buffer(const lora_p2p* c, int i) {
+  if (!c || i < 0 || i > 1) return nullptr;
+  return c->buf[i];
+}
+
+int lora_stencil_run_dist_p2p(lora_plan* p, lora_p2p* c, const double* in_local, double* out_local,
+                              int64_t timesteps, void* stream) {
+  using namespace lora;
+  if (!p || !c || !in_local || !out_local) return fail(LORA_ERR_INVALID_ARG, "NULL plan, endpoint, in or out");
+  if (timesteps < 0) return fail(LORA_ERR_INVALID_ARG, "timesteps must be >= 0");
+  if (p->ndim != c->ndim || p->R != c->R || p->engine != c->engine || p->N[0] != c->N[0] || p->N[1] != c->N[1] ||
+      p->N[2] != c->N[2])
+    return fail(LORA_ERR_INVALID_ARG, "plan does not match the endpoint's slab");
+  if ((c->rank > 0 && !c->lo.present) || (c->rank < c->nranks - 1 && !c->hi.present))
+    return fail(LORA_ERR_INVALID_ARG, "endpoint is not connected to its neighbours");
+  const size_t bytes = p->elems * sizeof(double);
+  const char* a = reinterpret_cast<const char*>(in_local);
+  const char* b = reinterpret_cast<const char*>(out_local);
+  // zero-copy use of the exchange buffers: in = buffer 0 and out = buffer T%2 may coincide (T even),
+  // `in` is fully consumed by step 1 and its halo is buffer 0's own
+  const bool zero_copy = in_local == c->buf[0] && out_local == c->buf[timesteps % 2];
+  if (!zero_copy && a < b + bytes && b < a + bytes) return fail(LORA_ERR_ALIAS, "in and out overlap");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  int dev = -1;
+  cudaGetDevice(&dev);
+  if (dev != c->device) return fail(LORA_ERR_INVALID_ARG, "endpoint is bound to another CUDA device");
+  int rc = ensure_device(*p, false);
+  if (rc) return rc;
+  if (timesteps == 0) {
+    cudaError_t e = cudaMemcpyAsync(out_local, in_local, bytes, cudaMemcpyDeviceToDevice, s);
+    return e == cudaSuccess ? LORA_OK : cuda_fail(e, "cudaMemcpyAsync");
+  }
+  const unsigned long long base = c->epoch;
+  cudaError_t e = cudaSuccess;
+  if (in_local != c->buf[0]) e = cudaMemcpyAsync(c->buf[0], in_local, bytes, cudaMemcpyDeviceToDevice, s);
+  if (e != cudaSuccess) return cuda_fail(e, "copy-in");
+  if ((e = launch_copy_halo(*p, in_local, c->buf[1], s)) != cudaSuccess) return cuda_fail(e, "copy_halo launch");
+  // my buffers are ready: neighbours may write their step-1 rows into buf[1]
+  if (c->lo.present) p2p_publish_kernel<<<1, 256, 0, s>>>(c->lo.flags + c->nunits, c->nunits, base + 1);
+  if (c->hi.present) p2p_publish_kernel<<<1, 256, 0, s>>>(c->hi.flags, c->nunits, base + 1);
+  if ((e = cudaGetLastError()) != cudaSuccess) return cuda_fail(e, "p2p publish launch");
+  P2PArgs d;
+  d.active = 1;
+  d.nunits = c->nunits;
+  d.nux = c->nux;
+  d.wait_lo = c->lo.present ? c->flags : nullptr;
+  d.wait_hi = c->hi.present ? c->flags + c->nunits : nullptr;
+  d.sig_lo = c->lo.present ? c->lo.flags + c->nunits : nullptr;   // I am the lower neighbour's upper side
+  d.sig_hi = c->hi.present ? c->hi.flags : nullptr;               // ... and the upper neighbour's lower side
+  d.off_lo = c->lo.present ? (long long)(c->lo.n0 * c->row) : 0;
+  d.off_hi = -(long long)(c->N[0] * c->row);
+  d.err = c->err;
+  for (int64_t t = 1; t <= timesteps; ++t) {
+    d.dst_lo = c->lo.present ? c->lo.buf[t % 2] : nullptr;
+    d.dst_hi = c->hi.present ? c->hi.buf[t % 2] : nullptr;
+    d.wait_val = base + (unsigned long long)t;
+    d.sig_val = base + 1 + (unsigned long long)t;
+    e = launch_step_p2p(*p, c->buf[(t - 1) % 2], c->buf[t % 2], s, d);
+    if (e != cudaSuccess) return cuda_fail(e, "stencil kernel launch (p2p)");
+  }
+  const unsigned long long fin = base + 1 + (unsigned long long)timesteps;
+  if (c->lo.present) p2p_wait_kernel<<<1, 32, 0, s>>>(c->flags, c->nunits, fin, c->err);
+  if (c->hi.present) p2p_wait_kernel<<<1, 32, 0, s>>>(c->flags + c->nunits, c->nunits, fin, c->err);
+  if ((e = cudaGetLastError()) != cudaSuccess) return cuda_fail(e, "p2p wait launch");
+  double* last = c->buf[timesteps % 2];
+  if (out_local != last) {
+    e = cudaMemcpyAsync(out_local, last, bytes, cudaMemcpyDeviceToDevice, s);
+    if (e != cudaSuccess) return cuda_fail(e, "copy-out");
+  }
+  c->epoch = base + (unsigned long long)timesteps + 2;
+  if (sync_check()) {
+    cudaError_t ce = cudaStreamSynchronize(s);
+    if (ce != cudaSuccess) return cuda_fail(ce, "LORA_SYNC_CHECK stream sync");
+    return lora_stencil_p2p_status(c);
+  }
+  return LORA_OK;
+}
+
+int lora_stencil_p2p_status(lora_p2p* c) {
+  using namespace lora;
+  if (!c) return fail(LORA_ERR_INVALID_ARG, "NULL endpoint");
+  int h = 0;
+  cudaError_t e = cudaMemcpy(&h, c->err, sizeof(int), cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return cuda_fail(e, "p2p status read");
+  if (h) return fail(LORA_ERR_CUDA, "device-initiated halo exchange: a neighbour's step counter did not advance for 20 s");
+  return LORA_OK;
+}
+
+void lora_stencil_p2p_destroy(lora_p2p* c) {
+  if (!c) return;
+  if (c->lo.ipc_base) cudaIpcCloseMemHandle(c->lo.ipc_base);
+  if (c->hi.ipc_base) cudaIpcCloseMemHandle(c->hi.ipc_base);
+  if (c->mem) cudaFree(c->mem);
+  delete c;
+}
+
+}  // extern "C"

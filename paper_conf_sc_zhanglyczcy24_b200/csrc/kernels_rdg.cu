@@ -21,6 +21,7 @@
 #include <cstring>
 
 #include "kernels.hpp"
+#include "p2p.cuh"
 #include "pipe.cuh"
 
 namespace lora {
@@ -198,6 +199,8 @@ template <int K>
 struct StageCtx {
   int lo, hi;               // final rows: stage-local rows I with lo <= I < hi are stored
   int64_t ooff;             // element offset of (final row for I = 0, lane column c0)
+  int rem_lo, rem_hi;       // device-initiated exchange: rows I < rem_lo also go to the lower
+                            // neighbour's halo, rows I >= rem_hi to the upper one's
   int hlo[K], hhi[K];       // intermediate stage S: row I is halo if I < hlo or I >= hhi
   int rlo[K], rhi[K];       //                     row I is inside the array if rlo <= I < rhi
   int64_t ioff[K];          //                     element offset of (row for I = 0, column 0) in `in`
@@ -223,7 +226,7 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
                                            double (&acc)[K][NH][2 * R + 1][2], const RdgParams& P,
                                            double* __restrict__ bufs, int par, const double* __restrict__ in,
                                            double* __restrict__ out, int64_t P1, const StageCtx<K>& sc,
-                                           const LaneCtx<NH>& lc) {
+                                           const LaneCtx<NH>& lc, const P2PArgs& dp) {
   constexpr int n = 2 * R + 1;
   constexpr int BUFD = Geom<R, NH>::BUFD;
   constexpr int Is = pmod(I0 - (S - 1) * (R + 1), n);   // ring index of stage S's input row (any per-stage constant)
@@ -271,33 +274,39 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
     for (int h = 0; h < NH; ++h) *reinterpret_cast<double2*>(o + 64 * h) = make_double2(v[h][0], v[h][1]);
   } else {
     if (I >= sc.lo && I < sc.hi) {
-      double* o = out + sc.ooff + int64_t(I) * P1;
+      const int64_t e = sc.ooff + int64_t(I) * P1;
+      // the row goes to this slab and, for the first / last R interior rows of a slab with a
+      // neighbour there, into that neighbour's halo as well (peer memory, csrc/dist_p2p.cu)
+      const int nd = 1 + (I < sc.rem_lo ? 1 : 0) + (I >= sc.rem_hi ? 1 : 0);
+      for (int d = 0; d < nd; ++d) {
+        double* o = d == 0 ? out + e : (I < sc.rem_lo && d == 1 ? dp.dst_lo + (e + dp.off_lo) : dp.dst_hi + (e + dp.off_hi));
 #pragma unroll
-      for (int h = 0; h < NH; ++h) {
-        if (lc.vec[h]) {
-          *reinterpret_cast<double2*>(o + 64 * h) = make_double2(v[h][0], v[h][1]);
-        } else {
-          if (lc.valid[h][0]) o[64 * h] = v[h][0];
-          if (lc.valid[h][1]) o[64 * h + 1] = v[h][1];
+        for (int h = 0; h < NH; ++h) {
+          if (lc.vec[h]) {
+            *reinterpret_cast<double2*>(o + 64 * h) = make_double2(v[h][0], v[h][1]);
+          } else {
+            if (lc.valid[h][0]) o[64 * h] = v[h][0];
+            if (lc.valid[h][1]) o[64 * h + 1] = v[h][1];
+          }
         }
       }
     }
   }
-  if constexpr (S > 1) fused_iter<R, SIG, K, NH, FULL, I0, I, S - 1>(st_row, p, acc, P, bufs, par, in, out, P1, sc, lc);
+  if constexpr (S > 1) fused_iter<R, SIG, K, NH, FULL, I0, I, S - 1>(st_row, p, acc, P, bufs, par, in, out, P1, sc, lc, dp);
 }
 
 template <int R, int SIG, int K, int NH, bool FULL, int I>
 __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p, double (&acc)[K][NH][2 * R + 1][2],
                                            const RdgParams& P, double* __restrict__ bufs,
                                            const double* __restrict__ in, double* __restrict__ out, int64_t P1,
-                                           const StageCtx<K>& sc, const LaneCtx<NH>& lc, int par0) {
+                                           const StageCtx<K>& sc, const LaneCtx<NH>& lc, int par0, const P2PArgs& dp) {
   constexpr int n = 2 * R + 1;
   if constexpr (I < Geom<R, NH>::SROWS) {
     constexpr int OFF = pmod(R - K * R, n);  // q0 mod n (RC is a multiple of n)
     fused_iter<R, SIG, K, NH, FULL, pmod(I + OFF, n), I, K>(st + I * Geom<R, NH>::BW, p, acc, P, bufs, (par0 + I) & 1,
-                                                            in, out, P1, sc, lc);
+                                                            in, out, P1, sc, lc, dp);
     if constexpr (K > 1) __syncwarp();
-    fused_rows<R, SIG, K, NH, FULL, I + 1>(st, p, acc, P, bufs, in, out, P1, sc, lc, par0);
+    fused_rows<R, SIG, K, NH, FULL, I + 1>(st, p, acc, P, bufs, in, out, P1, sc, lc, par0, dp);
   }
 }
 
@@ -331,7 +340,8 @@ template <int R, int SIG, int K, bool TMA>
 __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d_kernel(const double* __restrict__ in, double* __restrict__ out,
                                                               int64_t N0, int64_t N1, int nbands, int nitems, int RC,
                                                               int SI, const __grid_constant__ CUtensorMap tmap,
-                                                              const __grid_constant__ RdgParams prm) {
+                                                              const __grid_constant__ RdgParams prm,
+                                                              const __grid_constant__ P2PArgs dp) {
   constexpr int NH = rdg_nh<R, SIG, K>();
   using G = Geom<R, NH>;
   constexpr int SG = (R * (K - 1)) & 1;           // shift keeping the staged origin even (TMA: 16-B aligned start)
@@ -356,16 +366,35 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
   }
   __syncwarp();
   // item geometry: band b -> lane column 0 at padded column X0; chunk c -> final rows from A
+  const int nch = nitems / nbands;
   auto geom = [&](int item, int& X0, int& A) {
-    const int band = item % nbands, chunk = item / nbands;
+    const int band = item % nbands;
+    const int chunk = dp.active ? p2p_chunk_order(item / nbands, nch) : item / nbands;
     X0 = R + band * BS - R * (K - 1) - SG;
     A = R + chunk * RC;
+  };
+  // device-initiated exchange (K = 1 only): the item holding the first (last) R interior rows of
+  // the slab touches the lower (upper) neighbour; the host keeps that item unique per band
+  auto touches = [&](int A_, bool& lo, bool& hi) {
+    lo = dp.active && dp.dst_lo != nullptr && A_ < 2 * R;
+    hi = dp.active && dp.dst_hi != nullptr && A_ + RC - 1 >= N0;
   };
   // producer position (next stage to stage into the ring)
   int pitem = gw, pj = 0, pX0 = 0, pA = 0;
   if (gw < nitems) geom(pitem, pX0, pA);
   auto issue_next = [&](int slot) {
     const int x = pX0 - R, y = pA - K * R + pj * G::SROWS;
+    if (dp.active && pj == 0) {  // the halo this item stages was written by a neighbour: wait for it
+      bool lo, hi;
+      touches(pA, lo, hi);
+      if (lane == 0 && (lo || hi)) {
+        const int b = pitem % nbands, u0 = max(b - 1, 0), u1 = min(b + 1, nbands - 1);
+        if (lo) p2p_wait_units(dp.wait_lo, u0, u1, dp.wait_val, dp.err);
+        if (hi) p2p_wait_units(dp.wait_hi, u0, u1, dp.wait_val, dp.err);
+        fence_proxy_async_global();
+      }
+      __syncwarp();
+    }
     double* dst = reinterpret_cast<double*>(ring + slot * G::STAGE);
     if constexpr (TMA) {
       if (lane == 0) {  // x is even by construction; negative origins are zero-filled by TMA
@@ -397,6 +426,7 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
   StageCtx<K> sc{};
   int citem = gw, cj = 0, X0 = 0, A = 0, rows_valid_end = 0;
   bool all_fast = false;   // every lane of the item: 16-byte stores, no column halo / outside column
+  bool t_lo = false, t_hi = false;   // the current item touches the lower / upper neighbour
   int slot = 0, phase = 0;
   for (int q = 0; q < nstages; ++q) {
     if (q + RDG_NS - 1 < nstages) issue_next((slot + RDG_NS - 1) % RDG_NS);
@@ -435,6 +465,7 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
 #pragma unroll
       for (int h = 0; h < NH; ++h) mine = mine && lc.vec[h];
       all_fast = __all_sync(0xffffffffu, mine);
+      touches(A, t_lo, t_hi);
     }
     // stage bookkeeping: input row I of this stage is padded row yb + I
     const int yb = A - K * R + cj * G::SROWS;
@@ -443,6 +474,8 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
       sc.lo = A - yf;
       sc.hi = rows_valid_end - yf;
       sc.ooff = int64_t(yf) * P1 + lc.c0;
+      sc.rem_lo = t_lo ? 2 * R - yf : INT_MIN;          // padded rows [R, 2R)
+      sc.rem_hi = t_hi ? (int)N0 - yf : INT_MAX;        // padded rows [N0, N0 + R)
 #pragma unroll
       for (int S = 1; S < K; ++S) {
         const int ys = yb - S * R - (S - 1);  // stage-S row produced by input row I = 0
@@ -454,14 +487,19 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
       }
     }
     const double* st = reinterpret_cast<const double*>(ring + slot * G::STAGE);
-    bool full = all_fast && sc.lo <= 0 && sc.hi >= G::SROWS;
+    bool full = all_fast && sc.lo <= 0 && sc.hi >= G::SROWS && sc.rem_lo <= 0 && sc.rem_hi >= G::SROWS;
 #pragma unroll
     for (int S = 1; S < K; ++S) full = full && sc.hlo[S - 1] <= 0 && sc.hhi[S - 1] >= G::SROWS;
-    if (full) fused_rows<R, SIG, K, NH, true, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1);
-    else fused_rows<R, SIG, K, NH, false, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1);
+    if (full) fused_rows<R, SIG, K, NH, true, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp);
+    else fused_rows<R, SIG, K, NH, false, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp);
     __syncwarp();  // every lane is done with this slot before it is refilled
     if (++slot == RDG_NS) { slot = 0; phase ^= 1; }
-    if (++cj == SI) { cj = 0; citem += TW; }
+    if (++cj == SI) {
+      if (t_lo) p2p_signal_warp(dp.sig_lo, citem % nbands, dp.sig_val);   // my edge rows are in its halo,
+      if (t_hi) p2p_signal_warp(dp.sig_hi, citem % nbands, dp.sig_val);   // my halo reads are done
+      cj = 0;
+      citem += TW;
+    }
   }
 }
 
@@ -507,7 +545,7 @@ int signature(const Plan& p, RdgParams& prm) {
 
 template <int R, int SIG, int K, bool TMA>
 cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
-                       const RdgParams& prm) {
+                       const RdgParams& prm, const P2PArgs* d) {
   constexpr int NH = rdg_nh<R, SIG, K>();
   using G = Geom<R, NH>;
   constexpr int n = 2 * R + 1;
@@ -537,32 +575,46 @@ cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream
     rc2 = ((rc2 + n - 1) / n) * n;
     if (rc2 <= RDG_RC + n && rc2 >= 4 * K * R && nbands * ((p.N[0] + rc2 - 1) / rc2) <= rounds * TWmax) rc = rc2;
   }
+  if (d && d->active && rc < p.N[0]) {
+    // device-initiated exchange: exactly one chunk per band may hold the last R interior rows
+    // (the last chunk must have >= R rows), so that one item per band and side signals
+    int64_t ok = 0;
+    for (int64_t c = rc; c <= rc + 40 * n && !ok; c += n) {
+      const int64_t rem = p.N[0] % c;
+      if (rem == 0 || rem >= R) ok = c;
+    }
+    rc = ok ? ok : ((p.N[0] + n - 1) / n) * n;
+  }
   const int RC = (int)rc;
   const int SI = (RC + 2 * K * R + (K - 1) + G::SROWS - 1) / G::SROWS;
   const int nchunks = (int)((p.N[0] + RC - 1) / RC);
   const int nitems = nbands * nchunks;
   const int grid = (int)std::min<int64_t>(max_grid, (nitems + RDG_WARPS - 1) / RDG_WARPS);
+  static const P2PArgs none{};
   rdg2d_kernel<R, SIG, K, TMA><<<grid, RDG_WARPS * 32, smem, s>>>(src, dst, p.N[0], p.N[1], nbands, nitems, RC, SI,
-                                                                   map, prm);
+                                                                   map, prm, d ? *d : none);
   return cudaGetLastError();
 }
 
 template <int R, int SIG, int K>
-cudaError_t rdg_sig(const Plan& p, const double* src, double* dst, cudaStream_t s, const RdgParams& prm) {
+cudaError_t rdg_sig(const Plan& p, const double* src, double* dst, cudaStream_t s, const RdgParams& prm,
+                    const P2PArgs* d = nullptr) {
   using G = Geom<R, rdg_nh<R, SIG, K>()>;
   CUtensorMap map;
   const int64_t padded[2] = {p.P[0], p.P[1]};
   const int box[2] = {G::SROWS, G::BW};
   if (!p.force_no_tma && encode_tmap(&map, src, 2, padded, box))
-    return rdg_launch<R, SIG, K, true>(p, src, dst, s, map, prm);
+    return rdg_launch<R, SIG, K, true>(p, src, dst, s, map, prm, d);
   std::memset(&map, 0, sizeof(map));
-  return rdg_launch<R, SIG, K, false>(p, src, dst, s, map, prm);
+  return rdg_launch<R, SIG, K, false>(p, src, dst, s, map, prm, d);
 }
 
 constexpr int max_fuse(int R) { return R == 1 ? 4 : (R == 2 ? 3 : 2); }
 
 template <int R, int SIG>
-cudaError_t rdg_k(const Plan& p, const double* src, double* dst, cudaStream_t s, const RdgParams& prm, int k) {
+cudaError_t rdg_k(const Plan& p, const double* src, double* dst, cudaStream_t s, const RdgParams& prm, int k,
+                  const P2PArgs* d = nullptr) {
+  if (d) return k == 1 ? rdg_sig<R, SIG, 1>(p, src, dst, s, prm, d) : cudaErrorNotSupported;
   if constexpr (SIG == SIG_FULL || SIG == SIG_DIRECT) {
     if (k != 1) return cudaErrorNotSupported;
     return rdg_sig<R, SIG, 1>(p, src, dst, s, prm);
@@ -578,15 +630,15 @@ cudaError_t rdg_k(const Plan& p, const double* src, double* dst, cudaStream_t s,
 }
 
 template <int R>
-cudaError_t rdg_r(const Plan& p, const double* src, double* dst, cudaStream_t s, int k) {
+cudaError_t rdg_r(const Plan& p, const double* src, double* dst, cudaStream_t s, int k, const P2PArgs* d = nullptr) {
   RdgParams prm;
   const int sig = signature(p, prm);
-  if (sig == SIG_PMA) return rdg_k<R, SIG_PMA>(p, src, dst, s, prm, k);
+  if (sig == SIG_PMA) return rdg_k<R, SIG_PMA>(p, src, dst, s, prm, k, d);
   if constexpr (R >= 3) {
-    if (sig == SIG_ROWS) return rdg_k<R, SIG_ROWS>(p, src, dst, s, prm, k);
+    if (sig == SIG_ROWS) return rdg_k<R, SIG_ROWS>(p, src, dst, s, prm, k, d);
   }
-  if (sig == SIG_STAR) return rdg_k<R, SIG_STAR>(p, src, dst, s, prm, k);
-  if (sig == SIG_FULL) return rdg_k<R, SIG_FULL>(p, src, dst, s, prm, k);
+  if (sig == SIG_STAR) return rdg_k<R, SIG_STAR>(p, src, dst, s, prm, k, d);
+  if (sig == SIG_FULL) return rdg_k<R, SIG_FULL>(p, src, dst, s, prm, k, d);
   return cudaErrorNotSupported;
 }
 
@@ -599,7 +651,8 @@ bool rdg2d_supported(const Plan& p) {
   return signature(p, prm) >= 0;
 }
 
-cudaError_t launch_direct2d_stream(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+namespace {
+cudaError_t direct2d(const Plan& p, const double* src, double* dst, cudaStream_t s, const P2PArgs* d) {
   if (p.ndim != 2) return cudaErrorInvalidValue;
   RdgParams prm;
   std::memset(&prm, 0, sizeof(prm));
@@ -607,12 +660,17 @@ cudaError_t launch_direct2d_stream(const Plan& p, const double* src, double* dst
   for (int i = 0; i < n; ++i)
     for (int j = 0; j < n; ++j) prm.u[i][j] = p.W[size_t(i) * n + j];
   switch (p.R) {
-    case 1: return rdg_sig<1, SIG_DIRECT, 1>(p, src, dst, s, prm);
-    case 2: return rdg_sig<2, SIG_DIRECT, 1>(p, src, dst, s, prm);
-    case 3: return rdg_sig<3, SIG_DIRECT, 1>(p, src, dst, s, prm);
-    case 4: return rdg_sig<4, SIG_DIRECT, 1>(p, src, dst, s, prm);
+    case 1: return rdg_sig<1, SIG_DIRECT, 1>(p, src, dst, s, prm, d);
+    case 2: return rdg_sig<2, SIG_DIRECT, 1>(p, src, dst, s, prm, d);
+    case 3: return rdg_sig<3, SIG_DIRECT, 1>(p, src, dst, s, prm, d);
+    case 4: return rdg_sig<4, SIG_DIRECT, 1>(p, src, dst, s, prm, d);
   }
   return cudaErrorInvalidValue;
+}
+}  // namespace
+
+cudaError_t launch_direct2d_stream(const Plan& p, const double* src, double* dst, cudaStream_t s) {
+  return direct2d(p, src, dst, s, nullptr);
 }
 
 int rdg2d_max_fuse(const Plan& p) {
@@ -622,6 +680,30 @@ int rdg2d_max_fuse(const Plan& p) {
   const int sig = signature(p, prm);
   if (sig < 0 || sig == SIG_FULL) return 1;
   return max_fuse(p.R);
+}
+
+// Flag units per side of the device-initiated exchange (csrc/dist_p2p.cu): the 64-column bands of
+// the unfused 2D stream kernel; 3D: the 64 x BY columns of rdg3d_kernel.
+int p2p_units(const Plan& p, int* nux) {
+  if (nux) *nux = 0;
+  if (p.ndim == 3) return rdg3d_p2p_units(p, nux);
+  if (p.ndim != 2 || (p.engine != LORA_ENGINE_RDG_CUDA && p.engine != LORA_ENGINE_DIRECT)) return 0;
+  if (p.engine == LORA_ENGINE_RDG_CUDA && !rdg2d_supported(p)) return 0;
+  return (int)((p.N[1] + 63) / 64);
+}
+
+cudaError_t launch_step_p2p(const Plan& p, const double* src, double* dst, cudaStream_t s, const P2PArgs& d) {
+  if (p.ndim == 3) return launch_rdg3d_p2p(p, src, dst, s, d);
+  if (p.ndim != 2) return cudaErrorNotSupported;
+  if (p.engine == LORA_ENGINE_DIRECT) return direct2d(p, src, dst, s, &d);
+  if (p.engine != LORA_ENGINE_RDG_CUDA) return cudaErrorNotSupported;
+  switch (p.R) {
+    case 1: return rdg_r<1>(p, src, dst, s, 1, &d);
+    case 2: return rdg_r<2>(p, src, dst, s, 1, &d);
+    case 3: return rdg_r<3>(p, src, dst, s, 1, &d);
+    case 4: return rdg_r<4>(p, src, dst, s, 1, &d);
+  }
+  return cudaErrorInvalidValue;
 }
 
 cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s, int k) {

@@ -20,6 +20,7 @@
 #include <vector>
 
 #include "kernels.hpp"
+#include "p2p.cuh"
 #include "pipe.cuh"
 
 namespace lora {
@@ -190,7 +191,8 @@ template <int R, class SG, bool TMA>
 __global__ void __launch_bounds__(R3_WARPS * 32, RDG3_MINB) rdg3d_kernel(const double* __restrict__ in, double* __restrict__ out,
                                                                  int64_t N0, int64_t N1, int64_t N2, int nbx, int nby,
                                                                  int nitems, int ZC, int SI, const __grid_constant__ CUtensorMap tmap,
-                                                                 const __grid_constant__ R3Params prm) {
+                                                                 const __grid_constant__ R3Params prm,
+                                                                 const __grid_constant__ P2PArgs dp) {
   using G = G3<R>;
   constexpr int n = 2 * R + 1;
   extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -209,17 +211,39 @@ __global__ void __launch_bounds__(R3_WARPS * 32, RDG3_MINB) rdg3d_kernel(const d
   __syncwarp();
   // item -> (x band, y block, z chunk); producer and consumer walk their stage sequences with
   // incremental counters (one division set per item, none per plane)
+  const int nbz = nitems / (nbx * nby);
   auto geom = [&](int item, int& bx0, int& by0, int& bz0) {
-    const int bx = item % nbx, rest = item / nbx, by = rest % nby, bz = rest / nby;
+    const int bx = item % nbx, rest = item / nbx, by = rest % nby;
+    const int bz = dp.active ? p2p_chunk_order(rest / nby, nbz) : rest / nby;
     bx0 = bx * 64;           // padded column of the staged tile origin (= interior column of lane col 0)
     by0 = by * BY<R>;        // padded row of the staged tile origin (= interior row of output row 0)
     bz0 = bz * ZC;           // first padded input plane (= first interior output plane) of the chunk
   };
   int pitem = gw, pj = 0, px = 0, py = 0, pz = 0;
   if (gw < nitems) geom(pitem, px, py, pz);
+  // device-initiated exchange: the z-chunk holding the first (last) R interior planes of the slab
+  // touches the lower (upper) neighbour (the host keeps it unique per column)
+  auto touches = [&](int bz0, bool& lo, bool& hi) {
+    lo = dp.active && dp.dst_lo != nullptr && bz0 < R;
+    hi = dp.active && dp.dst_hi != nullptr && int64_t(bz0) + ZC > N0 - R;
+  };
   auto issue_next = [&](int slot) {
     double* dst = reinterpret_cast<double*>(ring + slot * G::STAGE);
     const int z = pz + pj;
+    if (dp.active && pj == 0) {  // this column's halo planes come from a neighbour: wait for them
+      bool lo, hi;
+      touches(pz, lo, hi);
+      if (lane == 0 && (lo || hi)) {
+        const int u = pitem % (nbx * nby), ux = u % nbx, uy = u / nbx;
+        for (int yy = max(uy - 1, 0); yy <= min(uy + 1, nby - 1); ++yy) {
+          const int u0 = yy * nbx + max(ux - 1, 0), u1 = yy * nbx + min(ux + 1, nbx - 1);
+          if (lo) p2p_wait_units(dp.wait_lo, u0, u1, dp.wait_val, dp.err);
+          if (hi) p2p_wait_units(dp.wait_hi, u0, u1, dp.wait_val, dp.err);
+        }
+        fence_proxy_async_global();
+      }
+      __syncwarp();
+    }
     if constexpr (TMA) {
       if (lane == 0) {
         fence_proxy_async();
@@ -250,6 +274,7 @@ __global__ void __launch_bounds__(R3_WARPS * 32, RDG3_MINB) rdg3d_kernel(const d
   int cz = 0, zend = 0, rowmask = 0;
   double* obase = out;
   bool c0ok = false, c1ok = false, vec = false;
+  bool t_lo = false, t_hi = false;
   // consumer: stages in groups of n so that the ring slot of every plane offset is static
   for (int q0 = 0; q0 < nstages; q0 += n) {
     auto one = [&](auto Ic) {
@@ -280,6 +305,7 @@ __global__ void __launch_bounds__(R3_WARPS * 32, RDG3_MINB) rdg3d_kernel(const d
         for (int y = 0; y < BY<R>; ++y) rowmask |= (by0 + y < N1) ? (1 << y) : 0;
         obase = out + (int64_t(R) * P1 + by0 + R) * P2 + R + col;   // (interior z = 0, row by0, column col)
         vec = c0ok && c1ok && ((reinterpret_cast<uintptr_t>(obase) & 15) == 0) && ((P2 & 1) == 0);
+        touches(bz0, t_lo, t_hi);
       }
       const double* st = reinterpret_cast<const double*>(ring + slot * G::STAGE);
       double x[BY<R> + 2 * R][2 * R + 2];
@@ -297,15 +323,22 @@ __global__ void __launch_bounds__(R3_WARPS * 32, RDG3_MINB) rdg3d_kernel(const d
       constexpr int s = (I + 1) % n;
       const int zi = cz + cj - 2 * R;
       if (cj >= 2 * R && zi < zend) {
-        double* o = obase + int64_t(zi) * P1 * P2;
+        // the plane goes to this slab and, for the first / last R interior planes of a slab with a
+        // neighbour there, into that neighbour's halo as well (peer memory, csrc/dist_p2p.cu)
+        const bool rlo = t_lo && zi < R, rhi = t_hi && zi >= N0 - R;
+        const int nd = 1 + (rlo ? 1 : 0) + (rhi ? 1 : 0);
+        for (int d = 0; d < nd; ++d) {
+          double* o = obase + int64_t(zi) * P1 * P2;
+          if (d > 0) o = (rlo && d == 1) ? dp.dst_lo + ((o - out) + dp.off_lo) : dp.dst_hi + ((o - out) + dp.off_hi);
 #pragma unroll
-        for (int y = 0; y < BY<R>; ++y) {
-          if (rowmask & (1 << y)) {
-            if (vec) {
-              *reinterpret_cast<double2*>(o + int64_t(y) * P2) = make_double2(acc[s][y][0], acc[s][y][1]);
-            } else {
-              if (c0ok) o[int64_t(y) * P2] = acc[s][y][0];
-              if (c1ok) o[int64_t(y) * P2 + 1] = acc[s][y][1];
+          for (int y = 0; y < BY<R>; ++y) {
+            if (rowmask & (1 << y)) {
+              if (vec) {
+                *reinterpret_cast<double2*>(o + int64_t(y) * P2) = make_double2(acc[s][y][0], acc[s][y][1]);
+              } else {
+                if (c0ok) o[int64_t(y) * P2] = acc[s][y][0];
+                if (c1ok) o[int64_t(y) * P2 + 1] = acc[s][y][1];
+              }
             }
           }
         }
@@ -313,7 +346,12 @@ __global__ void __launch_bounds__(R3_WARPS * 32, RDG3_MINB) rdg3d_kernel(const d
 #pragma unroll
       for (int y = 0; y < BY<R>; ++y) { acc[s][y][0] = 0.0; acc[s][y][1] = 0.0; }
       if (++slot == R3_NS) { slot = 0; phase ^= 1; }
-      if (++cj == SI) { cj = 0; citem += TW; }
+      if (++cj == SI) {
+        if (t_lo) p2p_signal_warp(dp.sig_lo, citem % (nbx * nby), dp.sig_val);
+        if (t_hi) p2p_signal_warp(dp.sig_hi, citem % (nbx * nby), dp.sig_val);
+        cj = 0;
+        citem += TW;
+      }
     };
     [&]<int... Is>(std::integer_sequence<int, Is...>) {
       (one(std::integral_constant<int, Is>{}), ...);
@@ -383,7 +421,7 @@ bool make_params3(const Plan& p, R3Params& prm, bool direct = false) {
 
 template <int R, class SG, bool TMA>
 cudaError_t rdg3d_launch(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
-                         const R3Params& prm) {
+                         const R3Params& prm, const P2PArgs* d) {
   using G = G3<R>;
   static int max_grid = 0;
   if (max_grid == 0) {
@@ -402,18 +440,30 @@ cudaError_t rdg3d_launch(const Plan& p, const double* src, double* dst, cudaStre
     const int64_t zc2 = (p.N[0] + nch - 1) / nch;
     if (zc2 >= 8 && zc2 <= 2 * R3_ZC && cols * ((p.N[0] + zc2 - 1) / zc2) <= rounds * TWmax) zc = zc2;
   }
+  if (d && d->active && zc < p.N[0]) {
+    // device-initiated exchange: exactly one z-chunk per column may hold the last R interior
+    // planes (the last chunk must have >= R planes)
+    int64_t ok = 0;
+    for (int64_t c = zc; c <= zc + 64 && !ok; ++c) {
+      const int64_t rem = p.N[0] % c;
+      if (rem == 0 || rem >= R) ok = c;
+    }
+    zc = ok ? ok : p.N[0];
+  }
   const int ZC = (int)zc;
   const int SI = (int)(((ZC + 2 * R) + G::n - 1) / G::n * G::n);
   const int nbz = (int)((p.N[0] + ZC - 1) / ZC);
   const int64_t nitems = int64_t(nbx) * nby * nbz;
   const int grid = (int)std::min<int64_t>(max_grid, (nitems + R3_WARPS - 1) / R3_WARPS);
+  static const P2PArgs none{};
   rdg3d_kernel<R, SG, TMA><<<grid, R3_WARPS * 32, G::SMEM, s>>>(src, dst, p.N[0], p.N[1], p.N[2], nbx, nby, (int)nitems,
-                                                           ZC, SI, map, prm);
+                                                           ZC, SI, map, prm, d ? *d : none);
   return cudaGetLastError();
 }
 
 template <int R>
-cudaError_t rdg3d_r(const Plan& p, const double* src, double* dst, cudaStream_t s, bool direct = false) {
+cudaError_t rdg3d_r(const Plan& p, const double* src, double* dst, cudaStream_t s, bool direct = false,
+                    const P2PArgs* d = nullptr) {
   using G = G3<R>;
   R3Params prm;
   if (!make_params3(p, prm, direct)) return cudaErrorNotSupported;
@@ -424,14 +474,14 @@ cudaError_t rdg3d_r(const Plan& p, const double* src, double* dst, cudaStream_t 
   if (!tma) std::memset(&map, 0, sizeof(map));
   if constexpr (R == 1) {  // Box-3D27P-like and Heat-3D-like plane signatures
     if (prm.mode[0] == PM_PMA1 && prm.mode[1] == PM_PMA1 && prm.mirror[0])
-      return tma ? rdg3d_launch<R, Sig3<PM_PMA1, PM_PMA1, 1>, true>(p, src, dst, s, map, prm)
-                 : rdg3d_launch<R, Sig3<PM_PMA1, PM_PMA1, 1>, false>(p, src, dst, s, map, prm);
+      return tma ? rdg3d_launch<R, Sig3<PM_PMA1, PM_PMA1, 1>, true>(p, src, dst, s, map, prm, d)
+                 : rdg3d_launch<R, Sig3<PM_PMA1, PM_PMA1, 1>, false>(p, src, dst, s, map, prm, d);
     if (prm.mode[0] == PM_POINT && prm.mode[1] == PM_STAR && prm.mirror[0])
-      return tma ? rdg3d_launch<R, Sig3<PM_POINT, PM_STAR, 1>, true>(p, src, dst, s, map, prm)
-                 : rdg3d_launch<R, Sig3<PM_POINT, PM_STAR, 1>, false>(p, src, dst, s, map, prm);
+      return tma ? rdg3d_launch<R, Sig3<PM_POINT, PM_STAR, 1>, true>(p, src, dst, s, map, prm, d)
+                 : rdg3d_launch<R, Sig3<PM_POINT, PM_STAR, 1>, false>(p, src, dst, s, map, prm, d);
   }
-  return tma ? rdg3d_launch<R, Sig3<-1, -1, -1>, true>(p, src, dst, s, map, prm)
-             : rdg3d_launch<R, Sig3<-1, -1, -1>, false>(p, src, dst, s, map, prm);
+  return tma ? rdg3d_launch<R, Sig3<-1, -1, -1>, true>(p, src, dst, s, map, prm, d)
+             : rdg3d_launch<R, Sig3<-1, -1, -1>, false>(p, src, dst, s, map, prm, d);
 }
 
 }  // namespace
@@ -440,6 +490,24 @@ cudaError_t launch_direct3d_stream(const Plan& p, const double* src, double* dst
   switch (p.R) {
     case 1: return rdg3d_r<1>(p, src, dst, s, true);
     case 2: return rdg3d_r<2>(p, src, dst, s, true);
+  }
+  return cudaErrorNotSupported;
+}
+
+int rdg3d_p2p_units(const Plan& p, int* nux) {
+  R3Params prm;
+  const bool direct = p.engine == LORA_ENGINE_DIRECT;
+  if (p.ndim != 3 || p.R > 2 || (p.engine != LORA_ENGINE_RDG_CUDA && !direct) || !make_params3(p, prm, direct)) return 0;
+  const int bx = (int)((p.N[2] + 63) / 64), by = (int)((p.N[1] + (p.R == 1 ? BY<1> : BY<2>) - 1) / (p.R == 1 ? BY<1> : BY<2>));
+  if (nux) *nux = bx;
+  return bx * by;
+}
+
+cudaError_t launch_rdg3d_p2p(const Plan& p, const double* src, double* dst, cudaStream_t s, const P2PArgs& d) {
+  const bool direct = p.engine == LORA_ENGINE_DIRECT;
+  switch (p.R) {
+    case 1: return rdg3d_r<1>(p, src, dst, s, direct, &d);
+    case 2: return rdg3d_r<2>(p, src, dst, s, direct, &d);
   }
   return cudaErrorNotSupported;
 }

@@ -1,0 +1,239 @@
+"""Device-initiated halo exchange (lora_stencil_run_dist_p2p) on one GPU (-m gpu).
+
+Several slab ranks share the B200: in one process they are wired with p2p_connect_local and run on
+their own streams concurrently (the boundary tiles of one rank spin on the step counters the
+neighbour's kernel publishes, exactly as across NVLink); across two processes they are wired with
+CUDA IPC handles.  The gathered slabs must equal a single-GPU run of the global grid BITWISE (the
+same kernels compute every point from the same neighbourhood; pin P10) and the oracle to 1e-12."""
+import os
+
+import numpy as np
+import pytest
+import torch.multiprocessing as mp
+
+import oracle
+import synth
+from tests._gpu_helpers import rel_err
+
+pytestmark = pytest.mark.gpu
+
+
+def _weights(kind, d, h, seed):
+    if kind == "rsym":
+        return synth.rsym_weights(d, h, seed)
+    if kind == "star":
+        return synth.star_weights(d, h, seed)
+    if kind == "asym":
+        return synth.asym_weights(d, h, seed)
+    if kind == "heat3d":
+        return synth.preset("heat3d")
+    raise KeyError(kind)
+
+
+def _split(n0, counts):
+    starts = np.concatenate([[0], np.cumsum(counts)[:-1]]).astype(int)
+    assert sum(counts) == n0
+    return list(zip(starts.tolist(), counts))
+
+
+def _run_local(W, g, h, shape, T, engine, counts, zero_copy=False, repeat=1):
+    """P slab ranks in this process; returns the gathered global padded result (halo = input)."""
+    import torch
+    import paper_conf_sc_zhanglyczcy24_b200 as L
+    from paper_conf_sc_zhanglyczcy24_b200 import dist as D
+    slabs = _split(shape[0], counts)
+    P = len(slabs)
+    sts, eps, xs, ys, streams = [], [], [], [], []
+    for r, (s0, c) in enumerate(slabs):
+        st = L.Stencil(W, (c,) + tuple(shape[1:]), engine=engine, fuse_k=1)
+        sts.append(st)
+        eps.append(L.lora_stencil_p2p_create(st.plan, P, r))
+        xs.append(torch.from_numpy(np.ascontiguousarray(D.local_slice(g, s0, c, h))).cuda())
+        ys.append(torch.full_like(xs[-1], float("nan")))
+        streams.append(torch.cuda.Stream())
+    for r in range(P):
+        L.lora_stencil_p2p_connect_local(eps[r], eps[r - 1] if r > 0 else None, eps[r + 1] if r < P - 1 else None)
+    torch.cuda.synchronize()
+    for _ in range(repeat):
+        if zero_copy:
+            # fill every rank's buffer 0 through a tensor view of the library buffer BEFORE any run is
+            # enqueued: a device-wide synchronize between the ranks' enqueues would wait on a kernel
+            # that spins for a neighbour whose run is not enqueued yet
+            for r in range(P):
+                torch.as_tensor(_DevBuf(L.lora_stencil_p2p_buffer(eps[r], 0), xs[r].shape), device="cuda").copy_(xs[r])
+            torch.cuda.synchronize()
+        for r in range(P):
+            inp, outp = xs[r].data_ptr(), ys[r].data_ptr()
+            if zero_copy:
+                inp = L.lora_stencil_p2p_buffer(eps[r], 0)
+                outp = L.lora_stencil_p2p_buffer(eps[r], T % 2)
+            L.lora_stencil_run_dist_p2p(sts[r].plan, eps[r], inp, outp, T, streams[r].cuda_stream)
+        torch.cuda.synchronize()
+    for r in range(P):
+        L.lora_stencil_p2p_status(eps[r])
+    out = g.copy()
+    for r, (s0, c) in enumerate(slabs):
+        if zero_copy:
+            res = torch.as_tensor(_DevBuf(L.lora_stencil_p2p_buffer(eps[r], T % 2), xs[r].shape), device="cuda")
+            res = res.cpu().numpy()
+        else:
+            res = ys[r].cpu().numpy()
+        out[h + s0:h + s0 + c] = res[h:h + c]
+    for r in range(P):
+        L.lora_stencil_p2p_destroy(eps[r])
+        sts[r].close()
+    return out
+
+
+class _DevBuf:
+    """__cuda_array_interface__ view of a library-owned device buffer (float64, C order)."""
+
+    def __init__(self, ptr, shape):
+        self.__cuda_array_interface__ = {"shape": tuple(shape), "typestr": "<f8", "data": (int(ptr), False),
+                                         "version": 3, "strides": None}
+
+
+def _global(W, g, T, engine):
+    import torch
+    import paper_conf_sc_zhanglyczcy24_b200 as L
+    h = (W.shape[0] - 1) // 2
+    shape = tuple(s - 2 * h for s in g.shape)
+    st = L.Stencil(W, shape, engine=engine, fuse_k=1)
+    x = torch.from_numpy(g).cuda()
+    y = torch.empty_like(x)
+    st.run(x, y, T)
+    torch.cuda.synchronize()
+    st.close()
+    return y.cpu().numpy()
+
+
+CASES = [
+    # d, h, kind, engine, global interior shape, slab row counts
+    (2, 3, "rsym", "rdg_cuda", (300, 200), [150, 150]),
+    (2, 3, "rsym", "rdg_cuda", (301, 130), [100, 3, 198]),        # a slab of exactly R rows
+    (2, 1, "rsym", "rdg_cuda", (517, 300), [129, 130, 128, 130]),
+    (2, 2, "star", "rdg_cuda", (260, 190), [130, 130]),
+    (2, 2, "asym", "rdg_cuda", (200, 77), [67, 133]),
+    (2, 3, "rsym", "direct", (257, 99), [128, 129]),
+    (3, 1, "rsym", "rdg_cuda", (96, 20, 66), [48, 48]),
+    (3, 1, "heat3d", "rdg_cuda", (130, 12, 40), [65, 1, 64]),
+    (3, 2, "rsym", "rdg_cuda", (70, 9, 33), [35, 35]),
+    (3, 1, "asym", "direct", (64, 10, 70), [30, 34]),
+]
+
+
+@pytest.mark.parametrize("case", CASES)
+def test_p2p_local_ranks_bitwise(case):
+    d, h, kind, engine, shape, counts = case
+    W = _weights(kind, d, h, 21 + h)
+    g = synth.grid(tuple(n + 2 * h for n in shape), 31)
+    for T in (1, 2, 5):
+        ref = _global(W, g, T, engine)
+        out = _run_local(W, g, h, shape, T, engine, counts)
+        assert np.array_equal(out, ref), (T, float(np.nanmax(np.abs(out - ref))))
+    if shape[0] * int(np.prod(shape[1:])) <= 40000:
+        assert rel_err(out, oracle.run(W, g, 5)) <= 1e-12
+
+
+def test_p2p_repeated_runs_and_zero_copy():
+    """Epochs: the same endpoints run three times (monotonic step counters, no reset); zero-copy
+    mode reads buffer 0 and leaves the result in buffer T % 2."""
+    W = synth.rsym_weights(2, 3, 8)
+    shape, h = (256, 150), 3
+    g = synth.grid(tuple(n + 2 * h for n in shape), 9)
+    for T in (3, 4):
+        ref = _global(W, g, T, "rdg_cuda")
+        assert np.array_equal(_run_local(W, g, h, shape, T, "rdg_cuda", [128, 128], repeat=3), ref)
+        assert np.array_equal(_run_local(W, g, h, shape, T, "rdg_cuda", [100, 156], zero_copy=True, repeat=2), ref)
+
+
+def test_p2p_large_slabs_many_items():
+    """Box-2D49P slabs large enough for a full persistent grid (many boundary items per step)."""
+    W, c = synth.config("box2d49p-10240")
+    shape, h = (2048, 4096), 3
+    g = synth.grid(tuple(n + 2 * h for n in shape), 20240103)
+    T = 3
+    ref = _global(W, g, T, "rdg_cuda")
+    out = _run_local(W, g, h, shape, T, "rdg_cuda", [512, 512, 512, 512])
+    assert np.array_equal(out, ref)
+
+
+def test_p2p_unsupported_and_errors():
+    import paper_conf_sc_zhanglyczcy24_b200 as L
+    W = synth.rsym_weights(2, 1, 2)
+    st = L.Stencil(W, (64, 64), engine="tc")
+    with pytest.raises(L.LoraError) as e:
+        L.lora_stencil_p2p_create(st.plan, 2, 0)
+    assert e.value.code == L.LORA_ERR_UNSUPPORTED
+    st.close()
+    st = L.Stencil(W, (64, 64), engine="rdg_cuda")
+    ep = L.lora_stencil_p2p_create(st.plan, 2, 0)
+    with pytest.raises(L.LoraError):   # not connected to its upper neighbour
+        L.lora_stencil_run_dist_p2p(st.plan, ep, L.lora_stencil_p2p_buffer(ep, 0), L.lora_stencil_p2p_buffer(ep, 1), 1)
+    with pytest.raises(L.LoraError):   # rank 0 has no lower neighbour: a handle there is an error
+        L.lora_stencil_p2p_connect(ep, b"\0" * 128, b"\0" * 128)
+    other = L.Stencil(W, (64, 66), engine="rdg_cuda")
+    ep2 = L.lora_stencil_p2p_create(other.plan, 2, 1)
+    with pytest.raises(L.LoraError):   # trailing extents differ
+        L.lora_stencil_p2p_connect_local(ep, None, ep2)
+    L.lora_stencil_p2p_destroy(ep)
+    L.lora_stencil_p2p_destroy(ep2)
+    st.close()
+    other.close()
+
+
+def _ipc_rank(rank, world, q_out, q_h, q_go):
+    try:
+        import sys
+        sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+        import torch
+        import paper_conf_sc_zhanglyczcy24_b200 as L
+        from paper_conf_sc_zhanglyczcy24_b200 import dist as D
+        torch.cuda.set_device(0)
+        W = synth.rsym_weights(2, 3, 5)
+        shape, h, T = (200, 130), 3, 3
+        g = synth.grid(tuple(n + 2 * h for n in shape), 6)
+        start, cnt = D.slab_bounds(shape[0], world, rank)
+        st = L.Stencil(W, (cnt, shape[1]), engine="rdg_cuda", fuse_k=1)
+        ep = L.lora_stencil_p2p_create(st.plan, world, rank)
+        q_h.put((rank, L.lora_stencil_p2p_get_handle(ep)))
+        hs = dict(q_go[rank].get(timeout=120))
+        L.lora_stencil_p2p_connect(ep, hs.get(rank - 1), hs.get(rank + 1))
+        x = torch.from_numpy(np.ascontiguousarray(D.local_slice(g, start, cnt, h))).cuda()
+        y = torch.empty_like(x)
+        L.lora_stencil_run_dist_p2p(st.plan, ep, x.data_ptr(), y.data_ptr(), T, torch.cuda.current_stream().cuda_stream)
+        torch.cuda.synchronize()
+        L.lora_stencil_p2p_status(ep)
+        q_out.put((rank, start, y[h:h + cnt].cpu().numpy()))
+        q_go[rank].get(timeout=120)      # keep the mapping alive until every rank is done
+        L.lora_stencil_p2p_destroy(ep)
+    except Exception:
+        import traceback
+        q_out.put((rank, -1, traceback.format_exc()))
+
+
+def test_p2p_two_processes_cuda_ipc():
+    """Two processes on the one GPU, wired by CUDA IPC handles (the multi-GPU wiring path)."""
+    import torch
+    world = 2
+    ctx = mp.get_context("spawn")
+    q_out, q_h = ctx.Queue(), ctx.Queue()
+    q_go = [ctx.Queue() for _ in range(world)]
+    procs = [ctx.Process(target=_ipc_rank, args=(r, world, q_out, q_h, q_go)) for r in range(world)]
+    for p in procs:
+        p.start()
+    hs = dict(q_h.get(timeout=180) for _ in range(world))
+    for r in range(world):
+        q_go[r].put(list(hs.items()))
+    res = [q_out.get(timeout=300) for _ in range(world)]
+    for r in range(world):
+        q_go[r].put(None)
+    for p in procs:
+        p.join(timeout=60)
+    for r, s, a in res:
+        assert s >= 0, a
+    W = synth.rsym_weights(2, 3, 5)
+    g = synth.grid((206, 136), 6)
+    ref = _global(W, g, 3, "rdg_cuda")
+    for r, s, a in res:
+        assert np.array_equal(a, ref[3 + s:3 + s + a.shape[0]])
