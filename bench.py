@@ -8,7 +8,9 @@ target) unless --workload says otherwise.  value = T * prod(N_i) * n_ranks / t (
     python bench.py --impl reference ...   # the CPU oracle (oracle/) on host cores, bounded sample
 
 N > 1 runs under torch.distributed.run, one rank per GPU: weak scaling, every rank owns a slab
-of the same local shape and exchanges halos through lora_stencil_run_dist (NCCL).
+of the same local shape.  Halos move by the device-initiated exchange (lora_stencil_run_dist_p2p:
+the stencil kernel stores its edge rows into the neighbour's halo over NVLink and signals it;
+--dist nccl selects the host-issued NCCL send/recv path lora_stencil_run_dist instead).
 """
 from __future__ import annotations
 
@@ -44,6 +46,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-engines", action="store_true", help="skip the per-engine comparison on the workload")
+    ap.add_argument("--dist", default="p2p", choices=["p2p", "nccl"],
+                    help="halo exchange for N > 1: device-initiated (kernel stores into the neighbour's halo) or NCCL")
     ap.add_argument("--force-dist", action="store_true",
                     help="use lora_stencil_run_dist even on one rank (exercises the slab path; LORA_DIST_SPLIT=1 "
                          "additionally forces the overlapped edge/interior split)")
@@ -207,7 +211,33 @@ def main():
     st = L.Stencil(W, shape, engine=args.engine, fuse_k=args.fuse)
     info = st.info()
     comm = None
-    if world > 1 or args.force_dist:
+    ep = None          # device-initiated exchange endpoint (lora_stencil_p2p_*)
+    exchange = None
+    if (world > 1 or args.force_dist) and args.dist == "p2p":
+        err = ""
+        try:
+            ep = L.lora_stencil_p2p_create(st.plan, world, rank)
+            hs = [L.lora_stencil_p2p_get_handle(ep)]
+            if world > 1:
+                hs = [None] * world
+                dist.all_gather_object(hs, L.lora_stencil_p2p_get_handle(ep))
+                L.lora_stencil_p2p_connect(ep, hs[rank - 1] if rank > 0 else None,
+                                           hs[rank + 1] if rank < world - 1 else None)
+        except L.LoraError as e:
+            err = str(e)
+        ok = torch.tensor([0 if err else 1], device=dev)
+        if world > 1:
+            dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+        if int(ok.item()) == 1:
+            exchange = "p2p (device-initiated: kernel stores edge rows into the neighbour's halo, per-tile step counters)"
+        else:   # every rank must use the same transport
+            print(f"[bench] p2p exchange unavailable on some rank ({err or 'peer'}); using NCCL", file=sys.stderr)
+            if ep is not None:
+                L.lora_stencil_p2p_destroy(ep)
+            ep = None
+            exchange = "nccl (p2p setup failed: " + (err or "on another rank") + ")"
+    if (world > 1 or args.force_dist) and ep is None:
+        exchange = exchange or "nccl (host-issued send/recv, boundary strips first, overlapped with the interior)"
         if world > 1:
             uid = L.lora_stencil_comm_get_id() if rank == 0 else None
             obj = [uid]
@@ -226,8 +256,22 @@ def main():
     stream = torch.cuda.current_stream(dev)
     sptr = stream.cuda_stream
 
+    if ep is not None:
+        # zero-copy use of the exchange buffers: the slab lives in buffer 0, the result lands in
+        # buffer T % 2 (T even: buffer 0 again, so each timed step continues the evolution)
+        b0 = L.lora_stencil_p2p_buffer(ep, 0)
+
+        class _Dev:
+            __cuda_array_interface__ = {"shape": tuple(x.shape), "typestr": "<f8", "data": (int(b0), False),
+                                        "version": 3, "strides": None}
+        torch.as_tensor(_Dev(), device=dev).copy_(x)
+        torch.cuda.synchronize(dev)
+        bT = L.lora_stencil_p2p_buffer(ep, T % 2)
+
     def step():
-        if comm is None:
+        if ep is not None:
+            L.lora_stencil_run_dist_p2p(st.plan, ep, b0, bT, T, sptr)
+        elif comm is None:
             L.lora_stencil_run(st.plan, x.data_ptr(), y.data_ptr(), T, sptr)
         else:
             L.lora_stencil_run_dist(st.plan, comm, x.data_ptr(), y.data_ptr(), T, sptr)
@@ -255,8 +299,10 @@ def main():
         t = float(tt.item())
     pts_per_step = float(np.prod(shape)) * T * world
     value = pts_per_step * args.steps / t / 1e9
-    fuse = info["fuse_k"]
+    fuse = 1 if (comm is not None or ep is not None) else info["fuse_k"]   # the dist paths step unfused
     launches_per_step = -(-T // fuse) + 2      # stencil launches + 2 halo-copy launches
+    if ep is not None:                         # T stencil launches + 1 halo copy + publish/wait per neighbour
+        launches_per_step = T + 1 + 2 * ((1 if rank > 0 else 0) + (1 if rank < world - 1 else 0))
 
     # roofline for the dominant kernel (the stencil kernel): algorithmic bytes per launch / avg launch time
     peak, peak_src = load_peaks()
@@ -278,7 +324,7 @@ def main():
     # problem's PCIe copies overlap the other's stencil steps.  "serial" = one synchronous
     # lora_stencil_run_host call per step (copies not overlapped).
     e2e = None
-    if not args.no_e2e and comm is None:
+    if not args.no_e2e and comm is None and ep is None:
         nbytes = host_in.numel() * 8
         L.lora_stencil_run_host(st.plan, host_in.numpy(), host_out.numpy(), T, sptr)
         torch.cuda.synchronize(dev)
@@ -377,7 +423,8 @@ def main():
                 "config": {"workload": args.workload, "grid_per_rank": list(shape), "T": T, "radius": h,
                            "ndim": cfg["ndim"], "global_grid": [shape[0] * world] + list(shape[1:]),
                            "engine": info["engine_name"], "fuse_k": fuse, "n_terms": info["n_terms"],
-                           "parallelism": f"slab{world}" if comm is not None else "single",
+                           "parallelism": f"slab{world}" if (comm is not None or ep is not None) else "single",
+                           "exchange": exchange,
                            "l2": "inputs (%.2f GB per buffer) larger than the 126 MB L2" % (8 * np.prod(padded) / 1e9)},
                 "clocks": clk.summary(), "gpu_launches": launches_per_step * args.steps,
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
@@ -391,6 +438,9 @@ def main():
         print(json.dumps(line), flush=True)
     if comm is not None:
         L.lora_stencil_comm_destroy(comm)
+    if ep is not None:
+        L.lora_stencil_p2p_status(ep)
+        L.lora_stencil_p2p_destroy(ep)
     st.close()
     if world > 1:
         dist.destroy_process_group()
