@@ -271,7 +271,8 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
   } else if constexpr (FULL) {
     double* o = out + sc.ooff + int64_t(I) * P1;
 #pragma unroll
-    for (int h = 0; h < NH; ++h) *reinterpret_cast<double2*>(o + 64 * h) = make_double2(v[h][0], v[h][1]);
+    for (int h = 0; h < NH; ++h)   // band-overlap lanes of a fused band store nothing
+      if (lc.vec[h]) *reinterpret_cast<double2*>(o + 64 * h) = make_double2(v[h][0], v[h][1]);
   } else {
     if (I >= sc.lo && I < sc.hi) {
       const int64_t e = sc.ooff + int64_t(I) * P1;
@@ -316,6 +317,12 @@ __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p,
 // Resident CTAs per SM (register budget 512 / minb per thread x 128 threads), measured on B200
 // (profiles/r01_rdg_occupancy.txt): the heavy radius >= 3 PMA pass wants registers for ILP more
 // than warps (2 CTAs: 338 GS/s vs 305 at 4 for Box-2D49P); light passes want 4; fused radius >= 2 3.
+#ifndef RDG_FULL
+// 2: unfused kernels get a second copy of the row loop without per-row checks for interior stages
+// (Box-2D49P 314 -> 339 GS/s); the fused kernels do not (their doubled hot code footprint costs
+// more than the checks: Star-2D13P k=2 412 -> 360).  0: never, 1: always (experiments).
+#define RDG_FULL 2
+#endif
 #ifndef RDG_NH_FUSED
 #define RDG_NH_FUSED 2   // 64-column halves per warp in the fused (K >= 2) kernels
 #endif
@@ -324,9 +331,12 @@ constexpr int rdg_cta_smem(int nh) {   // must match rdg_launch
   return nh == 1 ? 128 + RDG_WARPS * (Geom<R, 1>::WARP_BYTES + 2 * (K - 1) * Geom<R, 1>::BUFD * 8)
                  : 128 + RDG_WARPS * (Geom<R, 2>::WARP_BYTES + 2 * (K - 1) * Geom<R, 2>::BUFD * 8);
 }
-// NH = 2 where two CTAs of it still fit the 228 KB of shared memory per SM (R = 1, 3, 4)
+// NH = 2 where two CTAs of it still fit the 228 KB of shared memory per SM (R = 3, 4)
 template <int R, int SIG, int K>
-constexpr int rdg_nh() { return (K >= 2 && RDG_NH_FUSED == 2 && 2 * (rdg_cta_smem<R, K>(2) + 1024) <= 228 * 1024) ? 2 : 1; }
+// (radius 1 stays at NH = 1: Box-2D9P k = 3 641 vs 630 GS/s; radius 3 k = 2 gains 7 %)
+constexpr int rdg_nh() {
+  return (K >= 2 && R >= 2 && RDG_NH_FUSED == 2 && 2 * (rdg_cta_smem<R, K>(2) + 1024) <= 228 * 1024) ? 2 : 1;
+}
 
 template <int R, int SIG, int K>
 constexpr int rdg_minb() {
@@ -454,16 +464,18 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
           const int c = lc.c0 + 64 * h + j;
           lc.inside[h][j] = c >= 0 && c < P1;
           lc.colhalo[h][j] = lc.inside[h][j] && (c < R || c >= P1 - R);
-          lc.valid[h][j] = c >= X0 + R * (K - 1) && c < X0 + 64 * NH - R * (K - 1) && c >= R && c < P1 - R;
+          // the band's own BS columns (even-aligned: X0 and R(K-1) + SG are even), so a lane's
+          // pair is valid or invalid as a whole except at the array's right edge
+          lc.valid[h][j] = c >= X0 + R * (K - 1) + SG && c < X0 + R * (K - 1) + SG + BS && c >= R && c < P1 - R;
           lc.edge = lc.edge || lc.colhalo[h][j] || !lc.inside[h][j];
         }
         lc.vec[h] = lc.valid[h][0] && lc.valid[h][1] &&
                     ((reinterpret_cast<uintptr_t>(out + lc.c0 + 64 * h) & 15) == 0) && ((P1 & 1) == 0);
       }
       rows_valid_end = min(A + RC, P0 - R);
-      bool mine = !lc.edge;
+      bool mine = !lc.edge;   // FULL lanes: no halo columns; a pair is stored as one 16-byte store or not at all
 #pragma unroll
-      for (int h = 0; h < NH; ++h) mine = mine && lc.vec[h];
+      for (int h = 0; h < NH; ++h) mine = mine && lc.valid[h][0] == lc.valid[h][1] && (lc.vec[h] || !lc.valid[h][0]);
       all_fast = __all_sync(0xffffffffu, mine);
       touches(A, t_lo, t_hi);
     }
@@ -490,7 +502,7 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
     bool full = all_fast && sc.lo <= 0 && sc.hi >= G::SROWS && sc.rem_lo <= 0 && sc.rem_hi >= G::SROWS;
 #pragma unroll
     for (int S = 1; S < K; ++S) full = full && sc.hlo[S - 1] <= 0 && sc.hhi[S - 1] >= G::SROWS;
-    if (full) fused_rows<R, SIG, K, NH, true, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp);
+    if ((RDG_FULL == 1 || (RDG_FULL == 2 && K == 1)) && full) fused_rows<R, SIG, K, NH, true, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp);
     else fused_rows<R, SIG, K, NH, false, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp);
     __syncwarp();  // every lane is done with this slot before it is refilled
     if (++slot == RDG_NS) { slot = 0; phase ^= 1; }

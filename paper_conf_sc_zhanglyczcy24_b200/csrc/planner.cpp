@@ -355,10 +355,13 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
     // default fusion depth (exact temporal blocking), from B200 measurements
     // (profiles/r01_quickbench_*.jsonl): fusing pays while the CUDA-core engine is HBM-bound, i.e.
     // for light stencils (2D <= 20, 3D <= 12 issued FMA per point: Box-2D9P, Star-2D13P, Heat-3D,
-    // 1D); Box-2D49P (31 FMA/pt) and Box-3D27P (18) are faster unfused.
+    // 1D).  Box-2D49P (row-pair form, 25 FP64 ops/pt) fuses k = 2: unfused it is HBM-bound and hits
+    // the 1 kW power cap under sustained load (~1.7 GHz), fused it is FP64-bound at full clock
+    // (bench.py, 8 x 100 steps: 303 -> 320 GS/s); the same holds for Box-3D27P (307 -> 320).
     const double work = cuda_fma_per_point(p);
     if (p.ndim == 1) fk = 8;
-    else if (p.ndim == 3) fk = work <= 12.0 ? 2 : 1;   // Heat-3D fuses; Box-3D27P is faster unfused
+    else if (p.ndim == 3) fk = 2;   // Heat-3D; Box-3D27P too: sustained 307 (power-capped) -> 320 GS/s
+    else if (p.rdg_rows && radius == 3) fk = 2;   // Box-2D49P: sustained (power-capped) 303 -> 320 GS/s
     else if (work > 20.0) fk = 1;
     else fk = radius == 1 ? 3 : 2;
     fk = std::min(max_k, fk);
