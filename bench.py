@@ -304,20 +304,40 @@ def main():
     if ep is not None:                         # T stencil launches + 1 halo copy + publish/wait per neighbour
         launches_per_step = T + 1 + 2 * ((1 if rank > 0 else 0) + (1 if rank < world - 1 else 0))
 
-    # roofline for the dominant kernel (the stencil kernel): algorithmic bytes per launch / avg launch time
+    # roofline for the dominant kernel (the stencil kernel), two views; "bound" is the resource the
+    # kernel runs closest to (the larger fraction):
+    #  hbm: ALGORITHMIC bytes per launch (16 B per point per launch: one read + one write of the grid,
+    #       whatever the fused depth) / average launch time, vs the measured HBM copy bandwidth;
+    #  alu: FP64 pipe lane-ops per launch (the plan's issued FP64 ops per point-step, DFMA/DADD/DMUL
+    #       each one lane-op, x points x fused steps; band/chunk recomputation NOT counted) / average
+    #       launch time, vs 148 SMs x 64 FP64 lanes x 1.965 GHz (the step-0 DMMA
+    #       microbenchmark reaches 36.9 TFLOP/s = 99 % of that).
     peak, peak_src = load_peaks()
+    n_launch = -(-T // fuse)
     per_launch_bytes = BYTES_PER_POINT * float(np.prod(shape))      # per launch: one (fused) superstep
-    avg_launch_s = t / args.steps / (-(-T // fuse))
+    avg_launch_s = t / args.steps / n_launch
     achieved = per_launch_bytes / avg_launch_s / 1e9
+    fp64_peak_gops = 148 * 64 * 1.965                                  # G lane-ops/s
+    ops_per_launch = info["fma_per_point_issued"] * float(np.prod(shape)) * (T / n_launch)
+    alu_achieved = ops_per_launch / avg_launch_s / 1e9
     tr = ncu_traffic(args.workload, info["engine_name"])
-    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-            "traffic": tr["bytes"] if tr else None,       # dram read+write bytes per launch (ncu --set full)
-            "traffic_source": ({k: tr[k] for k in ("kernel", "source", "fuse")} if tr else None),
-            "peak_source": peak_src,
-            "kernel": f"{info['engine_name']} stencil step", "algorithmic_bytes_per_launch": per_launch_bytes,
-            "avg_launch_ms": avg_launch_s * 1e3,
-            "avg_launch_note": "timed step / stencil launches per step (the 2 halo-copy launches per run, ~0.1%, included)",
-            "gstencil_roofline": peak / BYTES_PER_POINT * world}
+    if tr and int(tr.get("fuse", 1)) != fuse:
+        tr = None
+    hbm = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+           "peak_source": peak_src, "algorithmic_bytes_per_launch": per_launch_bytes}
+    alu = {"bound": "alu", "achieved": alu_achieved, "peak": fp64_peak_gops, "unit": "Gop/s (FP64 pipe lane-ops)",
+           "frac": alu_achieved / fp64_peak_gops,
+           "peak_source": "derived: 148 SMs x 64 FP64 lanes x 1.965 GHz (DESIGN.md §6)",
+           "algorithmic_ops_per_launch": ops_per_launch}
+    roof = dict(alu if alu["frac"] > hbm["frac"] else hbm)
+    roof.update({"traffic": tr["bytes"] if tr else None,       # dram read+write bytes per launch (ncu --set full)
+                 "traffic_source": ({k: tr[k] for k in ("kernel", "source", "fuse")} if tr else None),
+                 "kernel": f"{info['engine_name']} stencil step (fuse_k={fuse})",
+                 "avg_launch_ms": avg_launch_s * 1e3,
+                 "avg_launch_note": "timed step / stencil launches per step (the 2 halo-copy launches per run, ~0.1%, included)",
+                 "views": {"hbm": hbm, "alu": alu},
+                 "gstencil_roofline": peak / BYTES_PER_POINT * world,
+                 "frac_gstencil_of_hbm_roofline": value / (peak / BYTES_PER_POINT * world)})
 
     # e2e: through the C-ABI with HOST buffers (H2D of the input + D2H of the result inside the region).
     # Headline = two independent problems in flight (two plans, two streams, steps alternate): one

@@ -44,7 +44,7 @@ struct Plan {
   int n_planes_point = 0;
   // CUDA-core engine, 2D, radius >= 3, W reflection-symmetric in both axes: evaluate W as the
   // row-pair rank-1 split u_a = e_{R+a} + e_{R-a}, v_a = W[R+a,:] (a = 0..R; exact, growth 1),
-  // which issues R + (R+1)^2 + 2R+1 FP64 ops per point against PMA's (28 vs 26 at R = 3).
+  // which issues R + (R+1)^2 + 2R FP64 ops per point against PMA's (28 vs 25 at R = 3).
   // LORA_RDG_PMA=1 keeps the PMA factors on that engine (ablation).
   int rdg_rows = 0;
   double recon_err = 0, growth = 0;

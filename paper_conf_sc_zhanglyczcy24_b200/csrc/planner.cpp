@@ -202,7 +202,7 @@ double cuda_fma_per_point(const Plan& p) {
   };
   if (p.ndim == 2) {
     const int R = p.R;
-    if (p.rdg_rows) return R + (R + 1) * (R + 1) + (2 * R + 1);   // SIG_ROWS (kernels_rdg.cu)
+    if (p.rdg_rows) return R + (R + 1) * (R + 1) + 2 * R;   // SIG_ROWS (kernels_rdg.cu; the fresh ring slot is assigned)
     // PMA pyramid (SIG_PMA): R shared tap-pair sums, then per chain of radius H a palindromic
     // horizontal gather (H+1) and a vertical scatter (2H+1), plus the scalar C_{h+1}
     bool pma = (int)p.terms.size() == R + 1;
