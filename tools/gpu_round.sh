@@ -12,7 +12,7 @@ timeout 900 python bench.py --per-stencil > gpurun_out/${TAG}_bench.json 2> gpur
 cat gpurun_out/${TAG}_bench.json
 timeout 600 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/${TAG}_bench_ref.json 2>&1; echo "ref rc=$?"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv \
-   python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu > /dev/null 2>&1; echo "ncu launches rc=$?"
+   python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu --no-engines > /dev/null 2>&1; echo "ncu launches rc=$?"
 for spec in "$@"; do
   IFS=: read -r KRE WL ENG FK <<< "$spec"
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:${KRE} -s 3 -c 1 \
