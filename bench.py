@@ -256,9 +256,11 @@ def main():
     stream = torch.cuda.current_stream(dev)
     sptr = stream.cuda_stream
 
-    if ep is not None:
-        # zero-copy use of the exchange buffers: the slab lives in buffer 0, the result lands in
-        # buffer T % 2 (T even: buffer 0 again, so each timed step continues the evolution)
+    zero_copy = ep is not None and (info["fuse_k"] == 1 or cfg["ndim"] == 3)
+    if zero_copy:
+        # zero-copy use of the exchange buffers (unfused launches keep the caller's layout): the slab
+        # lives in buffer 0, the result lands in buffer T % 2 (T even: buffer 0 again, so each timed
+        # step continues the evolution).  Fused launches use deep halos: copy-in / copy-out instead.
         b0 = L.lora_stencil_p2p_buffer(ep, 0)
 
         class _Dev:
@@ -270,7 +272,10 @@ def main():
 
     def step():
         if ep is not None:
-            L.lora_stencil_run_dist_p2p(st.plan, ep, b0, bT, T, sptr)
+            if zero_copy:
+                L.lora_stencil_run_dist_p2p(st.plan, ep, b0, bT, T, sptr)
+            else:
+                L.lora_stencil_run_dist_p2p(st.plan, ep, x.data_ptr(), y.data_ptr(), T, sptr)
         elif comm is None:
             L.lora_stencil_run(st.plan, x.data_ptr(), y.data_ptr(), T, sptr)
         else:
@@ -299,10 +304,12 @@ def main():
         t = float(tt.item())
     pts_per_step = float(np.prod(shape)) * T * world
     value = pts_per_step * args.steps / t / 1e9
-    fuse = 1 if (comm is not None or ep is not None) else info["fuse_k"]   # the dist paths step unfused
+    # the NCCL path steps unfused; the P2P path runs the plan's fused depth in 2D (deep halos)
+    fuse = 1 if (comm is not None or (ep is not None and cfg["ndim"] == 3)) else info["fuse_k"]
     launches_per_step = -(-T // fuse) + 2      # stencil launches + 2 halo-copy launches
-    if ep is not None:                         # T stencil launches + 1 halo copy + publish/wait per neighbour
-        launches_per_step = T + 1 + 2 * ((1 if rank > 0 else 0) + (1 if rank < world - 1 else 0))
+    if ep is not None:   # ceil(T/k) stencil launches + 1 halo copy + per neighbour: 2 publish, 2 wait, 1 push
+        nb = (1 if rank > 0 else 0) + (1 if rank < world - 1 else 0)
+        launches_per_step = -(-T // fuse) + 1 + 5 * nb
 
     # roofline for the dominant kernel (the stencil kernel), two views; "bound" is the resource the
     # kernel runs closest to (the larger fraction):

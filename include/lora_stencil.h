@@ -174,15 +174,18 @@ int lora_stencil_dist_exchange_plan(const lora_plan* p, int rank, int nranks, in
  * collective call per step at all.  Results are bitwise equal to lora_stencil_run_dist and to a
  * single-GPU run of the global grid (same kernels, same per-point arithmetic).
  *
- * Engines: the CUDA-core engine (2D, 3D radius <= 2) and the direct comparison kernel, unfused
- * (one step per launch); other plans return LORA_ERR_UNSUPPORTED.  Every rank's plan has the
- * same trailing extents and radius (the local n0 may differ).
+ * Engines: the CUDA-core engine (2D, 3D radius <= 2) and the direct comparison kernel; other
+ * plans return LORA_ERR_UNSUPPORTED.  2D CUDA-core plans keep their fusion depth k (plan fuse_k):
+ * each launch advances k steps and internal slab edges carry k*r-deep halos (every slab needs
+ * >= k*r rows, else LORA_ERR_INVALID_ARG); 3D and direct plans step unfused.  Every rank's plan has
+ * the same trailing extents, radius and fuse_k (the local n0 may differ).
  *
- * Exchange buffers: the communicator owns two padded slabs of the plan's local shape (the
- * ping-pong pair the neighbours write into) plus the flag words, allocated with cudaMalloc on
- * the current device (IPC-exportable).  lora_stencil_p2p_buffer exposes them: a caller that
- * fills buffer 0 directly and passes it as `in_local` (and buffer T%2 as `out_local`) avoids the
- * copy-in / copy-out.
+ * Exchange buffers: the communicator owns two padded slabs (the ping-pong pair the neighbours
+ * write into; rows = lower halo depth + n0 + upper halo depth) plus the flag words, allocated with
+ * cudaMalloc on the current device (IPC-exportable).  lora_stencil_p2p_buffer exposes them: for an
+ * unfused endpoint (k = 1) they have the caller's layout, and a caller that fills buffer 0 directly
+ * and passes it as `in_local` (and buffer L%2 as `out_local`, L = the number of launches = T for
+ * k = 1) avoids the copy-in / copy-out.
  *
  * A spin-wait that sees no progress for 20 s (a neighbour that never runs) gives up instead of
  * hanging the GPU and sets a device error word: lora_stencil_p2p_status reports it. */

@@ -30,6 +30,16 @@ struct P2PArgs {
   unsigned long long wait_val = 0; // boundary items wait until flags >= wait_val
   unsigned long long sig_val = 0;  // and publish sig_val when their stores are done
   int* err = nullptr;              // device error word (spin timeout => 1)
+  // Row bookkeeping in the launch's padded rows (2D; 3D uses planes with H = R).  A fused launch of k
+  // steps runs on a slab whose internal edges carry H = k_max R deep halos, presented to the kernel
+  // as a taller "view" (the deep halo rows beyond R count as interior rows of the view): only the
+  // rows [store_lo, store_hi) are this rank's and stored; the first H of them ([store_lo, lo_end))
+  // go to the lower neighbour, the last H ([hi_begin, store_hi)) to the upper one.
+  int H = 0, lo_end = 0, hi_begin = 0, store_lo = 0, store_hi = 0;
+  int prepare_only = 0;            // 1: only load the kernel (lazy module loading must not happen
+                                   // while a spin-waiting kernel of this process runs) and return
+  int wait_units = 0;              // > 0: wait on units [0, wait_units) (the neighbour's previous
+                                   // launch had another band geometry: a remainder launch)
 };
 
 // Copies the Dirichlet halo ring of `in` into `dst` (both padded arrays of the plan's shape).
@@ -52,8 +62,9 @@ cudaError_t launch_tc2d(const Plan& p, const double* src, double* dst, cudaStrea
 cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s, int k);
 // One unfused step of the 2D CUDA-core engine (any signature incl. the direct comparison kernel) or
 // of the 3D one, with the device-initiated halo exchange of `d` (d.active = 1).
-cudaError_t launch_step_p2p(const Plan& p, const double* src, double* dst, cudaStream_t s, const P2PArgs& d);
-int p2p_units(const Plan& p, int* nux);   // flag units per side, 0 if the plan's engine has no P2P path
+cudaError_t launch_step_p2p(const Plan& p, const double* src, double* dst, cudaStream_t s, const P2PArgs& d, int k);
+int p2p_units(const Plan& p, int* nux);   // flag units per side (unfused), 0 if the plan's engine has no P2P path
+int p2p_units_k(const Plan& p, int k);     // 2D: band count of the k-fused stream kernel
 int rdg2d_max_fuse(const Plan& p);
 
 // K2 on CUDA cores (3D, Alg. 2 with RDG per plane), one step.

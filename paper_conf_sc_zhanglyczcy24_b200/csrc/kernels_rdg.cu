@@ -291,6 +291,8 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
       const int64_t e = sc.ooff + int64_t(I) * P1;
       if constexpr (K > 1) {
         store_pairs<NH>(out + e, v, lc);
+        if (I < sc.rem_lo) store_pairs<NH>(dp.dst_lo + (e + dp.off_lo), v, lc);   // warp-uniform, rare
+        if (I >= sc.rem_hi) store_pairs<NH>(dp.dst_hi + (e + dp.off_hi), v, lc);
       } else {
         // the row goes to this slab and, for the first / last R interior rows of a slab with a
         // neighbour there, into that neighbour's halo as well (peer memory, csrc/dist_p2p.cu;
@@ -402,11 +404,12 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
     X0 = R + band * BS - R * (K - 1) - SG;
     A = R + chunk * RC;
   };
-  // device-initiated exchange (K = 1 only): the item holding the first (last) R interior rows of
-  // the slab touches the lower (upper) neighbour; the host keeps that item unique per band
+  // device-initiated exchange: the item holding the first (last) H rows of the slab touches the
+  // lower (upper) neighbour — it stores them into the neighbour's halo and stages the halo the
+  // neighbour wrote; the host keeps that item unique per band (RC >= 2H, last chunk >= 2H - R rows)
   auto touches = [&](int A_, bool& lo, bool& hi) {
-    lo = dp.active && dp.dst_lo != nullptr && A_ < 2 * R;
-    hi = dp.active && dp.dst_hi != nullptr && A_ + RC - 1 >= N0;
+    lo = dp.active && dp.dst_lo != nullptr && A_ < dp.lo_end;
+    hi = dp.active && dp.dst_hi != nullptr && A_ + RC - 1 >= dp.hi_begin;
   };
   // producer position (next stage to stage into the ring)
   int pitem = gw, pj = 0, pX0 = 0, pA = 0;
@@ -417,7 +420,8 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
       bool lo, hi;
       touches(pA, lo, hi);
       if (lane == 0 && (lo || hi)) {
-        const int b = pitem % nbands, u0 = max(b - 1, 0), u1 = min(b + 1, nbands - 1);
+        const int b = pitem % nbands;
+        const int u0 = dp.wait_units > 0 ? 0 : max(b - 1, 0), u1 = dp.wait_units > 0 ? dp.wait_units - 1 : min(b + 1, nbands - 1);
         if (lo) p2p_wait_units(dp.wait_lo, u0, u1, dp.wait_val, dp.err);
         if (hi) p2p_wait_units(dp.wait_hi, u0, u1, dp.wait_val, dp.err);
         fence_proxy_async_global();
@@ -491,7 +495,7 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
         lc.vec[h] = lc.valid[h][0] && lc.valid[h][1] &&
                     ((reinterpret_cast<uintptr_t>(out + lc.c0 + 64 * h) & 15) == 0) && ((P1 & 1) == 0);
       }
-      rows_valid_end = min(A + RC, P0 - R);
+      rows_valid_end = min(A + RC, dp.active ? dp.store_hi : P0 - R);
       bool mine = !lc.edge;   // FULL lanes: no halo columns; a pair is stored as one 16-byte store or not at all
 #pragma unroll
       for (int h = 0; h < NH; ++h) mine = mine && lc.valid[h][0] == lc.valid[h][1] && (lc.vec[h] || !lc.valid[h][0]);
@@ -502,11 +506,11 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
     const int yb = A - K * R + cj * G::SROWS;
     {
       const int yf = yb - K * R - (K - 1);  // final row produced by input row I = 0 (one-row lag per stage)
-      sc.lo = A - yf;
+      sc.lo = (dp.active ? max(A, dp.store_lo) : A) - yf;
       sc.hi = rows_valid_end - yf;
       sc.ooff = int64_t(yf) * P1 + lc.c0;
-      sc.rem_lo = t_lo ? 2 * R - yf : INT_MIN;          // padded rows [R, 2R)
-      sc.rem_hi = t_hi ? (int)N0 - yf : INT_MAX;        // padded rows [N0, N0 + R)
+      sc.rem_lo = t_lo ? dp.lo_end - yf : INT_MIN;       // rows [store_lo, lo_end)
+      sc.rem_hi = t_hi ? dp.hi_begin - yf : INT_MAX;     // rows [hi_begin, store_hi)
 #pragma unroll
       for (int S = 1; S < K; ++S) {
         const int ys = yb - S * R - (S - 1);  // stage-S row produced by input row I = 0
@@ -589,6 +593,7 @@ cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream
     if (e != cudaSuccess) return e;
     max_grid = persistent_grid((const void*)rdg2d_kernel<R, SIG, K, TMA>, RDG_WARPS * 32, smem, int64_t(1) << 40);
   }
+  if (d && d->prepare_only) return cudaSuccess;
   // chunk rows: a multiple of 2R+1 (static ring slots), <= RDG_RC; small grids get shorter chunks
   // so that every resident warp has a stream (>= 2 items per warp slot when the grid allows it)
   const int nbands = (int)((p.N[1] + BS - 1) / BS);
@@ -606,15 +611,19 @@ cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream
     rc2 = ((rc2 + n - 1) / n) * n;
     if (rc2 <= RDG_RC + n && rc2 >= 4 * K * R && nbands * ((p.N[0] + rc2 - 1) / rc2) <= rounds * TWmax) rc = rc2;
   }
-  if (d && d->active && rc < p.N[0]) {
-    // device-initiated exchange: exactly one chunk per band may hold the last R interior rows
-    // (the last chunk must have >= R rows), so that one item per band and side signals
-    int64_t ok = 0;
-    for (int64_t c = rc; c <= rc + 40 * n && !ok; c += n) {
-      const int64_t rem = p.N[0] % c;
-      if (rem == 0 || rem >= R) ok = c;
+  if (d && d->active) {
+    // device-initiated exchange: exactly one chunk per band and side may touch a neighbour: the
+    // first chunk must hold rows [store_lo, lo_end) (RC >= 2H) and the last one >= 2H - R rows
+    const int64_t H = std::max(d->H, R);
+    rc = std::max<int64_t>(rc, ((2 * H + n - 1) / n) * n);
+    if (rc < p.N[0]) {
+      int64_t ok = 0;
+      for (int64_t c = rc; c <= rc + 40 * n && !ok; c += n) {
+        const int64_t rem = p.N[0] % c;
+        if (rem == 0 || rem >= 2 * H - R) ok = c;
+      }
+      rc = ok ? ok : ((p.N[0] + n - 1) / n) * n;
     }
-    rc = ok ? ok : ((p.N[0] + n - 1) / n) * n;
   }
   const int RC = (int)rc;
   const int SI = (RC + 2 * K * R + (K - 1) + G::SROWS - 1) / G::SROWS;
@@ -645,16 +654,16 @@ constexpr int max_fuse(int R) { return R == 1 ? 4 : (R == 2 ? 3 : 2); }
 template <int R, int SIG>
 cudaError_t rdg_k(const Plan& p, const double* src, double* dst, cudaStream_t s, const RdgParams& prm, int k,
                   const P2PArgs* d = nullptr) {
-  if (d) return k == 1 ? rdg_sig<R, SIG, 1>(p, src, dst, s, prm, d) : cudaErrorNotSupported;
+  if (d && (k == 1 || SIG == SIG_FULL || SIG == SIG_DIRECT)) return k == 1 ? rdg_sig<R, SIG, 1>(p, src, dst, s, prm, d) : cudaErrorNotSupported;
   if constexpr (SIG == SIG_FULL || SIG == SIG_DIRECT) {
     if (k != 1) return cudaErrorNotSupported;
     return rdg_sig<R, SIG, 1>(p, src, dst, s, prm);
   } else {
     switch (k) {
-      case 1: return rdg_sig<R, SIG, 1>(p, src, dst, s, prm);
-      case 2: return rdg_sig<R, SIG, 2>(p, src, dst, s, prm);
-      case 3: if constexpr (max_fuse(R) >= 3) return rdg_sig<R, SIG, (max_fuse(R) >= 3 ? 3 : 1)>(p, src, dst, s, prm); break;
-      case 4: if constexpr (max_fuse(R) >= 4) return rdg_sig<R, SIG, (max_fuse(R) >= 4 ? 4 : 1)>(p, src, dst, s, prm); break;
+      case 1: return rdg_sig<R, SIG, 1>(p, src, dst, s, prm, d);
+      case 2: return rdg_sig<R, SIG, 2>(p, src, dst, s, prm, d);
+      case 3: if constexpr (max_fuse(R) >= 3) return rdg_sig<R, SIG, (max_fuse(R) >= 3 ? 3 : 1)>(p, src, dst, s, prm, d); break;
+      case 4: if constexpr (max_fuse(R) >= 4) return rdg_sig<R, SIG, (max_fuse(R) >= 4 ? 4 : 1)>(p, src, dst, s, prm, d); break;
     }
     return cudaErrorNotSupported;
   }
@@ -723,18 +732,38 @@ int p2p_units(const Plan& p, int* nux) {
   return (int)((p.N[1] + 63) / 64);
 }
 
-cudaError_t launch_step_p2p(const Plan& p, const double* src, double* dst, cudaStream_t s, const P2PArgs& d) {
-  if (p.ndim == 3) return launch_rdg3d_p2p(p, src, dst, s, d);
+cudaError_t launch_step_p2p(const Plan& p, const double* src, double* dst, cudaStream_t s, const P2PArgs& d, int k) {
+  if (p.ndim == 3) return k == 1 ? launch_rdg3d_p2p(p, src, dst, s, d) : cudaErrorNotSupported;
   if (p.ndim != 2) return cudaErrorNotSupported;
-  if (p.engine == LORA_ENGINE_DIRECT) return direct2d(p, src, dst, s, &d);
+  if (p.engine == LORA_ENGINE_DIRECT) return k == 1 ? direct2d(p, src, dst, s, &d) : cudaErrorNotSupported;
   if (p.engine != LORA_ENGINE_RDG_CUDA) return cudaErrorNotSupported;
   switch (p.R) {
-    case 1: return rdg_r<1>(p, src, dst, s, 1, &d);
-    case 2: return rdg_r<2>(p, src, dst, s, 1, &d);
-    case 3: return rdg_r<3>(p, src, dst, s, 1, &d);
-    case 4: return rdg_r<4>(p, src, dst, s, 1, &d);
+    case 1: return rdg_r<1>(p, src, dst, s, k, &d);
+    case 2: return rdg_r<2>(p, src, dst, s, k, &d);
+    case 3: return rdg_r<3>(p, src, dst, s, k, &d);
+    case 4: return rdg_r<4>(p, src, dst, s, k, &d);
   }
   return cudaErrorInvalidValue;
+}
+
+// Band count of the 2D stream kernel at fusion depth k (the flag units of the exchange).
+namespace {
+template <int R>
+int band_stride(int k) {
+  int nh = 1;
+  switch (k) {
+    case 2: nh = rdg_nh<R, SIG_PMA, 2>(); break;
+    case 3: nh = rdg_nh<R, SIG_PMA, 3>(); break;
+    case 4: nh = rdg_nh<R, SIG_PMA, 4>(); break;
+  }
+  return 64 * nh - 2 * R * (k - 1) - 2 * ((R * (k - 1)) & 1);
+}
+}  // namespace
+
+int p2p_units_k(const Plan& p, int k) {
+  if (p.ndim != 2 || k <= 1) return p2p_units(p, nullptr);
+  const int bs = p.R == 1 ? band_stride<1>(k) : p.R == 2 ? band_stride<2>(k) : p.R == 3 ? band_stride<3>(k) : band_stride<4>(k);
+  return (int)((p.N[1] + bs - 1) / bs);
 }
 
 cudaError_t launch_rdg2d(const Plan& p, const double* src, double* dst, cudaStream_t s, int k) {

@@ -429,6 +429,7 @@ cudaError_t rdg3d_launch(const Plan& p, const double* src, double* dst, cudaStre
     if (e != cudaSuccess) return e;
     max_grid = persistent_grid((const void*)rdg3d_kernel<R, SG, TMA>, R3_WARPS * 32, G::SMEM, int64_t(1) << 40);
   }
+  if (d && d->prepare_only) return cudaSuccess;
   const int nbx = (int)((p.N[2] + 63) / 64), nby = (int)((p.N[1] + BY<R> - 1) / BY<R>);
   // z-chunk length: the fewest whole rounds of resident warps, then the shortest chunk that fits
   const int64_t TWmax = int64_t(max_grid) * R3_WARPS;

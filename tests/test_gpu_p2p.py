@@ -36,7 +36,7 @@ def _split(n0, counts):
     return list(zip(starts.tolist(), counts))
 
 
-def _run_local(W, g, h, shape, T, engine, counts, zero_copy=False, repeat=1):
+def _run_local(W, g, h, shape, T, engine, counts, zero_copy=False, repeat=1, fuse_k=1):
     """P slab ranks in this process; returns the gathered global padded result (halo = input)."""
     import torch
     import paper_conf_sc_zhanglyczcy24_b200 as L
@@ -45,7 +45,7 @@ def _run_local(W, g, h, shape, T, engine, counts, zero_copy=False, repeat=1):
     P = len(slabs)
     sts, eps, xs, ys, streams = [], [], [], [], []
     for r, (s0, c) in enumerate(slabs):
-        st = L.Stencil(W, (c,) + tuple(shape[1:]), engine=engine, fuse_k=1)
+        st = L.Stencil(W, (c,) + tuple(shape[1:]), engine=engine, fuse_k=fuse_k)
         sts.append(st)
         eps.append(L.lora_stencil_p2p_create(st.plan, P, r))
         xs.append(torch.from_numpy(np.ascontiguousarray(D.local_slice(g, s0, c, h))).cuda())
@@ -135,6 +135,34 @@ def test_p2p_local_ranks_bitwise(case):
         assert rel_err(out, oracle.run(W, g, 5)) <= 1e-12
 
 
+FUSED = [
+    # d, h, kind, global interior shape, slab row counts, fusion depth k (deep halos H = k h)
+    (3, "rsym", (300, 200), [150, 150], 2),            # Box-2D49P row-pair form, the bench default
+    (3, "rsym", (301, 130), [100, 6, 195], 2),          # a slab of exactly H rows
+    (1, "rsym", (517, 300), [129, 130, 128, 130], 3),   # Box-2D9P default depth
+    (1, "rsym", (260, 70), [70, 60, 130], 4),
+    (2, "star", (260, 190), [130, 130], 3),
+    (2, "rsym", (200, 77), [67, 133], 2),
+    (3, "star", (256, 300), [128, 128], 2),
+]
+
+
+@pytest.mark.parametrize("case", FUSED)
+def test_p2p_fused_deep_halo_bitwise(case):
+    """k fused steps per launch across slab ranks: internal edges carry H = k h deep halos (the kernel
+    recomputes the rows between h and H redundantly and stores only its own rows); T covers remainder
+    launches (T mod k != 0) whose band geometry differs from the full launches."""
+    h, kind, shape, counts, k = case
+    W = _weights(kind, 2, h, 41 + h)
+    g = synth.grid(tuple(n + 2 * h for n in shape), 43)
+    for T in sorted({1, k, k + 1, 2 * k + 1, 7}):
+        ref = _global(W, g, T, "rdg_cuda")
+        out = _run_local(W, g, h, shape, T, "rdg_cuda", counts, fuse_k=k)
+        assert np.array_equal(out, ref), (T, float(np.nanmax(np.abs(out - ref))))
+    out = _run_local(W, g, h, shape, 5, "rdg_cuda", counts, fuse_k=k, repeat=2)
+    assert np.array_equal(out, _global(W, g, 5, "rdg_cuda"))
+
+
 def test_p2p_repeated_runs_and_zero_copy():
     """Epochs: the same endpoints run three times (monotonic step counters, no reset); zero-copy
     mode reads buffer 0 and leaves the result in buffer T % 2."""
@@ -156,6 +184,8 @@ def test_p2p_large_slabs_many_items():
     ref = _global(W, g, T, "rdg_cuda")
     out = _run_local(W, g, h, shape, T, "rdg_cuda", [512, 512, 512, 512])
     assert np.array_equal(out, ref)
+    out = _run_local(W, g, h, shape, 5, "rdg_cuda", [512, 512, 512, 512], fuse_k=2)   # the bench default
+    assert np.array_equal(out, _global(W, g, 5, "rdg_cuda"))
 
 
 def test_p2p_unsupported_and_errors():
