@@ -31,6 +31,10 @@ import numpy as np  # noqa: E402
 METRIC = "GStencil/s FP64 per stencil at 1/2/4/8 B200; % of HBM roofline"
 UNIT = "GStencil/s"
 BYTES_PER_POINT = 16.0  # algorithmic HBM bytes per point per time step: read 8 + write 8
+# algorithmic FP64 flops per point per time step: the separable minimum of the rank-1 method
+# (SURVEY §8(d) "Roofline"; FMA = 2 flops)
+ALG_FLOPS_PER_POINT = {"heat2d-256": 10.0, "box2d9p-10240": 14.0, "box2d49p-10240": 62.0, "heat3d-512": 14.0,
+                       "box3d27p-512": 42.0}
 
 
 def parse():
@@ -315,27 +319,33 @@ def main():
     # kernel runs closest to (the larger fraction):
     #  hbm: ALGORITHMIC bytes per launch (16 B per point per launch: one read + one write of the grid,
     #       whatever the fused depth) / average launch time, vs the measured HBM copy bandwidth;
-    #  alu: FP64 pipe lane-ops per launch (the plan's issued FP64 ops per point-step, DFMA/DADD/DMUL
-    #       each one lane-op, x points x fused steps; band/chunk recomputation NOT counted) / average
-    #       launch time, vs 148 SMs x 64 FP64 lanes x 1.965 GHz (the step-0 DMMA
-    #       microbenchmark reaches 36.9 TFLOP/s = 99 % of that).
+    #  alu: ALGORITHMIC FP64 flops per launch (SURVEY.md §8(d)'s per-point figure — the separable
+    #       minimum of the rank-1 method, FMA = 2 flops — x points x fused steps) / average launch
+    #       time, vs 148 SMs x 64 FP64 FMA/clk x 2 x 1.965 GHz = 37.2 TFLOP/s (the step-0
+    #       DMMA microbenchmark reaches 36.9).  "issued" adds what the kernel really puts through the
+    #       FP64 pipe: the plan's issued FP64 instructions per point-step (DFMA/DADD/DMUL, each one
+    #       lane slot) against 148 x 64 lane slots x 1.965 GHz.
     peak, peak_src = load_peaks()
     n_launch = -(-T // fuse)
     per_launch_bytes = BYTES_PER_POINT * float(np.prod(shape))      # per launch: one (fused) superstep
     avg_launch_s = t / args.steps / n_launch
     achieved = per_launch_bytes / avg_launch_s / 1e9
-    fp64_peak_gops = 148 * 64 * 1.965                                  # G lane-ops/s
-    ops_per_launch = info["fma_per_point_issued"] * float(np.prod(shape)) * (T / n_launch)
-    alu_achieved = ops_per_launch / avg_launch_s / 1e9
+    fp64_peak_tflops = 148 * 64 * 2 * 1.965e9 / 1e12
+    alg_flops_pt = ALG_FLOPS_PER_POINT.get(args.workload, 2.0 * info["fma_per_point_separable"])
+    flops_per_launch = alg_flops_pt * float(np.prod(shape)) * (T / n_launch)
+    alu_achieved = flops_per_launch / avg_launch_s / 1e12
+    issued_ops = info["fma_per_point_issued"] * float(np.prod(shape)) * (T / n_launch) / avg_launch_s
     tr = ncu_traffic(args.workload, info["engine_name"])
     if tr and int(tr.get("fuse", 1)) != fuse:
         tr = None
     hbm = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
            "peak_source": peak_src, "algorithmic_bytes_per_launch": per_launch_bytes}
-    alu = {"bound": "alu", "achieved": alu_achieved, "peak": fp64_peak_gops, "unit": "Gop/s (FP64 pipe lane-ops)",
-           "frac": alu_achieved / fp64_peak_gops,
-           "peak_source": "derived: 148 SMs x 64 FP64 lanes x 1.965 GHz (DESIGN.md §6)",
-           "algorithmic_ops_per_launch": ops_per_launch}
+    alu = {"bound": "alu", "achieved": alu_achieved, "peak": fp64_peak_tflops, "unit": "TFLOP/s",
+           "frac": alu_achieved / fp64_peak_tflops,
+           "peak_source": "derived: 148 SMs x 64 FP64 FMA/clk x 2 flops x 1.965 GHz (DESIGN.md §6)",
+           "algorithmic_flops_per_point": alg_flops_pt, "algorithmic_flops_per_launch": flops_per_launch,
+           "issued": {"fp64_instr_per_point": info["fma_per_point_issued"], "gop_s": issued_ops / 1e9,
+                      "frac_of_pipe": issued_ops / (148 * 64 * 1.965e9)}}
     roof = dict(alu if alu["frac"] > hbm["frac"] else hbm)
     roof.update({"traffic": tr["bytes"] if tr else None,       # dram read+write bytes per launch (ncu --set full)
                  "traffic_source": ({k: tr[k] for k in ("kernel", "source", "fuse")} if tr else None),
