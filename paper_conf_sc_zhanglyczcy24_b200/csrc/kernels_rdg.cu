@@ -27,7 +27,10 @@
 namespace lora {
 namespace {
 
-constexpr int RDG_RC = 128;     // output rows per work item (chunk)
+#ifndef RDG_RC_ROWS
+#define RDG_RC_ROWS 128   // experiments: chunk length
+#endif
+constexpr int RDG_RC = RDG_RC_ROWS;   // output rows per work item (chunk)
 constexpr int RDG_WARPS = 4;    // warps per CTA (independent streams)
 constexpr int RDG_NS = 3;       // ring stages per warp (3 keeps 4 CTAs = 16 warps per SM)
 
@@ -347,6 +350,13 @@ __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p,
 #ifndef RDG_NH_FUSED
 #define RDG_NH_FUSED 2   // 64-column halves per warp in the fused (K >= 2) kernels
 #endif
+// Check-free copy of the row loop for interior stages: unfused kernels, and the fused heavy
+// (radius >= 3 rows / PMA) kernels whose per-row FP64 work dwarfs the doubled code footprint
+// (Box-2D49P k = 2: 294-301 -> 312 GS/s, short runs); not the light fused kernels.
+template <int R, int SIG, int K>
+constexpr bool rdg_full() {
+  return RDG_FULL == 1 || (RDG_FULL == 2 && (K == 1 || (R >= 3 && (SIG == SIG_ROWS || SIG == SIG_PMA))));
+}
 template <int R, int K>
 constexpr int rdg_cta_smem(int nh) {   // must match rdg_launch
   return nh == 1 ? 128 + RDG_WARPS * (Geom<R, 1>::WARP_BYTES + 2 * (K - 1) * Geom<R, 1>::BUFD * 8)
@@ -525,7 +535,7 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
     bool full = all_fast && sc.lo <= 0 && sc.hi >= G::SROWS && sc.rem_lo <= 0 && sc.rem_hi >= G::SROWS;
 #pragma unroll
     for (int S = 1; S < K; ++S) full = full && sc.hlo[S - 1] <= 0 && sc.hhi[S - 1] >= G::SROWS;
-    if ((RDG_FULL == 1 || (RDG_FULL == 2 && K == 1)) && full) fused_rows<R, SIG, K, NH, true, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp);
+    if (rdg_full<R, SIG, K>() && full) fused_rows<R, SIG, K, NH, true, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp);
     else fused_rows<R, SIG, K, NH, false, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp);
     __syncwarp();  // every lane is done with this slot before it is refilled
     if (++slot == RDG_NS) { slot = 0; phase ^= 1; }
