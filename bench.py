@@ -40,7 +40,7 @@ ALG_FLOPS_PER_POINT = {"heat2d-256": 10.0, "box2d9p-10240": 14.0, "box2d49p-1024
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="box2d49p-10240")
@@ -48,6 +48,8 @@ def parse():
     ap.add_argument("--fuse", type=int, default=0)
     ap.add_argument("--per-stencil", action="store_true", help="also time the other single-GPU configs")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-inflight", type=int, default=3,
+                    help="independent problems in flight in the e2e run (one plan + stream each)")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-engines", action="store_true", help="skip the per-engine comparison on the workload")
     ap.add_argument("--dist", default="p2p", choices=["p2p", "nccl"],
@@ -357,9 +359,10 @@ def main():
                  "frac_gstencil_of_hbm_roofline": value / (peak / BYTES_PER_POINT * world)})
 
     # e2e: through the C-ABI with HOST buffers (H2D of the input + D2H of the result inside the region).
-    # Headline = two independent problems in flight (two plans, two streams, steps alternate): one
-    # problem's PCIe copies overlap the other's stencil steps.  "serial" = one synchronous
-    # lora_stencil_run_host call per step (copies not overlapped).
+    # Headline = M independent problems in flight (M plans, M streams, steps round-robin): the PCIe
+    # copies of some problems overlap the stencil steps of another (one problem's H2D + D2H take
+    # about as long as its T steps, so M = 2 leaves no slack; M = 3 keeps the SMs fed).  "serial" =
+    # one synchronous lora_stencil_run_host call per step (copies not overlapped).
     e2e = None
     if not args.no_e2e and comm is None and ep is None:
         nbytes = host_in.numel() * 8
@@ -369,25 +372,28 @@ def main():
         for _ in range(args.steps):
             L.lora_stencil_run_host(st.plan, host_in.numpy(), host_out.numpy(), T, sptr)
         te_serial = time.perf_counter() - t0
-        st2 = L.Stencil(W, shape, engine=args.engine, fuse_k=args.fuse)
-        plans = [st.plan, st2.plan]
-        streams = [torch.cuda.Stream(dev), torch.cuda.Stream(dev)]
-        hin = [host_in, torch.from_numpy(synth.grid(padded, cfg["seed"] + 1000 * rank + 1)).pin_memory()]
-        hout = [host_out, torch.empty_like(host_in).pin_memory()]
-        for j in range(2):
+        M = max(1, args.e2e_inflight)
+        extra = [L.Stencil(W, shape, engine=args.engine, fuse_k=args.fuse) for _ in range(M - 1)]
+        plans = [st.plan] + [e.plan for e in extra]
+        streams = [torch.cuda.Stream(dev) for _ in range(M)]
+        hin = [host_in] + [torch.from_numpy(synth.grid(padded, cfg["seed"] + 1000 * rank + j)).pin_memory()
+                           for j in range(1, M)]
+        hout = [host_out] + [torch.empty_like(host_in).pin_memory() for _ in range(1, M)]
+        for j in range(M):
             L.lora_stencil_run_host_async(plans[j], hin[j], hout[j], T, streams[j].cuda_stream)
         torch.cuda.synchronize(dev)
         t0 = time.perf_counter()
         for i in range(args.steps):
-            j = i & 1
+            j = i % M
             L.lora_stencil_run_host_async(plans[j], hin[j], hout[j], T, streams[j].cuda_stream)
         for s_ in streams:
             s_.synchronize()
         te = time.perf_counter() - t0
-        st2.close()
+        for e in extra:
+            e.close()
         e2e = {"value": pts_per_step * args.steps / te / 1e9, "unit": UNIT, "h2d_bytes_per_step": nbytes,
                "d2h_bytes_per_step": nbytes,
-               "api": "lora_stencil_run_host_async (pinned host buffers), 2 problems in flight on 2 streams",
+               "api": f"lora_stencil_run_host_async (pinned host buffers), {M} problems in flight on {M} streams",
                "serial": {"value": pts_per_step * args.steps / te_serial / 1e9,
                           "api": "lora_stencil_run_host, one synchronous call per step"},
                "clock": "host wall clock around the K steps"}

@@ -287,8 +287,13 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
   } else if constexpr (FULL) {
     double* o = out + sc.ooff + int64_t(I) * P1;
 #pragma unroll
-    for (int h = 0; h < NH; ++h)   // band-overlap lanes of a fused band store nothing
-      if (lc.vec[h]) *reinterpret_cast<double2*>(o + 64 * h) = make_double2(v[h][0], v[h][1]);
+    for (int h = 0; h < NH; ++h) {   // band-overlap lanes of a fused band store nothing
+      if constexpr (R & 1) {   // odd R: lane pairs start on odd columns (8-byte stores)
+        if (lc.valid[h][0]) { o[64 * h] = v[h][0]; o[64 * h + 1] = v[h][1]; }
+      } else {
+        if (lc.vec[h]) *reinterpret_cast<double2*>(o + 64 * h) = make_double2(v[h][0], v[h][1]);
+      }
+    }
   } else {
     if (I >= sc.lo && I < sc.hi) {
       const int64_t e = sc.ooff + int64_t(I) * P1;
@@ -342,20 +347,19 @@ __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p,
 // (profiles/r01_rdg_occupancy.txt): the heavy radius >= 3 PMA pass wants registers for ILP more
 // than warps (2 CTAs: 338 GS/s vs 305 at 4 for Box-2D49P); light passes want 4; fused radius >= 2 3.
 #ifndef RDG_FULL
-// 2: unfused kernels get a second copy of the row loop without per-row checks for interior stages
-// (Box-2D49P 314 -> 339 GS/s); the fused kernels do not (their doubled hot code footprint costs
-// more than the checks: Star-2D13P k=2 412 -> 360).  0: never, 1: always (experiments).
+// 2: unfused kernels get a second copy of the row loop without per-row checks for interior stages;
+// the fused kernels do not (see rdg_full).  0: never, 1: always (experiments).
 #define RDG_FULL 2
 #endif
 #ifndef RDG_NH_FUSED
 #define RDG_NH_FUSED 2   // 64-column halves per warp in the fused (K >= 2) kernels
 #endif
-// Check-free copy of the row loop for interior stages: unfused kernels, and the fused heavy
-// (radius >= 3 rows / PMA) kernels whose per-row FP64 work dwarfs the doubled code footprint
-// (Box-2D49P k = 2: 294-301 -> 312 GS/s, short runs); not the light fused kernels.
+// Check-free copy of the row loop for interior stages: unfused kernels only.  Measured on one box
+// (tools/gpu_variants.sh, short runs): the fused kernels are slower with it — Box-2D49P k = 2 310 ->
+// 261 GS/s, Star-2D13P k = 2 431 -> 351 — and the unfused ones gain little (Star-2D13P 311 -> 317).
 template <int R, int SIG, int K>
 constexpr bool rdg_full() {
-  return RDG_FULL == 1 || (RDG_FULL == 2 && (K == 1 || (R >= 3 && (SIG == SIG_ROWS || SIG == SIG_PMA))));
+  return RDG_FULL == 1 || (RDG_FULL == 2 && K == 1);
 }
 template <int R, int K>
 constexpr int rdg_cta_smem(int nh) {   // must match rdg_launch
@@ -506,9 +510,13 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
                     ((reinterpret_cast<uintptr_t>(out + lc.c0 + 64 * h) & 15) == 0) && ((P1 & 1) == 0);
       }
       rows_valid_end = min(A + RC, dp.active ? dp.store_hi : P0 - R);
-      bool mine = !lc.edge;   // FULL lanes: no halo columns; a pair is stored as one 16-byte store or not at all
+      // FULL lanes: no halo columns; a pair is stored as a whole or not at all — one 16-byte store
+      // for even R; for odd R the lane columns X0 + 2p are odd (the staged origin X0 - R is kept
+      // even for TMA), so the pair is two 8-byte stores
+      bool mine = !lc.edge;
 #pragma unroll
-      for (int h = 0; h < NH; ++h) mine = mine && lc.valid[h][0] == lc.valid[h][1] && (lc.vec[h] || !lc.valid[h][0]);
+      for (int h = 0; h < NH; ++h)
+        mine = mine && lc.valid[h][0] == lc.valid[h][1] && ((R & 1) || lc.vec[h] || !lc.valid[h][0]);
       all_fast = __all_sync(0xffffffffu, mine);
       touches(A, t_lo, t_hi);
     }
