@@ -155,11 +155,24 @@ __device__ __forceinline__ void load_rows(const double* __restrict__ base, int p
 
 // Intermediate stage S (1 <= S < K): the stage-S plane just completed in acc[S-1] (ring slot CS)
 // gets the fixed Dirichlet halo re-imposed and is published to its shared plane buffer.
+// fast: every element of the lane is strictly inside the array in x, y (precomputed per item) and
+// z (per plane) — no halo value to re-impose, no zero fill: plain stores.
 template <int K, int S, int CS>
 __device__ __forceinline__ void publish(double (&acc)[K][3][2][2], double* __restrict__ buf, int w, int lane,
                                         int Y0, int X0, int zs, int P0, int P1, int P2,
-                                        const double* __restrict__ in) {
+                                        const double* __restrict__ in, bool fast) {
   const int c0 = 2 * lane;
+  if (fast) {
+#pragma unroll
+    for (int y = 0; y < 2; ++y) {
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        buf[(2 * w + y) * F_S1W + 1 + c0 + e] = acc[S - 1][CS][y][e];
+        acc[S - 1][CS][y][e] = 0.0;
+      }
+    }
+    return;
+  }
 #pragma unroll
   for (int y = 0; y < 2; ++y) {
     double v[2] = {acc[S - 1][CS][y][0], acc[S - 1][CS][y][1]};
@@ -249,6 +262,10 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
   int citem = blockIdx.x, cj = 0, slot = 0, phase = 0;
   int X0 = 0, Y0 = 0, Z0 = 0, zend = 0;
   const int c0 = 2 * lane;  // lane's first column (relative to X0)
+  // per item: intermediate stage S rows/columns of this lane strictly inside (publish fast path);
+  // final elements of this lane to store (row / column validity, the z test is per plane)
+  bool xy_in[K > 1 ? K - 1 : 1];
+  bool st_ok[2][2];
   for (int q0 = 0; q0 < nstages; q0 += 3) {
     auto one = [&](auto Ic) {
       constexpr int I = decltype(Ic)::value;
@@ -258,6 +275,21 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
       if (cj == 0) {
         geom(citem, X0, Y0, Z0);
         zend = min(Z0 + ZC, P0 - 1);
+        const bool xs_in = X0 + c0 >= 1 && X0 + c0 + 1 < P2 - 1;
+#pragma unroll
+        for (int S = 1; S < K; ++S) {
+          const int gy = Y0 - (K - S) + 2 * w;
+          xy_in[S - 1] = xs_in && gy >= 1 && gy + 1 < P1 - 1;
+        }
+#pragma unroll
+        for (int y = 0; y < 2; ++y) {
+          const int gy = Y0 + 2 * w + y;
+#pragma unroll
+          for (int e = 0; e < 2; ++e) {
+            const int cx = X0 + c0 + e;
+            st_ok[y][e] = gy < P1 - 1 && gy < Y0 + TY && c0 + e >= K - 1 && c0 + e < 65 - K && cx >= 1 && cx < P2 - 1;
+          }
+        }
 #pragma unroll
         for (int k = 0; k < K; ++k)
 #pragma unroll
@@ -273,7 +305,8 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
         double x[4][4];
         load_rows(st + (2 * w) * F_BW, F_BW, lane, x);
         planes2<SG, I, 0>(x, prm, acc[0]);
-        publish<K, 1, (I + 1) % 3>(acc, sbuf + (0 * 2 + par) * S1B, w, lane, Y0, X0, p - 1, P0, P1, P2, in);
+        publish<K, 1, (I + 1) % 3>(acc, sbuf + (0 * 2 + par) * S1B, w, lane, Y0, X0, p - 1, P0, P1, P2, in,
+                                   xy_in[0] && p - 1 >= 1 && p - 1 < P0 - 1);
       }
       __syncthreads();  // stage-1 plane visible; every warp is done with the input slot
       if (q + F_NS - 1 < nstages) issue_next((slot + F_NS - 1) % F_NS);
@@ -290,25 +323,19 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
         }
         if constexpr (S < K) {
           if (active) publish<K, S, (IS + 1) % 3>(acc, sbuf + ((S - 1) * 2 + par) * S1B, w, lane, Y0, X0, p - S, P0, P1,
-                                                  P2, in);
+                                                  P2, in, xy_in[S - 1] && p - S >= 1 && p - S < P0 - 1);
           __syncthreads();
         } else if (active) {
           // final plane zf = p - K complete: ring slot (IS + 1) % 3
           constexpr int s = (IS + 1) % 3;
           const int zf = p - K;
           if (cj >= 2 * K && zf >= Z0 && zf < zend) {
+            double* o = out + (int64_t(zf) * P1 + Y0 + 2 * w) * P2 + X0 + c0;
 #pragma unroll
-            for (int y = 0; y < 2; ++y) {
-              const int gy = Y0 + 2 * w + y;
-              if (gy < P1 - 1 && gy < Y0 + TY) {
-                double* o = out + (int64_t(zf) * P1 + gy) * P2 + X0;
+            for (int y = 0; y < 2; ++y)
 #pragma unroll
-                for (int e = 0; e < 2; ++e) {
-                  const int cx = X0 + c0 + e;
-                  if (c0 + e >= K - 1 && c0 + e < 65 - K && cx >= 1 && cx < P2 - 1) o[c0 + e] = acc[K - 1][s][y][e];
-                }
-              }
-            }
+              for (int e = 0; e < 2; ++e)
+                if (st_ok[y][e]) o[y * P2 + e] = acc[K - 1][s][y][e];
           }
 #pragma unroll
           for (int y = 0; y < 2; ++y) { acc[K - 1][s][y][0] = 0.0; acc[K - 1][s][y][1] = 0.0; }
