@@ -63,17 +63,31 @@ struct Geom {
 __host__ __device__ constexpr int pmod(int a, int n) { return ((a % n) + n) % n; }
 
 // One input row r (r mod n == I mod n) of the stream: T for every term, scattered into the ring.
-template <int R, int SIG, int I>
-__device__ __forceinline__ void row_body(const double* __restrict__ xs, int p, double (&acc)[2 * R + 1][2],
-                                         const RdgParams& P) {
-  constexpr int n = 2 * R + 1;
-  double x[2 * R + 2];
+// The lane's 2R + 2 inputs of one row (columns 2p - R .. 2p + R + 1 of the band): R + 1 LDS.128.
+template <int R>
+__device__ __forceinline__ void load_x(const double* __restrict__ xs, int p, double (&x)[2 * R + 2]) {
 #pragma unroll
   for (int q = 0; q <= R; ++q) {
     const double2 t = *reinterpret_cast<const double2*>(xs + 2 * p + 2 * q);
     x[2 * q] = t.x;
     x[2 * q + 1] = t.y;
   }
+}
+
+template <int R, int SIG, int I>
+__device__ __forceinline__ void row_compute(const double (&x)[2 * R + 2], double (&acc)[2 * R + 1][2], const RdgParams& P);
+
+template <int R, int SIG, int I>
+__device__ __forceinline__ void row_body(const double* __restrict__ xs, int p, double (&acc)[2 * R + 1][2],
+                                         const RdgParams& P) {
+  double x[2 * R + 2];
+  load_x<R>(xs, p, x);
+  row_compute<R, SIG, I>(x, acc, P);
+}
+
+template <int R, int SIG, int I>
+__device__ __forceinline__ void row_compute(const double (&x)[2 * R + 2], double (&acc)[2 * R + 1][2], const RdgParams& P) {
+  constexpr int n = 2 * R + 1;
   if constexpr (SIG == SIG_PMA) {
     // PMA pyramid (eq. 15): term k has radius R-k; the last one is the scalar C_{h+1}.  The PMA
     // factors of a reflection-symmetric W are exactly palindromic (the planner takes the
@@ -237,18 +251,24 @@ __device__ __forceinline__ void store_pairs(double* o, const double (&v)[NH][2],
 // stage 1 by (S-1)(R+1) rows (StageCtx row offsets include the extra (S-1) rows).
 // FULL: every row of the stage is interior for every intermediate step, every final row is stored
 // and every lane stores a 16-byte pair (decided per stage, warp-uniform): no per-row checks.
-template <int R, int SIG, int K, int NH, bool FULL, int I0, int I, int S>
+// PRE: stage S's input row is already in xq (the prefetched stage-1 row); stages S down to SMIN run.
+template <int R, int SIG, int K, int NH, bool FULL, int I0, int I, int S, bool PRE = false, int SMIN = 1>
 __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, int p,
                                            double (&acc)[K][NH][2 * R + 1][2], const RdgParams& P,
                                            double* __restrict__ bufs, int par, const double* __restrict__ in,
                                            double* __restrict__ out, int64_t P1, const StageCtx<K>& sc,
-                                           const LaneCtx<NH>& lc, const P2PArgs& dp) {
+                                           const LaneCtx<NH>& lc, const P2PArgs& dp,
+                                           const double (&xq)[NH][2 * R + 2]) {
+  static_assert(!PRE || SMIN == S, "a preloaded stage runs alone");
   constexpr int n = 2 * R + 1;
   constexpr int BUFD = Geom<R, NH>::BUFD;
   constexpr int Is = pmod(I0 - (S - 1) * (R + 1), n);   // ring index of stage S's input row (any per-stage constant)
   const double* src = S == 1 ? st_row : bufs + (2 * (S - 2) + (par ^ 1)) * BUFD;
 #pragma unroll
-  for (int h = 0; h < NH; ++h) row_body<R, SIG, Is>(src + 64 * h, p, acc[S - 1][h], P);
+  for (int h = 0; h < NH; ++h) {
+    if constexpr (PRE) row_compute<R, SIG, Is>(xq[h], acc[S - 1][h], P);
+    else row_body<R, SIG, Is>(src + 64 * h, p, acc[S - 1][h], P);
+  }
   constexpr int cs = (Is + 1) % n;                // slot of the row this stage just completed
   double v[NH][2];
 #pragma unroll
@@ -322,21 +342,63 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
       }
     }
   }
-  if constexpr (S > 1) fused_iter<R, SIG, K, NH, FULL, I0, I, S - 1>(st_row, p, acc, P, bufs, par, in, out, P1, sc, lc, dp);
+  if constexpr (S > SMIN) fused_iter<R, SIG, K, NH, FULL, I0, I, S - 1, false, SMIN>(st_row, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq);
 }
 
+#ifndef RDG_PF
+#define RDG_PF 3   // fused kernels of radius >= RDG_PF: prefetch the next staged input row (0: never)
+#endif
+#ifndef RDG_PF2
+#define RDG_PF2 2  // K = 2: also load stage 2's input row before stage 1's work — 1: always, 2: star
+#endif             // arms only (Star-2D13P 435 -> 451 GS/s; Box-2D49P 322 -> 290: register spills), 0: never
+// Fused kernels with RDG_PF: stage 1 runs first on the row prefetched in the previous iteration,
+// then the next staged row (same TMA stage) is loaded into xq, then stages K .. 2 run — their FP64
+// work covers the shared-load latency of the next stage-1 row (which the per-row __syncwarp keeps
+// the compiler from hoisting).  The stages of an iteration are independent, so the order is free.
+// Measured (same box, short runs): Box-2D49P k = 2 312 -> 322 GS/s, Star-2D13P k = 2 unchanged;
+// radius 1 (Box-2D9P k = 3) not better, so radius >= 3 only.
 template <int R, int SIG, int K, int NH, bool FULL, int I>
 __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p, double (&acc)[K][NH][2 * R + 1][2],
                                            const RdgParams& P, double* __restrict__ bufs,
                                            const double* __restrict__ in, double* __restrict__ out, int64_t P1,
-                                           const StageCtx<K>& sc, const LaneCtx<NH>& lc, int par0, const P2PArgs& dp) {
+                                           const StageCtx<K>& sc, const LaneCtx<NH>& lc, int par0, const P2PArgs& dp,
+                                           double (&xq)[NH][2 * R + 2]) {
   constexpr int n = 2 * R + 1;
+  constexpr int BW = Geom<R, NH>::BW;
   if constexpr (I < Geom<R, NH>::SROWS) {
     constexpr int OFF = pmod(R - K * R, n);  // q0 mod n (RC is a multiple of n)
-    fused_iter<R, SIG, K, NH, FULL, pmod(I + OFF, n), I, K>(st + I * Geom<R, NH>::BW, p, acc, P, bufs, (par0 + I) & 1,
-                                                            in, out, P1, sc, lc, dp);
+    constexpr int I0 = pmod(I + OFF, n);
+    if constexpr (K > 1 && RDG_PF > 0 && R >= RDG_PF) {
+      if constexpr (I == 0) {
+#pragma unroll
+        for (int h = 0; h < NH; ++h) load_x<R>(st + 64 * h, p, xq[h]);
+      }
+      // PF2 (K = 2, light signatures): stage 2's input row (written by stage 1 in the previous
+      // iteration) is loaded before stage 1's work as well
+      constexpr bool PF2 = K == 2 && (RDG_PF2 == 1 || (RDG_PF2 == 2 && SIG == SIG_STAR));
+      double x2[NH][2 * R + 2];
+      if constexpr (PF2) {
+        const double* b2 = bufs + (((par0 + I) & 1) ^ 1) * Geom<R, NH>::BUFD;
+#pragma unroll
+        for (int h = 0; h < NH; ++h) load_x<R>(b2 + 64 * h, p, x2[h]);
+      }
+      fused_iter<R, SIG, K, NH, FULL, I0, I, 1, true, 1>(st + I * BW, p, acc, P, bufs, (par0 + I) & 1, in, out, P1, sc, lc,
+                                                         dp, xq);
+      if constexpr (I + 1 < Geom<R, NH>::SROWS) {
+#pragma unroll
+        for (int h = 0; h < NH; ++h) load_x<R>(st + (I + 1) * BW + 64 * h, p, xq[h]);
+      }
+      if constexpr (PF2)
+        fused_iter<R, SIG, K, NH, FULL, I0, I, 2, true, 2>(st + I * BW, p, acc, P, bufs, (par0 + I) & 1, in, out, P1, sc,
+                                                           lc, dp, x2);
+      else
+        fused_iter<R, SIG, K, NH, FULL, I0, I, K, false, 2>(st + I * BW, p, acc, P, bufs, (par0 + I) & 1, in, out, P1, sc,
+                                                            lc, dp, xq);
+    } else {
+      fused_iter<R, SIG, K, NH, FULL, I0, I, K>(st + I * BW, p, acc, P, bufs, (par0 + I) & 1, in, out, P1, sc, lc, dp, xq);
+    }
     if constexpr (K > 1) __syncwarp();
-    fused_rows<R, SIG, K, NH, FULL, I + 1>(st, p, acc, P, bufs, in, out, P1, sc, lc, par0, dp);
+    fused_rows<R, SIG, K, NH, FULL, I + 1>(st, p, acc, P, bufs, in, out, P1, sc, lc, par0, dp, xq);
   }
 }
 
@@ -543,8 +605,9 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
     bool full = all_fast && sc.lo <= 0 && sc.hi >= G::SROWS && sc.rem_lo <= 0 && sc.rem_hi >= G::SROWS;
 #pragma unroll
     for (int S = 1; S < K; ++S) full = full && sc.hlo[S - 1] <= 0 && sc.hhi[S - 1] >= G::SROWS;
-    if (rdg_full<R, SIG, K>() && full) fused_rows<R, SIG, K, NH, true, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp);
-    else fused_rows<R, SIG, K, NH, false, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp);
+    double xq[NH][2 * R + 2];   // prefetched stage-1 input row (RDG_PF)
+    if (rdg_full<R, SIG, K>() && full) fused_rows<R, SIG, K, NH, true, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
+    else fused_rows<R, SIG, K, NH, false, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
     __syncwarp();  // every lane is done with this slot before it is refilled
     if (++slot == RDG_NS) { slot = 0; phase ^= 1; }
     if (++cj == SI) {
