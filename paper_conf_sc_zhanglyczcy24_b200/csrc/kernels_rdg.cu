@@ -200,6 +200,100 @@ __device__ __forceinline__ void row_compute(const double (&x)[2 * R + 2], double
   }
 }
 
+// Shift-register form of the same row update, for the runtime row loop of the fused kernels
+// (RDG_LOOP): after input row r, p[j] holds output row r - R + j, so p'[j] = p[j+1] + (the
+// contributions of row r with vertical offset a = R - j) and p'[2R] = the first contribution of
+// row r + R; the completed row r - R is p[0].  The "shift" is only the choice of destination
+// register, so the row needs no static ring index and the loop need not be unrolled by 2R + 1
+// (the unrolled ring form's hot code overflows the instruction cache: ncu no_instruction stalls).
+// Per output row the contributions arrive in the same order as in the ring form (first one from
+// 0.0 or assigned exactly as there), so both forms give bitwise identical rows.
+template <int R, int SIG>
+__device__ __forceinline__ void row_shift(const double (&x)[2 * R + 2], double (&p)[2 * R + 1][2], const RdgParams& P) {
+  double sp0[R + 1], sp1[R + 1];
+  if constexpr (SIG == SIG_ROWS || SIG == SIG_PMA) {
+#pragma unroll
+    for (int b = 1; b <= R; ++b) {
+      sp0[b] = x[R - b] + x[R + b];
+      sp1[b] = x[R - b + 1] + x[R + b + 1];
+    }
+  }
+  if constexpr (SIG == SIG_ROWS) {
+    double t[R + 1][2];
+#pragma unroll
+    for (int a = 0; a <= R; ++a) {
+      double t0 = P.v[a][R] * x[R], t1 = P.v[a][R] * x[R + 1];
+#pragma unroll
+      for (int b = 1; b <= R; ++b) {
+        t0 = fma(P.v[a][R + b], sp0[b], t0);
+        t1 = fma(P.v[a][R + b], sp1[b], t1);
+      }
+      t[a][0] = t0;
+      t[a][1] = t1;
+    }
+#pragma unroll
+    for (int j = 0; j < 2 * R; ++j) {
+      const int a = j < R ? R - j : j - R;
+      p[j][0] = p[j + 1][0] + t[a][0];
+      p[j][1] = p[j + 1][1] + t[a][1];
+    }
+    p[2 * R][0] = t[R][0];
+    p[2 * R][1] = t[R][1];
+  } else if constexpr (SIG == SIG_PMA) {
+    double t[R][2];
+#pragma unroll
+    for (int k = 0; k < R; ++k) {
+      const int H = R - k;
+      double t0 = P.v[k][R] * x[R], t1 = P.v[k][R] * x[R + 1];
+#pragma unroll
+      for (int b = 1; b <= H; ++b) {
+        t0 = fma(P.v[k][R + b], sp0[b], t0);
+        t1 = fma(P.v[k][R + b], sp1[b], t1);
+      }
+      t[k][0] = t0;
+      t[k][1] = t1;
+    }
+#pragma unroll
+    for (int j = 0; j <= 2 * R; ++j) {
+      const int a = R - j;
+      double q0 = j < 2 * R ? p[j + 1][0] : 0.0, q1 = j < 2 * R ? p[j + 1][1] : 0.0;
+#pragma unroll
+      for (int k = 0; k < R; ++k) {
+        if (a <= R - k && -a <= R - k) {
+          q0 = fma(P.u[k][R + a], t[k][0], q0);
+          q1 = fma(P.u[k][R + a], t[k][1], q1);
+        }
+      }
+      if (a == 0) {
+        q0 = fma(P.c, x[R], q0);
+        q1 = fma(P.c, x[R + 1], q1);
+      }
+      p[j][0] = q0;
+      p[j][1] = q1;
+    }
+  } else if constexpr (SIG == SIG_STAR) {
+    double t0 = 0.0, t1 = 0.0;
+#pragma unroll
+    for (int b = -R; b <= R; ++b) {
+      t0 = fma(P.v[0][R + b], x[R + b], t0);
+      t1 = fma(P.v[0][R + b], x[R + b + 1], t1);
+    }
+#pragma unroll
+    for (int j = 0; j <= 2 * R; ++j) {
+      const int a = R - j;
+      double q0 = j < 2 * R ? p[j + 1][0] : 0.0, q1 = j < 2 * R ? p[j + 1][1] : 0.0;
+      if (a == 0) {
+        q0 += t0;
+        q1 += t1;
+      }
+      p[j][0] = fma(P.u[1][R + a], x[R], q0);
+      p[j][1] = fma(P.u[1][R + a], x[R + 1], q1);
+    }
+  } else {
+    static_assert(SIG == SIG_ROWS || SIG == SIG_PMA || SIG == SIG_STAR, "row_shift: fused signatures only");
+  }
+}
+
 // ---------------------------------------------------------------------------------------------
 // Exact temporal fusion (§IV-A; reading Q5): K time steps per HBM
 // round trip.  Stage 1 consumes the staged input rows; every completed step-s row is written to a
@@ -252,31 +346,49 @@ __device__ __forceinline__ void store_pairs(double* o, const double (&v)[NH][2],
 // FULL: every row of the stage is interior for every intermediate step, every final row is stored
 // and every lane stores a 16-byte pair (decided per stage, warp-uniform): no per-row checks.
 // PRE: stage S's input row is already in xq (the prefetched stage-1 row); stages S down to SMIN run.
-template <int R, int SIG, int K, int NH, bool FULL, int I0, int I, int S, bool PRE = false, int SMIN = 1>
+// LOOP: runtime row loop (row index Ir, shift-register row update row_shift) instead of the ring
+// form unrolled over the 2R + 1 ring positions (template row index I, ring position I0).
+template <int R, int SIG, int K, int NH, bool FULL, int I0, int I_, int S, bool PRE = false, int SMIN = 1, bool LOOP = false>
 __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, int p,
                                            double (&acc)[K][NH][2 * R + 1][2], const RdgParams& P,
                                            double* __restrict__ bufs, int par, const double* __restrict__ in,
                                            double* __restrict__ out, int64_t P1, const StageCtx<K>& sc,
                                            const LaneCtx<NH>& lc, const P2PArgs& dp,
-                                           const double (&xq)[NH][2 * R + 2]) {
+                                           const double (&xq)[NH][2 * R + 2], int Ir = 0) {
   static_assert(!PRE || SMIN == S, "a preloaded stage runs alone");
   constexpr int n = 2 * R + 1;
   constexpr int BUFD = Geom<R, NH>::BUFD;
+  const int I = LOOP ? Ir : I_;
   constexpr int Is = pmod(I0 - (S - 1) * (R + 1), n);   // ring index of stage S's input row (any per-stage constant)
   const double* src = S == 1 ? st_row : bufs + (2 * (S - 2) + (par ^ 1)) * BUFD;
-#pragma unroll
-  for (int h = 0; h < NH; ++h) {
-    if constexpr (PRE) row_compute<R, SIG, Is>(xq[h], acc[S - 1][h], P);
-    else row_body<R, SIG, Is>(src + 64 * h, p, acc[S - 1][h], P);
-  }
-  constexpr int cs = (Is + 1) % n;                // slot of the row this stage just completed
   double v[NH][2];
+  if constexpr (LOOP) {
 #pragma unroll
-  for (int h = 0; h < NH; ++h) {
-    v[h][0] = acc[S - 1][h][cs][0];
-    v[h][1] = acc[S - 1][h][cs][1];
-    acc[S - 1][h][cs][0] = 0.0;
-    acc[S - 1][h][cs][1] = 0.0;
+    for (int h = 0; h < NH; ++h) {
+      if constexpr (PRE) {
+        row_shift<R, SIG>(xq[h], acc[S - 1][h], P);
+      } else {
+        double x[2 * R + 2];
+        load_x<R>(src + 64 * h, p, x);
+        row_shift<R, SIG>(x, acc[S - 1][h], P);
+      }
+      v[h][0] = acc[S - 1][h][0][0];
+      v[h][1] = acc[S - 1][h][0][1];
+    }
+  } else {
+#pragma unroll
+    for (int h = 0; h < NH; ++h) {
+      if constexpr (PRE) row_compute<R, SIG, Is>(xq[h], acc[S - 1][h], P);
+      else row_body<R, SIG, Is>(src + 64 * h, p, acc[S - 1][h], P);
+    }
+    constexpr int cs = (Is + 1) % n;                // slot of the row this stage just completed
+#pragma unroll
+    for (int h = 0; h < NH; ++h) {
+      v[h][0] = acc[S - 1][h][cs][0];
+      v[h][1] = acc[S - 1][h][cs][1];
+      acc[S - 1][h][cs][0] = 0.0;
+      acc[S - 1][h][cs][1] = 0.0;
+    }
   }
   if constexpr (S < K) {
     // re-impose the fixed Dirichlet halo on the intermediate row (exact temporal blocking)
@@ -342,7 +454,8 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
       }
     }
   }
-  if constexpr (S > SMIN) fused_iter<R, SIG, K, NH, FULL, I0, I, S - 1, false, SMIN>(st_row, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq);
+  if constexpr (S > SMIN)
+    fused_iter<R, SIG, K, NH, FULL, I0, I_, S - 1, false, SMIN, LOOP>(st_row, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, Ir);
 }
 
 #ifndef RDG_PF
@@ -399,6 +512,48 @@ __device__ __forceinline__ void fused_rows(const double* __restrict__ st, int p,
     }
     if constexpr (K > 1) __syncwarp();
     fused_rows<R, SIG, K, NH, FULL, I + 1>(st, p, acc, P, bufs, in, out, P1, sc, lc, par0, dp, xq);
+  }
+}
+
+#ifndef RDG_LOOP
+#define RDG_LOOP 2   // runtime row loop + row_shift — 2: fused radius >= 3 rows / PMA kernels, 1: every
+#endif               // fused rows / PMA / star kernel, 0: never (ring form everywhere)
+// Measured (same box, short runs; tools/gpu_variants.sh): Box-2D49P k = 2 322 -> 327 GS/s (ncu:
+// no_instruction stalls 0.61 -> 0.14 per issue, 12 % more instructions), Box-2D9P k = 3 673 -> 655,
+// Star-2D13P k = 2 456 -> 418 (the ring form there also loads stage 2's row early, RDG_PF2).
+template <int R, int SIG, int K>
+constexpr bool rdg_loop() {
+  return K >= 2 && ((RDG_LOOP == 1 && (SIG == SIG_ROWS || SIG == SIG_PMA || SIG == SIG_STAR)) ||
+                    (RDG_LOOP == 2 && R >= 3 && (SIG == SIG_ROWS || SIG == SIG_PMA)));
+}
+
+// The rows of one staged tile as a runtime loop (one copy of the K x NH row code; see row_shift).
+template <int R, int SIG, int K, int NH, bool FULL>
+__device__ __forceinline__ void fused_rows_loop(const double* __restrict__ st, int p, double (&acc)[K][NH][2 * R + 1][2],
+                                                const RdgParams& P, double* __restrict__ bufs,
+                                                const double* __restrict__ in, double* __restrict__ out, int64_t P1,
+                                                const StageCtx<K>& sc, const LaneCtx<NH>& lc, int par0,
+                                                const P2PArgs& dp, double (&xq)[NH][2 * R + 2]) {
+  constexpr int BW = Geom<R, NH>::BW, SROWS = Geom<R, NH>::SROWS;
+  constexpr bool PF = RDG_PF > 0 && R >= RDG_PF;
+  if constexpr (PF) {
+#pragma unroll
+    for (int h = 0; h < NH; ++h) load_x<R>(st + 64 * h, p, xq[h]);
+  }
+#pragma unroll 1
+  for (int I = 0; I < SROWS; ++I) {
+    const int par = (par0 + I) & 1;
+    if constexpr (PF) {
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, 1, true, 1, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I);
+      if (I + 1 < SROWS) {
+#pragma unroll
+        for (int h = 0; h < NH; ++h) load_x<R>(st + (I + 1) * BW + 64 * h, p, xq[h]);
+      }
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 2, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I);
+    } else {
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 1, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I);
+    }
+    __syncwarp();
   }
 }
 
@@ -606,8 +761,13 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
 #pragma unroll
     for (int S = 1; S < K; ++S) full = full && sc.hlo[S - 1] <= 0 && sc.hhi[S - 1] >= G::SROWS;
     double xq[NH][2 * R + 2];   // prefetched stage-1 input row (RDG_PF)
-    if (rdg_full<R, SIG, K>() && full) fused_rows<R, SIG, K, NH, true, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
-    else fused_rows<R, SIG, K, NH, false, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
+    if constexpr (rdg_loop<R, SIG, K>()) {
+      if (rdg_full<R, SIG, K>() && full) fused_rows_loop<R, SIG, K, NH, true>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
+      else fused_rows_loop<R, SIG, K, NH, false>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
+    } else {
+      if (rdg_full<R, SIG, K>() && full) fused_rows<R, SIG, K, NH, true, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
+      else fused_rows<R, SIG, K, NH, false, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
+    }
     __syncwarp();  // every lane is done with this slot before it is refilled
     if (++slot == RDG_NS) { slot = 0; phase ^= 1; }
     if (++cj == SI) {
