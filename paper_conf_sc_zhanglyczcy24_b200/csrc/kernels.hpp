@@ -7,6 +7,19 @@
 
 namespace lora {
 
+// Radius-1 PMA plane factors (palindromic 3-tap u, v) rescaled so that the centre tap of v is
+// exactly 1: v' = v / v[1], u' = u * v[1] (u' v'^T = u v^T up to one rounding per factor).  The 3D
+// CUDA-core kernels then form the horizontal gather as T = x_0 + v'[0] (x_-1 + x_+1), one DADD and
+// one DFMA instead of a DADD, a DMUL and a DFMA.  Both 3D kernels (unfused and fused) use the same
+// rescaled factors, so their per-point arithmetic stays identical.  Returns false if v[1] == 0.
+inline bool pma1_unit_centre(const double* u, const double* v, double* uo, double* vo) {
+  if (v[1] == 0.0) return false;
+  const double c = v[1];
+  for (int i = 0; i < 3; ++i) { uo[i] = u[i] * c; vo[i] = v[i] / c; }
+  vo[1] = 1.0;
+  return true;
+}
+
 // Device-initiated halo exchange (csrc/dist_p2p.cu): the slab's boundary work items
 // store their edge rows/planes straight into the neighbour's halo over peer memory (NVLink P2P /
 // CUDA IPC) and publish a per-unit step counter there; the neighbour's boundary items wait on it

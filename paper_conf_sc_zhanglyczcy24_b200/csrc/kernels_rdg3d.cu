@@ -112,7 +112,8 @@ __device__ __forceinline__ void apply_plane(const double (&x)[BY<R> + 2 * R][2 *
     }
   } else if (mode == PM_PMA1) {
     // radius-1 radially symmetric plane (PMA, eq. 15): one 3x3 rank-1 chain + the centre scalar;
-    // palindromic factors: T = v0 x0 + v1 (x_-1 + x_+1)
+    // palindromic factors with the centre tap of v rescaled to 1 (pma1_unit_centre):
+    // T = x0 + v1 (x_-1 + x_+1)
 #pragma unroll
     for (int y = 0; y < BY<R>; ++y) {
       d[y][0] = P.w[A0] * x[y + R][R];
@@ -121,8 +122,8 @@ __device__ __forceinline__ void apply_plane(const double (&x)[BY<R> + 2 * R][2 *
     double T[BY<R> + 2 * R][2];
 #pragma unroll
     for (int r = 0; r < BY<R> + 2 * R; ++r) {
-      T[r][0] = fma(P.v[A0][0][R + 1], x[r][R - 1] + x[r][R + 1], P.v[A0][0][R] * x[r][R]);
-      T[r][1] = fma(P.v[A0][0][R + 1], x[r][R] + x[r][R + 2], P.v[A0][0][R] * x[r][R + 1]);
+      T[r][0] = fma(P.v[A0][0][R + 1], x[r][R - 1] + x[r][R + 1], x[r][R]);
+      T[r][1] = fma(P.v[A0][0][R + 1], x[r][R] + x[r][R + 2], x[r][R + 1]);
     }
 #pragma unroll
     for (int y = 0; y < BY<R>; ++y) {
@@ -398,10 +399,11 @@ bool make_params3(const Plan& p, R3Params& prm, bool direct = false) {
     }
     if (R == 1 && ts.size() == 2 && ts[0]->kind == kChain && ts[0]->r == 1 && ts[1]->kind == kPoint &&
         ts[1]->r == 0 && ts[1]->u[R] == 1.0 && ts[0]->u[0] == ts[0]->u[2] && ts[0]->v[0] == ts[0]->v[2]) {
-      prm.mode[a0] = PM_PMA1;  // palindromic chain + centre scalar
-      for (int i = 0; i < n; ++i) { prm.u[a0][0][i] = ts[0]->u[i]; prm.v[a0][0][i] = ts[0]->v[i]; }
-      prm.w[a0] = ts[1]->v[R];
-      continue;
+      if (pma1_unit_centre(ts[0]->u, ts[0]->v, prm.u[a0][0], prm.v[a0][0])) {
+        prm.mode[a0] = PM_PMA1;  // palindromic chain (centre tap of v rescaled to 1) + centre scalar
+        prm.w[a0] = ts[1]->v[R];
+        continue;
+      }
     }
     if ((int)ts.size() > R3_MAXK) return false;
     prm.mode[a0] = PM_CHAINS;

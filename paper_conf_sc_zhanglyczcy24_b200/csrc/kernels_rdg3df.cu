@@ -73,11 +73,12 @@ __device__ __forceinline__ bool plane2(const double (&x)[4][4], const FParams& P
       d[y][0] = t0; d[y][1] = t1;
     }
   } else if (mode == PM_PMA1) {
+    // factors with v[1] == 1 (pma1_unit_centre): T = x_0 + v[2] (x_-1 + x_+1)
     double T[4][2];
 #pragma unroll
     for (int r = 0; r < 4; ++r) {
-      T[r][0] = fma(P.v[A0][0][2], x[r][0] + x[r][2], P.v[A0][0][1] * x[r][1]);
-      T[r][1] = fma(P.v[A0][0][2], x[r][1] + x[r][3], P.v[A0][0][1] * x[r][2]);
+      T[r][0] = fma(P.v[A0][0][2], x[r][0] + x[r][2], x[r][1]);
+      T[r][1] = fma(P.v[A0][0][2], x[r][1] + x[r][3], x[r][2]);
     }
 #pragma unroll
     for (int y = 0; y < 2; ++y) {
@@ -374,10 +375,11 @@ bool make_fparams(const Plan& p, FParams& prm) {
     }
     if (ts.size() == 2 && ts[0]->kind == kChain && ts[0]->r == 1 && ts[1]->kind == kPoint && ts[1]->r == 0 &&
         ts[1]->u[R] == 1.0 && ts[0]->u[0] == ts[0]->u[2] && ts[0]->v[0] == ts[0]->v[2]) {
-      prm.mode[a0] = PM_PMA1;
-      for (int i = 0; i < n; ++i) { prm.u[a0][0][i] = ts[0]->u[i]; prm.v[a0][0][i] = ts[0]->v[i]; }
-      prm.w[a0] = ts[1]->v[R];
-      continue;
+      if (pma1_unit_centre(ts[0]->u, ts[0]->v, prm.u[a0][0], prm.v[a0][0])) {
+        prm.mode[a0] = PM_PMA1;
+        prm.w[a0] = ts[1]->v[R];
+        continue;
+      }
     }
     if ((int)ts.size() > F_MAXK) return false;
     prm.mode[a0] = PM_CHAINS;
