@@ -102,7 +102,7 @@ __device__ __forceinline__ void row_compute(const double (&x)[2 * R + 2], double
 #pragma unroll
     for (int k = 0; k < R; ++k) {
       const int H = R - k;
-      double t0 = P.v[k][R] * x[R], t1 = P.v[k][R] * x[R + 1];
+      double t0 = x[R], t1 = x[R + 1];   // v_k[R] == 1 (signature() rescales the PMA factors)
 #pragma unroll
       for (int b = 1; b <= H; ++b) {
         t0 = fma(P.v[k][R + b], sp0[b], t0);
@@ -244,7 +244,7 @@ __device__ __forceinline__ void row_shift(const double (&x)[2 * R + 2], double (
 #pragma unroll
     for (int k = 0; k < R; ++k) {
       const int H = R - k;
-      double t0 = P.v[k][R] * x[R], t1 = P.v[k][R] * x[R + 1];
+      double t0 = x[R], t1 = x[R + 1];   // v_k[R] == 1 (signature() rescales the PMA factors)
 #pragma unroll
       for (int b = 1; b <= H; ++b) {
         t0 = fma(P.v[k][R + b], sp0[b], t0);
@@ -792,10 +792,16 @@ int signature(const Plan& p, RdgParams& prm) {
   bool pma = (int)p.terms.size() == R + 1;
   for (int k = 0; pma && k < R; ++k) pma = p.terms[k].kind == kChain && p.terms[k].r == R - k;
   if (pma) pma = p.terms[R].kind == kPoint && p.terms[R].u[R] == 1.0 && p.terms[R].r == 0;
+  for (int k = 0; pma && k < R; ++k) pma = p.terms[k].v[R] != 0.0;
   if (pma) {
+    // each chain rescaled so that the centre tap of v is exactly 1 (v' = v / v[R], u' = u v[R]):
+    // the horizontal gather starts from x_0 itself, one DMUL less per term and element
     prm.K = R;
-    for (int k = 0; k < R; ++k)
-      for (int i = 0; i < n; ++i) { prm.u[k][i] = p.terms[k].u[i]; prm.v[k][i] = p.terms[k].v[i]; }
+    for (int k = 0; k < R; ++k) {
+      const double c = p.terms[k].v[R];
+      for (int i = 0; i < n; ++i) { prm.u[k][i] = p.terms[k].u[i] * c; prm.v[k][i] = p.terms[k].v[i] / c; }
+      prm.v[k][R] = 1.0;
+    }
     prm.c = p.terms[R].v[R];
     return SIG_PMA;
   }
