@@ -196,7 +196,7 @@ double cuda_fma_per_point(const Plan& p) {
     (void)pma_like;
     if (p.ndim == 3 && cnt > 0 && !(cnt == 1) && !(cnt == 2 && all_arms)) {
       bool pma1 = p.R == 1 && cnt == 2;
-      f = pma1 ? 3.0 * 1.5 + 3.0 + 1.0 : cnt * 2.0 * n;  // PM_PMA1 (BY = 4: 6 T rows per 4 outputs) / general
+      f = pma1 ? 2.0 * 1.5 + 3.0 + 1.0 : cnt * 2.0 * n;  // PM_PMA1 (unit centre tap: T = 1 DADD + 1 DFMA; BY = 4: 6 T rows per 4 outputs) / general
     }
     return f;
   };
@@ -204,13 +204,14 @@ double cuda_fma_per_point(const Plan& p) {
     const int R = p.R;
     if (p.rdg_rows) return R + (R + 1) * (R + 1) + 2 * R;   // SIG_ROWS (kernels_rdg.cu; the fresh ring slot is assigned)
     // PMA pyramid (SIG_PMA): R shared tap-pair sums, then per chain of radius H a palindromic
-    // horizontal gather (H+1) and a vertical scatter (2H+1), plus the scalar C_{h+1}
+    // horizontal gather (H: the chain is rescaled to a unit centre tap of v, kernels_rdg.cu
+    // signature()) and a vertical scatter (2H+1), plus the scalar C_{h+1}
     bool pma = (int)p.terms.size() == R + 1;
     for (int k = 0; pma && k < R; ++k) pma = p.terms[k].kind == kChain && p.terms[k].r == R - k;
     if (pma) pma = p.terms[R].kind == kPoint && p.terms[R].r == 0;
     if (pma) {
       double f = R + 1;
-      for (int k = 0; k < R; ++k) f += (R - k + 1) + (2 * (R - k) + 1);
+      for (int k = 0; k < R; ++k) f += (R - k) + (2 * (R - k) + 1);
       return f;
     }
     return plane_cost(0);
@@ -316,7 +317,10 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
     if (rows) {  // only where it issues less than the planner's own factors (not for star arms)
       const double f_terms = cuda_fma_per_point(p);
       p.rdg_rows = 1;
-      if (cuda_fma_per_point(p) >= f_terms) p.rdg_rows = 0;
+      // a tie goes to the row pairs: their vertical gather is DADDs, which the FP64 pipe sustains at
+      // its full rate, the PMA scatter DFMAs with three register operands (~75 %,
+      // tools/ubench/fp64_operands.cu) — Box-2D49P: 25 vs 25
+      if (cuda_fma_per_point(p) > f_terms) p.rdg_rows = 0;
     }
   }
   p.fma_direct = nnz;
