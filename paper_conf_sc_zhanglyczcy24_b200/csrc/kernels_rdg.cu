@@ -326,10 +326,16 @@ struct LaneCtx {
 
 // Stores the lane's column pairs of one row: a 16-byte store where the pair is valid and aligned,
 // else predicated 8-byte stores (array edges, band-overlap lanes of fused bands store nothing).
-template <int NH>
+// ODD (odd R): lane pairs start on odd columns, never 16-byte aligned (no vector-store code).
+template <int NH, bool ODD = false>
 __device__ __forceinline__ void store_pairs(double* o, const double (&v)[NH][2], const LaneCtx<NH>& lc) {
 #pragma unroll
   for (int h = 0; h < NH; ++h) {
+    if constexpr (ODD) {
+      if (lc.valid[h][0]) o[64 * h] = v[h][0];
+      if (lc.valid[h][1]) o[64 * h + 1] = v[h][1];
+      continue;
+    }
     const bool p0 = !lc.vec[h] && lc.valid[h][0], p1 = !lc.vec[h] && lc.valid[h][1];
     if (lc.vec[h]) *reinterpret_cast<double2*>(o + 64 * h) = make_double2(v[h][0], v[h][1]);
     if (p0) o[64 * h] = v[h][0];
@@ -354,7 +360,8 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
                                            double* __restrict__ bufs, int par, const double* __restrict__ in,
                                            double* __restrict__ out, int64_t P1, const StageCtx<K>& sc,
                                            const LaneCtx<NH>& lc, const P2PArgs& dp,
-                                           const double (&xq)[NH][2 * R + 2], int Ir = 0) {
+                                           const double (&xq)[NH][2 * R + 2], int Ir = 0,
+                                           double* __restrict__ orow = nullptr) {
   static_assert(!PRE || SMIN == S, "a preloaded stage runs alone");
   constexpr int n = 2 * R + 1;
   constexpr int BUFD = Geom<R, NH>::BUFD;
@@ -428,12 +435,17 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
     }
   } else {
     if (I >= sc.lo && I < sc.hi) {
-      const int64_t e = sc.ooff + int64_t(I) * P1;
       if constexpr (K > 1) {
-        store_pairs<NH>(out + e, v, lc);
-        if (I < sc.rem_lo) store_pairs<NH>(dp.dst_lo + (e + dp.off_lo), v, lc);   // warp-uniform, rare
-        if (I >= sc.rem_hi) store_pairs<NH>(dp.dst_hi + (e + dp.off_hi), v, lc);
+        // LOOP: orow is this row's output pointer, advanced by the loop (no 64-bit index per row)
+        double* o = LOOP ? orow : out + (sc.ooff + int64_t(I) * P1);
+        store_pairs<NH, (R & 1) != 0>(o, v, lc);
+        if (I < sc.rem_lo || I >= sc.rem_hi) {   // warp-uniform, rare
+          const int64_t e = sc.ooff + int64_t(I) * P1;
+          if (I < sc.rem_lo) store_pairs<NH>(dp.dst_lo + (e + dp.off_lo), v, lc);
+          if (I >= sc.rem_hi) store_pairs<NH>(dp.dst_hi + (e + dp.off_hi), v, lc);
+        }
       } else {
+        const int64_t e = sc.ooff + int64_t(I) * P1;
         // the row goes to this slab and, for the first / last R interior rows of a slab with a
         // neighbour there, into that neighbour's halo as well (peer memory, csrc/dist_p2p.cu;
         // the device-initiated exchange runs unfused).  This form measured faster for K = 1
@@ -455,7 +467,8 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
     }
   }
   if constexpr (S > SMIN)
-    fused_iter<R, SIG, K, NH, FULL, I0, I_, S - 1, false, SMIN, LOOP>(st_row, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, Ir);
+    fused_iter<R, SIG, K, NH, FULL, I0, I_, S - 1, false, SMIN, LOOP>(st_row, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, Ir,
+                                                                      orow);
 }
 
 #ifndef RDG_PF
@@ -540,18 +553,22 @@ __device__ __forceinline__ void fused_rows_loop(const double* __restrict__ st, i
 #pragma unroll
     for (int h = 0; h < NH; ++h) load_x<R>(st + 64 * h, p, xq[h]);
   }
+  double* orow = out + sc.ooff;   // output row of the final stage for I = 0 (only dereferenced when stored)
 #pragma unroll 1
-  for (int I = 0; I < SROWS; ++I) {
+  for (int I = 0; I < SROWS; ++I, orow += P1) {
     const int par = (par0 + I) & 1;
     if constexpr (PF) {
-      fused_iter<R, SIG, K, NH, FULL, 0, 0, 1, true, 1, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I);
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, 1, true, 1, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
+                                                              orow);
       if (I + 1 < SROWS) {
 #pragma unroll
         for (int h = 0; h < NH; ++h) load_x<R>(st + (I + 1) * BW + 64 * h, p, xq[h]);
       }
-      fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 2, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I);
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 2, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
+                                                               orow);
     } else {
-      fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 1, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I);
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 1, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
+                                                               orow);
     }
     __syncwarp();
   }
