@@ -30,7 +30,11 @@ namespace {
 #ifndef RDG_RC_ROWS
 #define RDG_RC_ROWS 128   // experiments: chunk length
 #endif
-constexpr int RDG_RC = RDG_RC_ROWS;   // output rows per work item (chunk)
+constexpr int RDG_RC = RDG_RC_ROWS;
+#ifndef RDG_LOOP_UNROLL
+#define RDG_LOOP_UNROLL 2   // unroll factor of the fused row loop (Box-2D49P k=2: 1: 337, 2: 347, 3: 251, 4: 283, 7: 326 GS/s)
+#endif
+constexpr int kRowUnroll = RDG_LOOP_UNROLL;   // (#pragma arguments are not macro-expanded)   // output rows per work item (chunk)
 constexpr int RDG_WARPS = 4;    // warps per CTA (independent streams)
 constexpr int RDG_NS = 3;       // ring stages per warp (3 keeps 4 CTAs = 16 warps per SM)
 
@@ -554,7 +558,7 @@ __device__ __forceinline__ void fused_rows_loop(const double* __restrict__ st, i
     for (int h = 0; h < NH; ++h) load_x<R>(st + 64 * h, p, xq[h]);
   }
   double* orow = out + sc.ooff;   // output row of the final stage for I = 0 (only dereferenced when stored)
-#pragma unroll 1
+#pragma unroll kRowUnroll
   for (int I = 0; I < SROWS; ++I, orow += P1) {
     const int par = (par0 + I) & 1;
     if constexpr (PF) {
