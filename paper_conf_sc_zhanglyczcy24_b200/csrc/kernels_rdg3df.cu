@@ -120,6 +120,10 @@ __device__ __forceinline__ bool plane2(const double (&x)[4][4], const FParams& P
 template <int M0, int M1, int MIR>
 struct Sig3 {
   static constexpr int m0 = M0, m1 = M1, mir = MIR;
+  // plane 0 statically non-empty and its result an FMA chain: its contribution assigns (a bare
+  // product, PM_POINT, would let nvcc contract it with the next addition into one FMA, which the
+  // unfused kernel's 0 + w x does not: results would differ from two single steps in the last bit)
+  static constexpr bool assign0 = M0 > 0 && M0 != 1 /* PM_POINT */;
 };
 
 // All plane operators of one input plane (ring position I) into a z-ring of 3 planes x 2 rows.
@@ -132,8 +136,15 @@ __device__ __forceinline__ void planes2(const double (&x)[4][4], const FParams& 
       double d[2][2];
       if (plane2<A0, MODE>(x, P, d)) {
         constexpr int s1 = pm3(I - A0);
+        if constexpr (A0 == 0 && SG::assign0) {
+          // plane 0's contribution is the first one its output plane receives (the slot was
+          // emitted after input plane I - 1): assigned, so emitted slots need no zeroing
 #pragma unroll
-        for (int y = 0; y < 2; ++y) { acc[s1][y][0] += d[y][0]; acc[s1][y][1] += d[y][1]; }
+          for (int y = 0; y < 2; ++y) { acc[s1][y][0] = d[y][0]; acc[s1][y][1] = d[y][1]; }
+        } else {
+#pragma unroll
+          for (int y = 0; y < 2; ++y) { acc[s1][y][0] += d[y][0]; acc[s1][y][1] += d[y][1]; }
+        }
         if (A0 == 0 && mirror) {
           constexpr int s2 = pm3(I - 2);
 #pragma unroll
@@ -158,7 +169,8 @@ __device__ __forceinline__ void load_rows(const double* __restrict__ base, int p
 // gets the fixed Dirichlet halo re-imposed and is published to its shared plane buffer.
 // fast: every element of the lane is strictly inside the array in x, y (precomputed per item) and
 // z (per plane) — no halo value to re-impose, no zero fill: plain stores.
-template <int K, int S, int CS>
+// ZERO: clear the emitted slot (not needed when plane 0's contribution assigns, Sig3::assign0).
+template <int K, int S, int CS, bool ZERO = true>
 __device__ __forceinline__ void publish(double (&acc)[K][3][2][2], double* __restrict__ buf, int w, int lane,
                                         int Y0, int X0, int zs, int P0, int P1, int P2,
                                         const double* __restrict__ in, bool fast) {
@@ -169,7 +181,7 @@ __device__ __forceinline__ void publish(double (&acc)[K][3][2][2], double* __res
 #pragma unroll
       for (int e = 0; e < 2; ++e) {
         buf[(2 * w + y) * F_S1W + 1 + c0 + e] = acc[S - 1][CS][y][e];
-        acc[S - 1][CS][y][e] = 0.0;
+        if constexpr (ZERO) acc[S - 1][CS][y][e] = 0.0;
       }
     }
     return;
@@ -177,7 +189,7 @@ __device__ __forceinline__ void publish(double (&acc)[K][3][2][2], double* __res
 #pragma unroll
   for (int y = 0; y < 2; ++y) {
     double v[2] = {acc[S - 1][CS][y][0], acc[S - 1][CS][y][1]};
-    acc[S - 1][CS][y][0] = 0.0; acc[S - 1][CS][y][1] = 0.0;
+    if constexpr (ZERO) { acc[S - 1][CS][y][0] = 0.0; acc[S - 1][CS][y][1] = 0.0; }
     const int gy = Y0 - (K - S) + 2 * w + y;  // padded row of this stage-S row
     const bool zin = zs >= 0 && zs < P0, yin = gy >= 0 && gy < P1;
     const bool zh = zs < 1 || zs >= P0 - 1, yh = gy < 1 || gy >= P1 - 1;
@@ -306,7 +318,7 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
         double x[4][4];
         load_rows(st + (2 * w) * F_BW, F_BW, lane, x);
         planes2<SG, I, 0>(x, prm, acc[0]);
-        publish<K, 1, (I + 1) % 3>(acc, sbuf + (0 * 2 + par) * S1B, w, lane, Y0, X0, p - 1, P0, P1, P2, in,
+        publish<K, 1, (I + 1) % 3, !SG::assign0>(acc, sbuf + (0 * 2 + par) * S1B, w, lane, Y0, X0, p - 1, P0, P1, P2, in,
                                    xy_in[0] && p - 1 >= 1 && p - 1 < P0 - 1);
       }
       __syncthreads();  // stage-1 plane visible; every warp is done with the input slot
@@ -323,7 +335,7 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
           planes2<SG, IS, 0>(x, prm, acc[S - 1]);
         }
         if constexpr (S < K) {
-          if (active) publish<K, S, (IS + 1) % 3>(acc, sbuf + ((S - 1) * 2 + par) * S1B, w, lane, Y0, X0, p - S, P0, P1,
+          if (active) publish<K, S, (IS + 1) % 3, !SG::assign0>(acc, sbuf + ((S - 1) * 2 + par) * S1B, w, lane, Y0, X0, p - S, P0, P1,
                                                   P2, in, xy_in[S - 1] && p - S >= 1 && p - S < P0 - 1);
           __syncthreads();
         } else if (active) {
@@ -338,8 +350,10 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
               for (int e = 0; e < 2; ++e)
                 if (st_ok[y][e]) o[y * P2 + e] = acc[K - 1][s][y][e];
           }
+          if constexpr (!SG::assign0) {
 #pragma unroll
-          for (int y = 0; y < 2; ++y) { acc[K - 1][s][y][0] = 0.0; acc[K - 1][s][y][1] = 0.0; }
+            for (int y = 0; y < 2; ++y) { acc[K - 1][s][y][0] = 0.0; acc[K - 1][s][y][1] = 0.0; }
+          }
         }
       };
       [&]<int... Ss>(std::integer_sequence<int, Ss...>) {
