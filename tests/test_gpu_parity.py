@@ -366,3 +366,49 @@ def test_identity_shift_zero_weights(engine, d):
     ref = g.copy()
     ref[tuple(slice(1, -1) for _ in range(d))] = 0.0
     assert np.array_equal(out, ref)
+
+
+def _zero_centre_tap_2d(h):
+    """Reflection-symmetric 2D W whose PMA chain factor v has a zero centre tap (the centre column
+    of W vanishes outside the centre): the unit-centre rescaling of the CUDA-core engine cannot apply
+    (kernels_rdg.cu signature() falls back to the general rank-1 form)."""
+    n = 2 * h + 1
+    W = np.zeros((n, n))
+    for a in range(n):
+        for b in range(n):
+            if b != h and a != h:
+                W[a, b] = 1.0 + 0.25 * (abs(a - h) + 2 * abs(b - h))
+    W[h, h] = 2.0
+    return W / W.sum()
+
+
+@pytest.mark.parametrize("h", [1, 2])
+def test_zero_centre_tap_fallback_2d(h):
+    """PMA factors with v[R] == 0 (no unit-centre rescaling possible) still match the oracle, on
+    every engine and at the planner's default fusion depth."""
+    W = _zero_centre_tap_2d(h)
+    g = synth.grid((67 + 2 * h, 129 + 2 * h), 5)
+    ref = oracle.run(W, g, 4)
+    for eng in ("auto", "rdg_cuda", "tc", "direct"):
+        out, _ = run_gpu(W, g, 4, engine=eng)
+        assert rel_err(out, ref) <= 1e-12, eng
+
+
+def test_zero_centre_tap_fallback_3d():
+    """Radius-1 3D W whose planes have zero edge taps (PMA v[1] == 0): pma1_unit_centre declines and
+    both 3D CUDA-core kernels take the general chain mode; fused == unfused bitwise, both match the
+    oracle."""
+    W = np.zeros((3, 3, 3))
+    for z in range(3):
+        for y in range(3):
+            for x in range(3):
+                if (y == 1) == (x == 1):   # corners and centre of each plane
+                    W[z, y, x] = 1.0 + 0.5 * abs(z - 1) + 0.25 * (y != 1)
+    W /= W.sum()
+    g = synth.grid((17 + 2, 9 + 2, 33 + 2), 8)
+    ref = oracle.run(W, g, 3)
+    a, _ = run_gpu(W, g, 3, engine="rdg_cuda", fuse_k=1)
+    b, info = run_gpu(W, g, 3, engine="rdg_cuda", fuse_k=2)
+    assert info["fuse_k"] == 2
+    assert np.array_equal(a, b)
+    assert rel_err(a, ref) <= 1e-12
