@@ -28,7 +28,10 @@
 namespace lora {
 namespace {
 
-constexpr int F_NS = 3;              // TMA ring stages
+#ifndef RDG3F_NS
+#define RDG3F_NS 3
+#endif
+constexpr int F_NS = RDG3F_NS;       // TMA ring stages
 constexpr int F_WARPS = 8;
 constexpr int F_S1 = 16;             // stage-1 rows per CTA column (2 per warp); stage s: 16 - 2(s-1)
 constexpr int F_IN = 18;             // staged input rows
