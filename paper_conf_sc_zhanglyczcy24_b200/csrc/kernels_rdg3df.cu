@@ -29,9 +29,8 @@ namespace lora {
 namespace {
 
 #ifndef RDG3F_NS
-#define RDG3F_NS 3
+#define RDG3F_NS 0   // TMA ring stages; 0: per signature (f_ns)
 #endif
-constexpr int F_NS = RDG3F_NS;       // TMA ring stages
 constexpr int F_WARPS = 8;
 constexpr int F_S1 = 16;             // stage-1 rows per CTA column (2 per warp); stage s: 16 - 2(s-1)
 constexpr int F_IN = 18;             // staged input rows
@@ -123,6 +122,9 @@ __device__ __forceinline__ bool plane2(const double (&x)[4][4], const FParams& P
 template <int M0, int M1, int MIR>
 struct Sig3 {
   static constexpr int m0 = M0, m1 = M1, mir = MIR;
+  // TMA ring stages: 4 for the light point + star (Heat-3D) kernel (420 -> 430 GS/s), 3 otherwise
+  // (Box-3D27P: 392 with 3, 388 with 4; tools/gpu_variants.sh, same box)
+  static constexpr int ns = RDG3F_NS > 0 ? RDG3F_NS : ((M0 == 1 && M1 == 3) ? 4 : 3);
   // plane 0 statically non-empty and its result an FMA chain: its contribution assigns (a bare
   // product, PM_POINT, would let nvcc contract it with the next addition into one FMA, which the
   // unfused kernel's 0 + w x does not: results would differ from two single steps in the last bit)
@@ -220,6 +222,7 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
                                                                  const __grid_constant__ CUtensorMap tmap,
                                                                  const __grid_constant__ FParams prm) {
   constexpr int STAGE = ((F_IN * F_BW * 8 + 127) / 128) * 128;
+  constexpr int F_NS = SG::ns;
   constexpr int S1B = F_S1 * F_S1W;          // doubles per intermediate plane buffer
   constexpr int TY = F_S1 - 2 * (K - 1);     // final rows per CTA column
   constexpr int SG1 = (K - 1) & 1;           // keeps the staged x origin even
@@ -415,7 +418,7 @@ template <class SG, int K, bool TMA>
 cudaError_t launch_f(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
                      const FParams& prm) {
   constexpr int STAGE = ((F_IN * F_BW * 8 + 127) / 128) * 128;
-  const int smem = 128 + F_NS * STAGE + 2 * (K - 1) * F_S1 * F_S1W * 8;
+  const int smem = 128 + SG::ns * STAGE + 2 * (K - 1) * F_S1 * F_S1W * 8;
   static int max_grid = 0;
   if (max_grid == 0) {
     cudaError_t e = cudaFuncSetAttribute(rdg3df_kernel<SG, K, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
