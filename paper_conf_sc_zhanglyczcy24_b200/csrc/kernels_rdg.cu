@@ -36,7 +36,10 @@ constexpr int RDG_RC = RDG_RC_ROWS;
 #endif
 constexpr int kRowUnroll = RDG_LOOP_UNROLL;   // (#pragma arguments are not macro-expanded)   // output rows per work item (chunk)
 constexpr int RDG_WARPS = 4;    // warps per CTA (independent streams)
-constexpr int RDG_NS = 3;       // ring stages per warp (3 keeps 4 CTAs = 16 warps per SM)
+#ifndef RDG_NS_STAGES
+#define RDG_NS_STAGES 3
+#endif
+constexpr int RDG_NS = RDG_NS_STAGES;   // ring stages per warp (3 keeps 4 CTAs = 16 warps per SM)
 
 enum { SIG_PMA = 0, SIG_STAR = 1, SIG_FULL = 2, SIG_DIRECT = 3, SIG_ROWS = 4 };   // DIRECT: W itself in u[][] (K11)
 
