@@ -31,6 +31,9 @@ namespace {
 #define RDG_RC_ROWS 128   // experiments: chunk length
 #endif
 constexpr int RDG_RC = RDG_RC_ROWS;
+#ifndef RDG_UNIFORM_WL
+#define RDG_UNIFORM_WL 1
+#endif
 #ifndef RDG_LOOP_UNROLL
 #define RDG_LOOP_UNROLL 2   // unroll factor of the fused row loop (Box-2D49P k=2: 1: 337, 2: 347, 3: 251, 4: 283, 7: 326 GS/s)
 #endif
@@ -329,6 +332,7 @@ struct LaneCtx {
   int c0;                   // padded column of the lane's first column (may be < 0); half h adds 64h
   bool inside[NH][2], colhalo[NH][2], valid[NH][2], vec[NH];
   bool edge;                // some column of the lane is a column halo or outside the array
+  bool edge_any;            // ... of some lane of the warp (warp-uniform: a uniform branch)
 };
 
 // Stores the lane's column pairs of one row: a 16-byte store where the pair is valid and aligned,
@@ -414,7 +418,7 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
       for (int h = 0; h < NH; ++h)
 #pragma unroll
         for (int j = 0; j < 2; ++j) v[h][j] = (row_in && lc.inside[h][j]) ? ir[64 * h + j] : 0.0;
-    } else if (lc.edge) {
+    } else if (lc.edge_any) {   // per-lane tests inside (lanes without edge columns keep v)
       const double* ir = in + sc.ioff[S - 1] + int64_t(I) * P1 + lc.c0;
 #pragma unroll
       for (int h = 0; h < NH; ++h)
@@ -634,7 +638,10 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
   constexpr int BS = 64 * NH - 2 * R * (K - 1) - 2 * SG;  // band stride (valid final columns per band)
   constexpr int BUFD = G::BUFD;
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  // the warp index through a shuffle from lane 0: ptxas then knows it (and all item geometry derived
+  // from it) is warp-uniform — uniform branches and uniform-datapath address arithmetic
+  const int wl = RDG_UNIFORM_WL ? __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0) : (int)(threadIdx.x >> 5);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw) + wl * RDG_NS;
   unsigned char* wbase = smem_raw + 128 + wl * (G::WARP_BYTES + 2 * (K - 1) * BUFD * 8);
   unsigned char* ring = wbase;
@@ -754,6 +761,7 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
       // FULL lanes: no halo columns; a pair is stored as a whole or not at all — one 16-byte store
       // for even R; for odd R the lane columns X0 + 2p are odd (the staged origin X0 - R is kept
       // even for TMA), so the pair is two 8-byte stores
+      lc.edge_any = __any_sync(0xffffffffu, lc.edge);
       bool mine = !lc.edge;
 #pragma unroll
       for (int h = 0; h < NH; ++h)
