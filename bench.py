@@ -128,20 +128,24 @@ def ncu_traffic(workload, engine):
 
 def cpu_oracle_sample(W, cfg, budget_s=12.0):
     """The oracle as it stands, on all host cores, on a bounded sample of the workload: a band of
-    full-width rows (2D) or planes (3D) of the same grid, stepped T_s times (T_s sized to ~budget_s)."""
+    full-width rows (2D) or planes (3D) of the same grid, stepped the workload's T times; the band
+    height is sized from a one-step probe so that the sample takes about budget_s."""
     import oracle
     import synth
     h = cfg["radius"]
     shape = list(cfg["shape"])
-    shape[0] = min(shape[0], 256 if cfg["ndim"] == 2 else 16)
-    padded = tuple(n + 2 * h for n in shape)
-    g = synth.grid(padded, cfg["seed"])
-    t0 = time.perf_counter(); oracle.run(W, g, 1); t1 = time.perf_counter() - t0
-    Ts = int(max(1, min(cfg["T"], budget_s / max(t1, 1e-6))))
-    t0 = time.perf_counter(); oracle.run(W, g, Ts); dt = time.perf_counter() - t0
-    pts = float(np.prod(shape)) * Ts
+    probe = min(shape[0], 64 if cfg["ndim"] == 2 else 8)
+    pshape = [probe] + shape[1:]
+    g = synth.grid(tuple(n + 2 * h for n in pshape), cfg["seed"])
+    t0 = time.perf_counter(); oracle.run(W, g, 2); t1 = (time.perf_counter() - t0) / 2
+    T = cfg["T"]
+    rows = int(max(1, min(shape[0], probe * budget_s / max(t1 * T, 1e-9))))
+    shape[0] = rows
+    g = synth.grid(tuple(n + 2 * h for n in shape), cfg["seed"])
+    t0 = time.perf_counter(); oracle.run(W, g, T); dt = time.perf_counter() - t0
+    pts = float(np.prod(shape)) * T
     return {"value": pts / dt / 1e9, "unit": UNIT, "cores": oracle.max_threads(), "kind": "oracle",
-            "sample": f"{'x'.join(map(str, shape))} interior band of {cfg['name']}, {Ts} steps, {dt:.1f} s"}
+            "sample": f"{'x'.join(map(str, shape))} interior band of {cfg['name']}, {T} steps, {dt:.1f} s"}
 
 
 def host_info():
