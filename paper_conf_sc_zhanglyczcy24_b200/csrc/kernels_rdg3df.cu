@@ -172,11 +172,54 @@ __device__ __forceinline__ void load_rows(const double* __restrict__ base, int p
 
 // Intermediate stage S (1 <= S < K): the stage-S plane just completed in acc[S-1] (ring slot CS)
 // gets the fixed Dirichlet halo re-imposed and is published to its shared plane buffer.
-// fast: every element of the lane is strictly inside the array in x, y (precomputed per item) and
-// z (per plane) — no halo value to re-impose, no zero fill: plain stores.
 // ZERO: clear the emitted slot (not needed when plane 0's contribution assigns, Sig3::assign0).
+// The Dirichlet values a slow-path publish substitutes for the lane's 4 elements of the stage-S
+// row pair at plane zs: bit 2y+e of the result set = element replaced by hv[y][e] (the input's halo
+// value, or 0 outside the array).  Issued at the start of the plane so the global loads overlap the
+// plane's arithmetic instead of stalling the shared-memory stores of publish.
+template <int K, int S>
+__device__ __forceinline__ unsigned halo_fetch(int w, int lane, int Y0, int X0, int zs, int P0, int P1, int P2,
+                                               const double* __restrict__ in, double (&hv)[2][2]) {
+  const int c0 = 2 * lane;
+  unsigned m = 0;
+#pragma unroll
+  for (int y = 0; y < 2; ++y) {
+    const int gy = Y0 - (K - S) + 2 * w + y;  // padded row of this stage-S row
+    const bool zin = zs >= 0 && zs < P0, yin = gy >= 0 && gy < P1;
+    const bool zh = zs < 1 || zs >= P0 - 1, yh = gy < 1 || gy >= P1 - 1;
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {
+      const int cx = X0 + c0 + e;
+      const bool xin = cx >= 0 && cx < P2, xh = cx < 1 || cx >= P2 - 1;
+      const bool inside = zin && yin && xin, halo = inside && (zh || yh || xh);
+      hv[y][e] = halo ? in[(int64_t(zs) * P1 + gy) * P2 + cx] : 0.0;
+      if (!inside || halo) m |= 1u << (2 * y + e);
+    }
+  }
+  return m;
+}
+
+// fast: every element of the lane is strictly inside the array (hm == 0): plain stores; otherwise
+// the elements flagged in hm take the prefetched Dirichlet values hv (halo_fetch).
 template <int K, int S, int CS, bool ZERO = true>
 __device__ __forceinline__ void publish(double (&acc)[K][3][2][2], double* __restrict__ buf, int w, int lane,
+                                        unsigned hm, const double (&hv)[2][2]) {
+  const int c0 = 2 * lane;
+#pragma unroll
+  for (int y = 0; y < 2; ++y) {
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {
+      const double v = acc[S - 1][CS][y][e];
+      buf[(2 * w + y) * F_S1W + 1 + c0 + e] = ((hm >> (2 * y + e)) & 1u) ? hv[y][e] : v;
+      if constexpr (ZERO) acc[S - 1][CS][y][e] = 0.0;
+    }
+  }
+}
+
+// K = 3: the Dirichlet values are loaded in place (a prefetch would cost registers the K = 3
+// kernel does not have; fast: the lane's elements are strictly inside, plain stores).
+template <int K, int S, int CS, bool ZERO = true>
+__device__ __forceinline__ void publish_ip(double (&acc)[K][3][2][2], double* __restrict__ buf, int w, int lane,
                                         int Y0, int X0, int zs, int P0, int P1, int P2,
                                         const double* __restrict__ in, bool fast) {
   const int c0 = 2 * lane;
@@ -321,11 +364,20 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
       // ---------------- stage 1: rows 2w, 2w+1 (16 rows) from input tile rows 2w .. 2w+3
       {
         const double* st = reinterpret_cast<const double*>(ring + slot * STAGE);
+        // K = 2: the Dirichlet values are fetched before the plane's arithmetic (their latency hides
+        // behind it: Heat-3D 431 -> 452 GS/s); K = 3 has no registers to spare (spills), fetches late
+        const bool fast1 = xy_in[0] && p - 1 >= 1 && p - 1 < P0 - 1;
+        double hv[2][2];
+        unsigned hm = 0;
+        if (K == 2 && !fast1) hm = halo_fetch<K, 1>(w, lane, Y0, X0, p - 1, P0, P1, P2, in, hv);
         double x[4][4];
         load_rows(st + (2 * w) * F_BW, F_BW, lane, x);
         planes2<SG, I, 0>(x, prm, acc[0]);
-        publish<K, 1, (I + 1) % 3, !SG::assign0>(acc, sbuf + (0 * 2 + par) * S1B, w, lane, Y0, X0, p - 1, P0, P1, P2, in,
-                                   xy_in[0] && p - 1 >= 1 && p - 1 < P0 - 1);
+        if constexpr (K == 2)
+          publish<K, 1, (I + 1) % 3, !SG::assign0>(acc, sbuf + (0 * 2 + par) * S1B, w, lane, hm, hv);
+        else
+          publish_ip<K, 1, (I + 1) % 3, !SG::assign0>(acc, sbuf + (0 * 2 + par) * S1B, w, lane, Y0, X0, p - 1, P0, P1, P2, in,
+                                                      fast1);
       }
       __syncthreads();  // stage-1 plane visible; every warp is done with the input slot
       if (q + F_NS - 1 < nstages) issue_next((slot + F_NS - 1) % F_NS);
@@ -341,8 +393,9 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
           planes2<SG, IS, 0>(x, prm, acc[S - 1]);
         }
         if constexpr (S < K) {
-          if (active) publish<K, S, (IS + 1) % 3, !SG::assign0>(acc, sbuf + ((S - 1) * 2 + par) * S1B, w, lane, Y0, X0, p - S, P0, P1,
-                                                  P2, in, xy_in[S - 1] && p - S >= 1 && p - S < P0 - 1);
+          // (S < K only for K = 3: in-place Dirichlet loads)
+          if (active) publish_ip<K, S, (IS + 1) % 3, !SG::assign0>(acc, sbuf + ((S - 1) * 2 + par) * S1B, w, lane, Y0, X0, p - S,
+                                                                  P0, P1, P2, in, xy_in[S - 1] && p - S >= 1 && p - S < P0 - 1);
           __syncthreads();
         } else if (active) {
           // final plane zf = p - K complete: ring slot (IS + 1) % 3
