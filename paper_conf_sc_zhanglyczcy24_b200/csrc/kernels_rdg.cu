@@ -38,7 +38,10 @@ constexpr int RDG_RC = RDG_RC_ROWS;
 #define RDG_LOOP_UNROLL 2   // unroll factor of the fused row loop (Box-2D49P k=2: 1: 337, 2: 347, 3: 251, 4: 283, 7: 326 GS/s)
 #endif
 constexpr int kRowUnroll = RDG_LOOP_UNROLL;   // (#pragma arguments are not macro-expanded)   // output rows per work item (chunk)
-constexpr int RDG_WARPS = 4;    // warps per CTA (independent streams)
+#ifndef RDG_WARPS_PER_CTA
+#define RDG_WARPS_PER_CTA 4   // (Box-2D49P k=2: 2 warps 351, 4 warps 350, 8 warps 270 GS/s; Box-2D9P k=3: 654 / 692)
+#endif
+constexpr int RDG_WARPS = RDG_WARPS_PER_CTA;   // warps per CTA (independent streams)
 #ifndef RDG_NS_STAGES
 #define RDG_NS_STAGES 3
 #endif
