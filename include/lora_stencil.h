@@ -83,6 +83,23 @@ typedef struct {               /* filled by lora_stencil_plan_query             
   double fma_per_point_issued; /* FP64 FMAs issued per point per step by the chosen engine    */
   double fma_per_point_direct; /* (2r+1)^d, nonzero weights only                              */
   double fma_per_point_separable; /* sum over terms of (len u + len v) + point-wise terms      */
+  /* The paper's analytic cost model for its A100 tiling at the plan's radius h (host arithmetic on
+   * h only; reported so that the counts printed in the paper can be checked against the library):
+   *   P:225  grid points updated at once            32 ceil(h/2) ceil(h/4)
+   *   eq. 12 RDG fragment loads from shared memory  ab/8            -> per point 1/8
+   *   eq. 13 ConvStencil fragment loads             2 ceil((2h+1)^2/4) per 8(2h+2) points
+   *   eq. 14 ConvStencil / RDG                      ceil((2h+1)^2/4) / (h+1)   (3.25 at h=3, 4.2 at h=4)
+   *   eq. 16 LoRAStencil MMAs                       2h ceil(h/2) (2 ceil(h/4)+1) per 32 ceil(h/2) ceil(h/4) points
+   *                                                 (36 per 64 points at h=3; ConvStencil: eq. 13, 26)
+   *   P:340  FP64 fragment elements wasted by one 8x8 update (eight 4x8 fragments = 256 loaded,
+   *          (8+2h)^2 used): 256 - (8+2h)^2 (156 at h=1, 60 at h=3: fusing 3 Box-2D9P steps saves 96) */
+  int    paper_points_per_update;
+  double paper_rdg_frag_per_point;
+  double paper_convstencil_frag_per_point;
+  double paper_convstencil_over_rdg;
+  double paper_mma_per_point;
+  double paper_convstencil_mma_per_point;
+  int    paper_fragment_waste;
 } lora_plan_info;
 
 /* Plans a stencil.  Host-only work (no CUDA call): validates, factors every 2D plane
@@ -103,7 +120,10 @@ lora_plan* lora_stencil_plan_ex(const double* weights, int ndim, int radius, con
  * enable TMA staging).  `in` is never written; on return (stream-ordered) `out` holds step T
  * in its interior and a copy of `in`'s halo.  timesteps = 0 copies.  in/out must not overlap
  * (LORA_ERR_ALIAS).  `stream` is a cudaStream_t (NULL = legacy default stream).  The first
- * call allocates the plan's device scratch (one padded buffer) on the current device. */
+ * call allocates the plan's device scratch (one padded buffer) on the current device.
+ * Launch-bound problems (<= 4 Mi padded points, >= 4 launches, a non-default stream): the second
+ * identical call (same in, out, T, stream) captures the time loop as a CUDA graph and later identical
+ * calls replay it; a stream the caller is already capturing gets the launches enqueued eagerly. */
 int lora_stencil_run(lora_plan* p, const double* in, double* out, int64_t timesteps, void* stream);
 
 /* The same computation from HOST buffers: copies `in_host` to plan-owned device memory,
@@ -211,7 +231,10 @@ double* lora_stencil_p2p_buffer(const lora_p2p* c, int i);
  * final wait for the neighbours' last rows, copy-out (skipped if out_local is buffer T%2). */
 int lora_stencil_run_dist_p2p(lora_plan* p, lora_p2p* c, const double* in_local, double* out_local,
                               int64_t timesteps, void* stream);
-/* Synchronises the device and reports a spin-wait timeout (LORA_ERR_CUDA) if one occurred. */
+/* Synchronises the device and reports a spin-wait timeout (LORA_ERR_CUDA) if one occurred.  A
+ * timeout leaves the endpoint's monotonic step counters out of step with its neighbours for good:
+ * once reported, the endpoint is POISONED and every later lora_stencil_run_dist_p2p on it returns
+ * LORA_ERR_INVALID_ARG — destroy it and create (and connect) a new one. */
 int lora_stencil_p2p_status(lora_p2p* c);
 void lora_stencil_p2p_destroy(lora_p2p* c);
 

@@ -50,7 +50,11 @@ class lora_plan_info(ctypes.Structure):
                 ("z_symmetric", ctypes.c_int), ("fuse_k", ctypes.c_int), ("halo_depth", ctypes.c_int),
                 ("tile_m", ctypes.c_int), ("tile_n", ctypes.c_int), ("recon_err", ctypes.c_double),
                 ("growth", ctypes.c_double), ("fma_per_point_issued", ctypes.c_double),
-                ("fma_per_point_direct", ctypes.c_double), ("fma_per_point_separable", ctypes.c_double)]
+                ("fma_per_point_direct", ctypes.c_double), ("fma_per_point_separable", ctypes.c_double),
+                ("paper_points_per_update", ctypes.c_int), ("paper_rdg_frag_per_point", ctypes.c_double),
+                ("paper_convstencil_frag_per_point", ctypes.c_double), ("paper_convstencil_over_rdg", ctypes.c_double),
+                ("paper_mma_per_point", ctypes.c_double), ("paper_convstencil_mma_per_point", ctypes.c_double),
+                ("paper_fragment_waste", ctypes.c_int)]
 
     def as_dict(self):
         d = {f: getattr(self, f) for f, _ in self._fields_}
@@ -142,10 +146,39 @@ def lora_stencil_plan_query(plan) -> dict:
     return info.as_dict()
 
 
-def lora_stencil_plan_terms(plan, radius: int):
+def _padded_elems(plan) -> int:
+    info = lora_stencil_plan_query(plan)
+    n = 1
+    for i in range(info["ndim"]):
+        n *= int(info["grid"][i]) + 2 * int(info["radius"])
+    return n
+
+
+def _host_ptr(a, plan, what: str) -> int:
+    """Pointer of a host buffer after checking that it is what the C side will copy: float64,
+    C-contiguous, exactly the plan's padded element count (prod(N_i + 2r))."""
+    n = _padded_elems(plan)
+    if isinstance(a, np.ndarray):
+        ok = a.dtype == np.float64 and a.flags["C_CONTIGUOUS"] and a.size == n
+        ptr = a.ctypes.data
+    else:  # torch CPU tensor
+        ok = (not a.is_cuda) and a.dtype.is_floating_point and a.element_size() == 8 and a.is_contiguous() \
+            and a.numel() == n
+        ptr = a.data_ptr()
+    if not ok:
+        raise ValueError(f"{what}: expected a C-contiguous float64 host buffer of {n} elements (the plan's padded shape)")
+    return ptr
+
+
+def lora_stencil_plan_terms(plan, radius: int | None = None):
+    """The plan's rank-1 terms.  The term length is taken from the plan itself (2r+1 with the
+    plan's radius); `radius`, if given, must match it."""
+    r = int(lora_stencil_plan_query(plan)["radius"])
+    if radius is not None and int(radius) != r:
+        raise ValueError(f"radius {radius} does not match the plan's radius {r}")
     n = ctypes.c_int(0)
     _check(_lib.lora_stencil_plan_terms(plan, 0, ctypes.byref(n), None, None, None, None, None))
-    k, m = n.value, 2 * radius + 1
+    k, m = n.value, 2 * r + 1
     plane = np.zeros(k, np.int32); kind = np.zeros(k, np.int32); rad = np.zeros(k, np.int32)
     u = np.zeros((k, m)); v = np.zeros((k, m))
     if k:
@@ -161,15 +194,15 @@ def lora_stencil_run(plan, in_ptr: int, out_ptr: int, timesteps: int, stream: in
 
 def lora_stencil_run_host(plan, in_host: np.ndarray, out_host: np.ndarray, timesteps: int, stream: int = 0) -> None:
     """Host buffers (numpy arrays or torch CPU tensors, ideally pinned); synchronous."""
-    ip = in_host.ctypes.data if isinstance(in_host, np.ndarray) else in_host.data_ptr()
-    op = out_host.ctypes.data if isinstance(out_host, np.ndarray) else out_host.data_ptr()
+    ip = _host_ptr(in_host, plan, "in_host")
+    op = _host_ptr(out_host, plan, "out_host")
     _check(_lib.lora_stencil_run_host(plan, ip, op, int(timesteps), stream or None))
 
 
 def lora_stencil_run_host_async(plan, in_host, out_host, timesteps: int, stream: int) -> None:
     """Host buffers (pinned); enqueued on `stream` (not 0), the caller synchronises it."""
-    ip = in_host.ctypes.data if isinstance(in_host, np.ndarray) else in_host.data_ptr()
-    op = out_host.ctypes.data if isinstance(out_host, np.ndarray) else out_host.data_ptr()
+    ip = _host_ptr(in_host, plan, "in_host")
+    op = _host_ptr(out_host, plan, "out_host")
     _check(_lib.lora_stencil_run_host_async(plan, ip, op, int(timesteps), stream or None))
 
 
@@ -267,7 +300,7 @@ class Stencil:
         return lora_stencil_plan_query(self.plan)
 
     def terms(self):
-        return lora_stencil_plan_terms(self.plan, self.radius)
+        return lora_stencil_plan_terms(self.plan)
 
     def run(self, x_in, x_out, timesteps: int, stream=None) -> None:
         for x in (x_in, x_out):
@@ -280,6 +313,9 @@ class Stencil:
         lora_stencil_run(self.plan, x_in.data_ptr(), x_out.data_ptr(), timesteps, s)
 
     def run_host(self, a_in, a_out, timesteps: int, stream: int = 0) -> None:
+        for a in (a_in, a_out):
+            if tuple(a.shape) != self.padded_shape:
+                raise ValueError(f"expected host arrays of shape {self.padded_shape}")
         lora_stencil_run_host(self.plan, a_in, a_out, timesteps, stream)
 
     def close(self):

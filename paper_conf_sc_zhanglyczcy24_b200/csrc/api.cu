@@ -98,6 +98,11 @@ bool use_graph(const Plan& p, int64_t launches, cudaStream_t s) {
   static int off = [] { const char* e = std::getenv("LORA_NO_GRAPH"); return e && e[0] == '1' ? 1 : 0; }();
   // the legacy / per-thread default streams cannot be captured
   if (s == nullptr || s == cudaStreamLegacy || s == cudaStreamPerThread) return false;
+  // a stream the caller is already capturing (e.g. torch.cuda.graph around run): enqueue eagerly into
+  // the caller's capture instead of starting a nested one, which would fail and invalidate it
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(s, &cs) != cudaSuccess) { cudaGetLastError(); return false; }
+  if (cs != cudaStreamCaptureStatusNone) return false;
   return !off && launches >= 4 && p.elems <= (size_t(1) << 22);
 }
 
@@ -209,6 +214,19 @@ int lora_stencil_plan_query(const lora_plan* p, lora_plan_info* info) {
   info->fma_per_point_issued = p->fma_issued;
   info->fma_per_point_direct = p->fma_direct;
   info->fma_per_point_separable = p->fma_separable;
+  {  // the paper's cost model at h = R (include/lora_stencil.h; eq. 12-14, eq. 16)
+    const int h = p->R;
+    auto cdiv = [](int a, int b) { return (a + b - 1) / b; };
+    const int pts = 32 * cdiv(h, 2) * cdiv(h, 4);
+    const int box = cdiv((2 * h + 1) * (2 * h + 1), 4);
+    info->paper_points_per_update = pts;
+    info->paper_rdg_frag_per_point = 1.0 / 8.0;
+    info->paper_convstencil_frag_per_point = 2.0 * box / (8.0 * (2 * h + 2));
+    info->paper_convstencil_over_rdg = double(box) / (h + 1);
+    info->paper_mma_per_point = double(2 * h * cdiv(h, 2) * (2 * cdiv(h, 4) + 1)) / pts;
+    info->paper_convstencil_mma_per_point = info->paper_convstencil_frag_per_point;   // no fragment reuse
+    info->paper_fragment_waste = 256 - (8 + 2 * h) * (8 + 2 * h);
+  }
   return LORA_OK;
 }
 

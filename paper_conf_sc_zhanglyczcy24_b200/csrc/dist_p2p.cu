@@ -99,6 +99,7 @@ struct lora_p2p {
   int* err = nullptr;
   Peer lo, hi;
   unsigned long long epoch = 0;
+  bool poisoned = false;           // a spin-wait timed out: the flag protocol is out of step for good
 };
 
 namespace {
@@ -312,6 +313,8 @@ int lora_stencil_run_dist_p2p(lora_plan* p, lora_p2p* c, const double* in_local,
     return fail(LORA_ERR_INVALID_ARG, "plan does not match the endpoint's slab");
   if ((c->rank > 0 && !c->lo.present) || (c->rank < c->nranks - 1 && !c->hi.present))
     return fail(LORA_ERR_INVALID_ARG, "endpoint is not connected to its neighbours");
+  if (c->poisoned)
+    return fail(LORA_ERR_INVALID_ARG, "endpoint is poisoned by an earlier exchange timeout: destroy it and create a new one");
   const int R = p->R;
   const size_t bytes = p->elems * sizeof(double);          // the caller's layout (R-deep halos)
   // launches: ceil(T / k) of k steps, the last one taking the remainder
@@ -417,7 +420,11 @@ int lora_stencil_p2p_status(lora_p2p* c) {
   int h = 0;
   cudaError_t e = cudaMemcpy(&h, c->err, sizeof(int), cudaMemcpyDeviceToHost);
   if (e != cudaSuccess) return cuda_fail(e, "p2p status read");
-  if (h) return fail(LORA_ERR_CUDA, "device-initiated halo exchange: a neighbour's step counter did not advance for 20 s");
+  if (h) {
+    c->poisoned = true;   // every later run_dist_p2p on this endpoint is refused
+    return fail(LORA_ERR_CUDA, "device-initiated halo exchange: a neighbour's step counter did not advance for 20 s "
+                               "(endpoint poisoned: destroy and re-create it)");
+  }
   return LORA_OK;
 }
 

@@ -81,11 +81,10 @@ template <int R, int K>
 cudaError_t launch_k(const Plan& p, const double* src, double* dst, cudaStream_t s) {
   constexpr int LEN = S1_SEG + 2 * K * R + 8;
   const int smem = 2 * LEN * 8;
-  static int max_grid = 0;
-  if (max_grid == 0) {
-    cudaError_t e = cudaFuncSetAttribute(stencil1d_kernel<R, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  int max_grid = 0;
+  {
+    cudaError_t e = kernel_setup((const void*)stencil1d_kernel<R, K>, S1_THREADS, smem, &max_grid);
     if (e != cudaSuccess) return e;
-    max_grid = persistent_grid((const void*)stencil1d_kernel<R, K>, S1_THREADS, smem, int64_t(1) << 40);
   }
   W1 w{};
   for (int i = 0; i < 2 * R + 1; ++i) w.w[i] = p.W[i];

@@ -869,11 +869,10 @@ cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream
   constexpr int BS = 64 * NH - 2 * R * (K - 1) - 2 * ((R * (K - 1)) & 1);
   constexpr int BUFD = G::BUFD;
   const int smem = 128 + RDG_WARPS * (G::WARP_BYTES + 2 * (K - 1) * BUFD * 8);
-  static int max_grid = 0;
-  if (max_grid == 0) {
-    cudaError_t e = cudaFuncSetAttribute(rdg2d_kernel<R, SIG, K, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  int max_grid = 0;
+  {
+    cudaError_t e = kernel_setup((const void*)rdg2d_kernel<R, SIG, K, TMA>, RDG_WARPS * 32, smem, &max_grid);
     if (e != cudaSuccess) return e;
-    max_grid = persistent_grid((const void*)rdg2d_kernel<R, SIG, K, TMA>, RDG_WARPS * 32, smem, int64_t(1) << 40);
   }
   if (d && d->prepare_only) return cudaSuccess;
   // chunk rows: a multiple of 2R+1 (static ring slots), <= RDG_RC; small grids get shorter chunks

@@ -425,11 +425,10 @@ template <int R, class SG, bool TMA>
 cudaError_t rdg3d_launch(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
                          const R3Params& prm, const P2PArgs* d) {
   using G = G3<R>;
-  static int max_grid = 0;
-  if (max_grid == 0) {
-    cudaError_t e = cudaFuncSetAttribute(rdg3d_kernel<R, SG, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, G::SMEM);
+  int max_grid = 0;
+  {
+    cudaError_t e = kernel_setup((const void*)rdg3d_kernel<R, SG, TMA>, R3_WARPS * 32, G::SMEM, &max_grid);
     if (e != cudaSuccess) return e;
-    max_grid = persistent_grid((const void*)rdg3d_kernel<R, SG, TMA>, R3_WARPS * 32, G::SMEM, int64_t(1) << 40);
   }
   if (d && d->prepare_only) return cudaSuccess;
   const int nbx = (int)((p.N[2] + 63) / 64), nby = (int)((p.N[1] + BY<R> - 1) / BY<R>);

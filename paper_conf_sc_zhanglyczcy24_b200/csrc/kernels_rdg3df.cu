@@ -472,11 +472,10 @@ cudaError_t launch_f(const Plan& p, const double* src, double* dst, cudaStream_t
                      const FParams& prm) {
   constexpr int STAGE = ((F_IN * F_BW * 8 + 127) / 128) * 128;
   const int smem = 128 + SG::ns * STAGE + 2 * (K - 1) * F_S1 * F_S1W * 8;
-  static int max_grid = 0;
-  if (max_grid == 0) {
-    cudaError_t e = cudaFuncSetAttribute(rdg3df_kernel<SG, K, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  int max_grid = 0;
+  {
+    cudaError_t e = kernel_setup((const void*)rdg3df_kernel<SG, K, TMA>, F_WARPS * 32, smem, &max_grid);
     if (e != cudaSuccess) return e;
-    max_grid = persistent_grid((const void*)rdg3df_kernel<SG, K, TMA>, F_WARPS * 32, smem, int64_t(1) << 40);
   }
   constexpr int TY = F_S1 - 2 * (K - 1), BS = 64 - 2 * (K - 1) - 2 * ((K - 1) & 1);
   const int nbx = (int)((p.N[2] + BS - 1) / BS), nby = (int)((p.N[1] + TY - 1) / TY);

@@ -130,11 +130,10 @@ cudaError_t tc_launch(const Plan& p, const double* src, double* dst, cudaStream_
   const size_t smem = 128 + 2 * BUF;
   const int ntx = (int)((p.N[1] + TC_BN - 1) / TC_BN), nty = (int)((p.N[0] + TC_BM - 1) / TC_BM);
   const int64_t ntiles = int64_t(ntx) * nty;
-  static int max_grid = 0;
-  if (max_grid == 0) {
-    cudaError_t e = cudaFuncSetAttribute(tc2d_kernel<R, TMA, NOBVS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  int max_grid = 0;
+  {
+    cudaError_t e = kernel_setup((const void*)tc2d_kernel<R, TMA, NOBVS>, 256, smem, &max_grid);
     if (e != cudaSuccess) return e;
-    max_grid = persistent_grid((const void*)tc2d_kernel<R, TMA, NOBVS>, 256, smem, int64_t(1) << 40);
   }
   const int grid = (int)std::min<int64_t>(max_grid, ntiles);
   const TcParams prm = make_params(p);

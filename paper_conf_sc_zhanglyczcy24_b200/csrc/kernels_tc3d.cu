@@ -216,11 +216,10 @@ template <int R, bool TMA>
 cudaError_t tc3d_launch(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
                         const TcParams& prm, const Tc3Planes& pl) {
   using G = T3G<R>;
-  static int max_grid = 0;
-  if (max_grid == 0) {
-    cudaError_t e = cudaFuncSetAttribute(tc3d_kernel<R, TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize, G::SMEM);
+  int max_grid = 0;
+  {
+    cudaError_t e = kernel_setup((const void*)tc3d_kernel<R, TMA>, 256, G::SMEM, &max_grid);
     if (e != cudaSuccess) return e;
-    max_grid = persistent_grid((const void*)tc3d_kernel<R, TMA>, 256, G::SMEM, int64_t(1) << 40);
   }
   const int ntx = (int)((p.N[2] + TC_BN - 1) / TC_BN), nty = (int)((p.N[1] + TC_BM - 1) / TC_BM);
   const int ntz = (int)((p.N[0] + T3_ZC - 1) / T3_ZC);

@@ -107,4 +107,9 @@ bool encode_tmap(CUtensorMap* map, const double* base, int rank, const int64_t* 
 
 int persistent_grid(const void* kernel, int threads, size_t smem, int64_t ntiles);
 
+// Per-device, thread-safe kernel preparation: sets the kernel's dynamic shared-memory limit on the
+// CURRENT device (function attributes are per device context) the first time this (kernel, device)
+// pair is seen, and returns the persistent grid size (SMs x resident CTAs) for it in *max_grid.
+cudaError_t kernel_setup(const void* kernel, int threads, size_t smem, int* max_grid);
+
 }  // namespace lora

@@ -3,7 +3,9 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 
+#include <map>
 #include <mutex>
+#include <utility>
 
 #include "pipe.cuh"
 
@@ -62,6 +64,23 @@ int persistent_grid(const void* kernel, int threads, size_t smem, int64_t ntiles
   int64_t g = int64_t(sms) * occ;
   if (g > ntiles) g = ntiles;
   return (int)(g < 1 ? 1 : g);
+}
+
+cudaError_t kernel_setup(const void* kernel, int threads, size_t smem, int* max_grid) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, int> cache;   // (kernel, device) -> persistent grid
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  std::lock_guard<std::mutex> lock(mu);
+  auto it = cache.find({kernel, dev});
+  if (it != cache.end()) { *max_grid = it->second; return cudaSuccess; }
+  e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  const int g = persistent_grid(kernel, threads, smem, int64_t(1) << 40);
+  cache[{kernel, dev}] = g;
+  *max_grid = g;
+  return cudaSuccess;
 }
 
 }  // namespace lora

@@ -363,7 +363,8 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
     // the 1 kW power cap under sustained load (~1.7 GHz), fused it is FP64-bound at full clock
     // (bench.py, 8 x 100 steps: 303 -> 320 GS/s); the same holds for Box-3D27P (307 -> 320).
     const double work = cuda_fma_per_point(p);
-    if (p.ndim == 1) fk = 8;
+    if (eng != LORA_ENGINE_RDG_CUDA) fk = 1;   // composed fusion on tensor cores is opt-in (fuse_k > 1)
+    else if (p.ndim == 1) fk = 8;
     else if (p.ndim == 3) fk = 2;   // Heat-3D; Box-3D27P too: sustained 307 (power-capped) -> 320 GS/s
     else if (p.rdg_rows && radius == 3) fk = 2;   // Box-2D49P: sustained (power-capped) 303 -> 320 GS/s
     else if (work > 20.0) fk = 1;
@@ -371,7 +372,6 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
     fk = std::min(max_k, fk);
   }
   p.fuse_k = fk;
-  if (eng == LORA_ENGINE_TC && fk == 0) p.fuse_k = 1;   // composed fusion on tensor cores is opt-in
   if (eng == LORA_ENGINE_TC && p.fuse_k > 1) {
     // composed kernel: W_k = W (*) W_{k-1} (full 2D convolution of the offset weights: applying the
     // correlation twice adds the offsets), radius kR; factored by the same planner (PMA / arms /
