@@ -31,10 +31,6 @@ import numpy as np  # noqa: E402
 METRIC = "GStencil/s FP64 per stencil at 1/2/4/8 B200; % of HBM roofline"
 UNIT = "GStencil/s"
 BYTES_PER_POINT = 16.0  # algorithmic HBM bytes per point per time step: read 8 + write 8
-# algorithmic FP64 flops per point per time step: the separable minimum of the rank-1 method
-# (SURVEY §8(d) "Roofline"; FMA = 2 flops)
-ALG_FLOPS_PER_POINT = {"heat2d-256": 10.0, "box2d9p-10240": 14.0, "box2d49p-10240": 62.0, "heat3d-512": 14.0,
-                       "box3d27p-512": 42.0}
 
 
 def parse():
@@ -46,7 +42,8 @@ def parse():
     ap.add_argument("--workload", default="box2d49p-10240")
     ap.add_argument("--engine", default="auto")
     ap.add_argument("--fuse", type=int, default=0)
-    ap.add_argument("--per-stencil", action="store_true", help="also time the other single-GPU configs")
+    ap.add_argument("--per-stencil", action="store_true", help="also time the other Table II kernels (NEXT-3)")
+    ap.add_argument("--no-configs", action="store_true", help="skip the per-config records of the BASELINE configs")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-inflight", type=int, default=3,
                     help="independent problems in flight in the e2e run (one plan + stream each)")
@@ -115,6 +112,45 @@ def load_peaks():
         d = json.load(open(p))
         return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def load_fp64_peak():
+    """Measured FP64 pipe peak (lane-ops/s: one DFMA/DADD/DMUL per lane = 1) from the newest committed
+    profiles/*_fp64_peak.json (tools/fp64_peak.py); else the nominal 148 SMs x 64 FP64 lanes/clk x
+    1.965 GHz (B200_PROFILING.md unit counts), saying which."""
+    import glob
+    fs = sorted(glob.glob(os.path.join(ROOT, "profiles", "*_fp64_peak.json")))
+    if fs:
+        d = json.load(open(fs[-1]))
+        return float(d["ops"]["dfma_uniform"]["lane_ops_per_s"]), f"measured: {os.path.relpath(fs[-1], ROOT)} (DFMA, uniform weight operand)"
+    return 148 * 64 * 1.965e9, "derived: 148 SMs x 64 FP64 lanes/clk x 1.965 GHz (no measured FP64 peak committed)"
+
+
+def roofline_views(info, shape, T, fuse, t_run, hbm_peak, hbm_src, fp64_peak, fp64_src, world=1):
+    """Two rooflines of the dominant (stencil) kernel from one timed run of T steps:
+    hbm : ALGORITHMIC bytes per launch (16/k B per point-step x k steps = 16 B per point
+          per launch, one read + one write of the grid) / average launch time, vs the measured copy BW;
+    fp64: ALGORITHMIC FP64 lane-ops per launch (the plan's per-point FP64 instruction count of the
+          chosen rank-1 form, e.g. 25 for the Box-2D49P row-pair split, x points x k; redundant halo
+          recomputation NOT counted) / average launch time, vs the measured FP64 pipe peak.
+    `bound` is the view with the larger fraction (the resource the kernel runs closest to)."""
+    pts = float(np.prod(shape))
+    n_launch = -(-T // fuse)
+    avg = t_run / n_launch
+    hb = BYTES_PER_POINT * pts
+    hbm = {"bound": "hbm", "achieved": hb / avg / 1e9, "peak": hbm_peak, "unit": "GB/s",
+           "frac": hb / avg / 1e9 / hbm_peak, "peak_source": hbm_src, "algorithmic_bytes_per_launch": hb}
+    ops = info["fma_per_point_issued"] * pts * (T / n_launch)
+    fp = {"bound": "alu", "achieved": ops / avg / 1e9, "peak": fp64_peak / 1e9, "unit": "GFP64-op/s",
+          "frac": ops / avg / fp64_peak, "peak_source": fp64_src,
+          "fp64_ops_per_point_step": info["fma_per_point_issued"], "algorithmic_ops_per_launch": ops,
+          "note": "one FP64 lane-op = one DFMA, DADD or DMUL on one lane (the pipe's issue unit)"}
+    roof = dict(fp if fp["frac"] > hbm["frac"] else hbm)
+    roof.update({"avg_launch_ms": avg * 1e3, "launches_per_run": n_launch, "views": {"hbm": hbm, "fp64": fp},
+                 "gstencil_roofline_hbm_unfused": hbm_peak / BYTES_PER_POINT * world,
+                 "gstencil_ceiling": min(hbm_peak * fuse / BYTES_PER_POINT, fp64_peak / 1e9 / info["fma_per_point_issued"]),
+                 "gstencil_ceiling_note": "min(HBM at 16/k B per point-step, FP64 peak / ops per point-step)"})
+    return roof
 
 
 def ncu_traffic(workload, engine):
@@ -326,45 +362,17 @@ def main():
         nb = (1 if rank > 0 else 0) + (1 if rank < world - 1 else 0)
         launches_per_step = -(-T // fuse) + 1 + 5 * nb
 
-    # roofline for the dominant kernel (the stencil kernel), two views; "bound" is the resource the
-    # kernel runs closest to (the larger fraction):
-    #  hbm: ALGORITHMIC bytes per launch (16 B per point per launch: one read + one write of the grid,
-    #       whatever the fused depth) / average launch time, vs the measured HBM copy bandwidth;
-    #  alu: ALGORITHMIC FP64 flops per launch (SURVEY.md §8(d)'s per-point figure — the separable
-    #       minimum of the rank-1 method, FMA = 2 flops — x points x fused steps) / average launch
-    #       time, vs 148 SMs x 64 FP64 FMA/clk x 2 x 1.965 GHz = 37.2 TFLOP/s (the step-0
-    #       DMMA microbenchmark reaches 36.9).  "issued" adds what the kernel really puts through the
-    #       FP64 pipe: the plan's issued FP64 instructions per point-step (DFMA/DADD/DMUL, each one
-    #       lane slot) against 148 x 64 lane slots x 1.965 GHz.
+    # roofline of the dominant kernel (the stencil kernel): HBM and FP64 views (roofline_views)
     peak, peak_src = load_peaks()
-    n_launch = -(-T // fuse)
-    per_launch_bytes = BYTES_PER_POINT * float(np.prod(shape))      # per launch: one (fused) superstep
-    avg_launch_s = t / args.steps / n_launch
-    achieved = per_launch_bytes / avg_launch_s / 1e9
-    fp64_peak_tflops = 148 * 64 * 2 * 1.965e9 / 1e12
-    alg_flops_pt = ALG_FLOPS_PER_POINT.get(args.workload, 2.0 * info["fma_per_point_separable"])
-    flops_per_launch = alg_flops_pt * float(np.prod(shape)) * (T / n_launch)
-    alu_achieved = flops_per_launch / avg_launch_s / 1e12
-    issued_ops = info["fma_per_point_issued"] * float(np.prod(shape)) * (T / n_launch) / avg_launch_s
+    fp64_peak, fp64_src = load_fp64_peak()
+    roof = roofline_views(info, shape, T, fuse, t / args.steps, peak, peak_src, fp64_peak, fp64_src, world)
     tr = ncu_traffic(args.workload, info["engine_name"])
     if tr and int(tr.get("fuse", 1)) != fuse:
         tr = None
-    hbm = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-           "peak_source": peak_src, "algorithmic_bytes_per_launch": per_launch_bytes}
-    alu = {"bound": "alu", "achieved": alu_achieved, "peak": fp64_peak_tflops, "unit": "TFLOP/s",
-           "frac": alu_achieved / fp64_peak_tflops,
-           "peak_source": "derived: 148 SMs x 64 FP64 FMA/clk x 2 flops x 1.965 GHz (DESIGN.md §6)",
-           "algorithmic_flops_per_point": alg_flops_pt, "algorithmic_flops_per_launch": flops_per_launch,
-           "issued": {"fp64_instr_per_point": info["fma_per_point_issued"], "gop_s": issued_ops / 1e9,
-                      "frac_of_pipe": issued_ops / (148 * 64 * 1.965e9)}}
-    roof = dict(alu if alu["frac"] > hbm["frac"] else hbm)
     roof.update({"traffic": tr["bytes"] if tr else None,       # dram read+write bytes per launch (ncu --set full)
                  "traffic_source": ({k: tr[k] for k in ("kernel", "source", "fuse")} if tr else None),
                  "kernel": f"{info['engine_name']} stencil step (fuse_k={fuse})",
-                 "avg_launch_ms": avg_launch_s * 1e3,
-                 "avg_launch_note": "timed step / stencil launches per step (the 2 halo-copy launches per run, ~0.1%, included)",
-                 "views": {"hbm": hbm, "alu": alu},
-                 "gstencil_roofline": peak / BYTES_PER_POINT * world,
+                 "avg_launch_note": "timed run / stencil launches per run (the 2 halo-copy launches per run, ~0.1%, included)",
                  "frac_gstencil_of_hbm_roofline": value / (peak / BYTES_PER_POINT * world)})
 
     # e2e: through the C-ABI with HOST buffers (H2D of the input + D2H of the result inside the region).
@@ -407,37 +415,68 @@ def main():
                           "api": "lora_stencil_run_host, one synchronous call per step"},
                "clock": "host wall clock around the K steps"}
 
-    per_stencil = None
-    if args.per_stencil and rank == 0 and world == 1:
-        per_stencil = {}
-        for name in ("heat2d-256", "box2d9p-10240", "box2d49p-10240", "heat3d-512", "box3d27p-512",
-                     "star2d13p-10240", "heat1d-10240000", "1d5p-10240000"):
+    # per-config records: every BASELINE single-GPU config (configs[0..3]), planner defaults, seeded
+    # SplitMix64 inputs generated on the device (bit-identical to synth.grid), CUDA events around each
+    # run on the launching stream, L2 flushed (a 256 MB write) before each run, NVML clocks sampled
+    # during the timed runs; --per-stencil adds the other Table II kernels.
+    per_config = None
+    if rank == 0 and world == 1 and not args.no_configs:
+        per_config = {}
+        names = ["heat2d-256", "box2d9p-10240", "box2d49p-10240", "heat3d-512", "box3d27p-512"]
+        if args.per_stencil:
+            names += ["star2d13p-10240", "heat1d-10240000", "1d5p-10240000"]
+        flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+        for name in names:
             Wn, cn = synth.config(name)
-            s2 = L.Stencil(Wn, cn["shape"], engine=args.engine)
-            xa = torch.rand(cn["padded"], dtype=torch.float64, device=dev) + 0.5
+            s2 = L.Stencil(Wn, cn["shape"])
+            i2 = s2.info()
+            xa = synth.grid_torch(cn["padded"], cn["seed"], device=dev)
             ya = torch.empty_like(xa)
-            L.lora_stencil_run(s2.plan, xa.data_ptr(), ya.data_ptr(), cn["T"], sptr)
-            torch.cuda.synchronize(dev)
-            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            a0.record(stream)
+            reps = 20 if np.prod(cn["shape"]) < 1e7 else 5
             for _ in range(3):
                 L.lora_stencil_run(s2.plan, xa.data_ptr(), ya.data_ptr(), cn["T"], sptr)
-            a1.record(stream)
             torch.cuda.synchronize(dev)
-            ts = a0.elapsed_time(a1) / 3e3
-            gs = float(np.prod(cn["shape"])) * cn["T"] / ts / 1e9
-            per_stencil[name] = {"GStencil_s": gs, "frac_hbm_roofline": gs / (peak / BYTES_PER_POINT),
-                                 "engine": s2.info()["engine_name"], "ms": ts * 1e3}
+            ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+            with ClockSampler(local) as clk2:
+                for a0, a1 in ev:
+                    flush.fill_(1)
+                    a0.record(stream)
+                    L.lora_stencil_run(s2.plan, xa.data_ptr(), ya.data_ptr(), cn["T"], sptr)
+                    a1.record(stream)
+                torch.cuda.synchronize(dev)
+            ts = sorted(a0.elapsed_time(a1) / 1e3 for a0, a1 in ev)
+            tmed = ts[len(ts) // 2]
+            gs = float(np.prod(cn["shape"])) * cn["T"] / tmed / 1e9
+            rf = roofline_views(i2, cn["shape"], cn["T"], i2["fuse_k"], tmed, peak, peak_src, fp64_peak, fp64_src)
+            per_config[name] = {"value": gs, "unit": UNIT, "grid": list(cn["shape"]), "T": cn["T"],
+                                "ms_per_run_median": tmed * 1e3, "ms_per_run_best": ts[0] * 1e3, "runs": reps,
+                                "engine": i2["engine_name"], "fuse_k": i2["fuse_k"],
+                                "fp64_ops_per_point_step": i2["fma_per_point_issued"],
+                                "frac_gstencil_of_hbm_roofline": gs / (peak / BYTES_PER_POINT),
+                                "roofline": {k: rf[k] for k in ("bound", "achieved", "peak", "unit", "frac")} |
+                                            {"views": {v: {k: rf["views"][v][k] for k in ("achieved", "peak", "unit", "frac")}
+                                                       for v in rf["views"]},
+                                             "gstencil_ceiling": rf["gstencil_ceiling"]},
+                                "clocks": clk2.summary(), "l2": "flushed before each run (256 MB write)",
+                                "weights": cn["weights"]}
             s2.close()
             del xa, ya
+        del flush
+        torch.cuda.empty_cache()
 
     # the same workload on every engine (the paper's tensor-core chain, the CUDA-core RDG, direct)
     engines = None
     if rank == 0 and world == 1 and not args.no_engines:
         engines = {}
-        for eng in ("tc", "rdg_cuda", "direct"):
+        for eng in ("tc", "rdg_cuda", "rdg_cuda_pma", "rdg_cuda_k1", "direct"):
             try:
-                s3 = L.Stencil(W, shape, engine=eng)
+                if eng == "rdg_cuda_pma":   # the paper's PMA pyramid on the CUDA-core engine (LORA_RDG_PMA=1)
+                    os.environ["LORA_RDG_PMA"] = "1"
+                try:
+                    s3 = L.Stencil(W, shape, engine=eng[:8] if eng.startswith("rdg_cuda") else eng,
+                                   fuse_k=1 if eng == "rdg_cuda_k1" else 0)
+                finally:
+                    os.environ.pop("LORA_RDG_PMA", None)
             except L.LoraError as ex:
                 engines[eng] = {"unsupported": str(ex)}
                 continue
@@ -454,13 +493,13 @@ def main():
             i3 = s3.info()
             # issued FP64 rate against the measured FP64 pipe peak (step-0 microbenchmark, DESIGN.md §5:
             # DMMA 36.9 TF, DFMA 33.8 TF; profiles/r01_step0_fp64_pipes.jsonl)
-            fp64_peak = 36.9e12 if eng == "tc" else 33.8e12
-            issued_tf = gs * 1e9 * i3["fma_per_point_issued"] * 2
+            rf = roofline_views(i3, shape, T, i3["fuse_k"], ts, peak, peak_src, fp64_peak, fp64_src)
             engines[eng] = {"GStencil_s": gs, "frac_hbm_roofline": gs / (peak / BYTES_PER_POINT), "fuse_k": i3["fuse_k"],
-                            "fma_per_point_issued": i3["fma_per_point_issued"], "ms_per_step": ts * 1e3,
-                            "issued_fp64_tflops": issued_tf / 1e12,
-                            "frac_fp64_pipe_peak": issued_tf / fp64_peak,
-                            "fp64_pipe": "DMMA (tensor)" if eng == "tc" else "DFMA"}
+                            "fp64_ops_per_point_step": i3["fma_per_point_issued"], "ms_per_step": ts * 1e3,
+                            "n_terms": i3["n_terms"],
+                            "roofline_fracs": {v: rf["views"][v]["frac"] for v in rf["views"]},
+                            "fp64_pipe": ("DMMA (tensor): ops = issued FMA slots incl. band padding" if eng == "tc"
+                                          else "DFMA/DADD/DMUL")}
             s3.close()
 
     cpu = None
@@ -483,8 +522,8 @@ def main():
                 "fma_per_point": {"issued": info["fma_per_point_issued"], "direct": info["fma_per_point_direct"],
                                   "separable": info["fma_per_point_separable"]},
                 "host": host_info()}
-        if per_stencil:
-            line["per_stencil"] = per_stencil
+        if per_config:
+            line["configs"] = per_config
         if engines:
             line["engines"] = engines
         print(json.dumps(line), flush=True)
