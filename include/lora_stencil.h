@@ -78,6 +78,8 @@ typedef struct {               /* filled by lora_stencil_plan_query             
   int fuse_k;                  /* time steps per HBM round trip                               */
   int halo_depth;              /* fuse_k * radius                                             */
   int tile_m, tile_n;          /* CTA output tile (rows, columns of the fastest axis)         */
+  int single_launch;           /* 1: small 2D grid, all T steps in ONE thread-block-cluster launch
+                                  holding the grid in shared memory (DSMEM halo exchange)       */
   double recon_err;            /* max|sum u v^T - W| / max|W|                                 */
   double growth;               /* sum_k ||u_k||_1 ||v_k||_1 / ||W||_1                         */
   double fma_per_point_issued; /* FP64 FMAs issued per point per step by the chosen engine    */

@@ -48,7 +48,8 @@ class lora_plan_info(ctypes.Structure):
                 ("engine", ctypes.c_int), ("n_terms", ctypes.c_int), ("n_tc_chain", ctypes.c_int),
                 ("n_tc_single", ctypes.c_int), ("n_cuda", ctypes.c_int), ("n_planes_pointwise", ctypes.c_int),
                 ("z_symmetric", ctypes.c_int), ("fuse_k", ctypes.c_int), ("halo_depth", ctypes.c_int),
-                ("tile_m", ctypes.c_int), ("tile_n", ctypes.c_int), ("recon_err", ctypes.c_double),
+                ("tile_m", ctypes.c_int), ("tile_n", ctypes.c_int), ("single_launch", ctypes.c_int),
+                ("recon_err", ctypes.c_double),
                 ("growth", ctypes.c_double), ("fma_per_point_issued", ctypes.c_double),
                 ("fma_per_point_direct", ctypes.c_double), ("fma_per_point_separable", ctypes.c_double),
                 ("paper_points_per_update", ctypes.c_int), ("paper_rdg_frag_per_point", ctypes.c_double),

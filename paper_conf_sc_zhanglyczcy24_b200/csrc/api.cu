@@ -112,11 +112,22 @@ int run_device(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s
     cudaError_t e = cudaMemcpyAsync(out, in, bytes, cudaMemcpyDeviceToDevice, s);
     return e == cudaSuccess ? LORA_OK : cuda_fail(e, "cudaMemcpyAsync");
   }
+  cudaError_t e;
+  if (small2d_eligible(p)) {   // small 2D grid: every step in one cluster launch (kernels_small.cu)
+    int rc = ensure_device(p, false);
+    if (rc) return rc;
+    e = launch_small2d(p, in, out, T, s);
+    if (e == cudaSuccess) {
+      if (sync_check() && (e = cudaStreamSynchronize(s)) != cudaSuccess) return cuda_fail(e, "LORA_SYNC_CHECK stream sync");
+      return LORA_OK;
+    }
+    if (e != cudaErrorNotSupported) return cuda_fail(e, "small-grid cluster launch");
+    cudaGetLastError();   // the device cannot schedule the cluster: the streaming path below
+  }
   const int64_t L = (int64_t)launch_plan(p, T).size();
   const bool two = L >= 2;
   int rc = ensure_device(p, two);
   if (rc) return rc;
-  cudaError_t e;
   if (use_graph(p, L, s)) {
     const bool same = p.g_in == in && p.g_out == out && p.g_T == T && p.g_stream == (void*)s;
     if (same && p.graph_exec) {
@@ -209,6 +220,7 @@ int lora_stencil_plan_query(const lora_plan* p, lora_plan_info* info) {
   info->fuse_k = p->fuse_k;
   info->halo_depth = p->fuse_k * p->R;
   info->tile_m = p->tile_m; info->tile_n = p->tile_n;
+  info->single_launch = small2d_eligible(*p) ? 1 : 0;
   info->recon_err = p->recon_err;
   info->growth = p->growth;
   info->fma_per_point_issued = p->fma_issued;

@@ -40,7 +40,8 @@ struct Plan {
   int tile_m = 0, tile_n = 0;
   int z_symmetric = 0;
   int force_no_tma = 0;   // LORA_NO_TMA=1: use the LDGSTS staging path (tests both loaders)
-  int tc_no_bvs = 0;      // LORA_TC_NO_BVS=1: the Fig. 9 ablation (shuffle-based stage 2) in the TC engine
+  int tc_no_bvs = 0;
+  int no_small = 0;       // LORA_NO_SMALL=1: no single-launch cluster path for small 2D grids (tests)      // LORA_TC_NO_BVS=1: the Fig. 9 ablation (shuffle-based stage 2) in the TC engine
   int n_planes_point = 0;
   // CUDA-core engine, 2D, radius >= 3, W reflection-symmetric in both axes: evaluate W as the
   // row-pair rank-1 split u_a = e_{R+a} + e_{R-a}, v_a = W[R+a,:] (a = 0..R; exact, growth 1),

@@ -415,6 +415,8 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
     p.force_no_tma = (e && e[0] == '1') ? 1 : 0;
     const char* b = std::getenv("LORA_TC_NO_BVS");
     p.tc_no_bvs = (b && b[0] == '1') ? 1 : 0;
+    const char* sm = std::getenv("LORA_NO_SMALL");
+    p.no_small = (sm && sm[0] == '1') ? 1 : 0;
   }
   p.tile_m = eng == LORA_ENGINE_TC ? 64 : (p.ndim == 2 ? 64 : 8);
   p.tile_n = eng == LORA_ENGINE_TC ? 64 : 32;

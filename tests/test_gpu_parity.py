@@ -412,3 +412,22 @@ def test_zero_centre_tap_fallback_3d():
     assert info["fuse_k"] == 2
     assert np.array_equal(a, b)
     assert rel_err(a, ref) <= 1e-12
+
+
+@pytest.mark.parametrize("kind,h", [("heat2d", 1), ("star", 1), ("star", 2), ("star", 3), ("star", 4)])
+@pytest.mark.parametrize("shape", [(256, 256), (64, 100), (48, 33), (32, 258)])
+def test_small_cluster_path_bitwise(kind, h, shape, monkeypatch):
+    """Small 2D star grids run all T steps in one thread-block-cluster launch (kernels_small.cu,
+    DSMEM halo exchange): bitwise equal to the streaming engine's per-step launches
+    (LORA_NO_SMALL=1) and within 1e-12 of the oracle, for T on both sides of the fusion depth."""
+    W = synth.preset("heat2d") if kind == "heat2d" else synth.star_weights(2, h, 11 + h)
+    g = synth.grid(tuple(n + 2 * h for n in shape), 20240101 + h)
+    for T in (1, 2, 5, 10):
+        out, info = run_gpu(W, g, T)
+        assert info["single_launch"] == 1, info
+        monkeypatch.setenv("LORA_NO_SMALL", "1")
+        ref_stream, info2 = run_gpu(W, g, T)
+        monkeypatch.delenv("LORA_NO_SMALL")
+        assert info2["single_launch"] == 0
+        assert np.array_equal(out, ref_stream), (T, float(np.max(np.abs(out - ref_stream))))
+        assert rel_err(out, oracle.run(W, g, T)) <= 1e-12

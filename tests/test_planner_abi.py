@@ -238,3 +238,17 @@ def test_plan_query_fields(L):
         L.Stencil(W, (100, 200), engine="rdg_cuda", fuse_k=3)   # exceeds the radius-3 maximum
     with pytest.raises(L.LoraError):
         L.Stencil(synth.preset("heat1d"), (100,), engine="tc")   # no tensor-core 1D engine
+
+
+def test_single_launch_path_selection(L, monkeypatch):
+    """Small 2D star grids (Heat-2D 256^2, BASELINE configs[0]) take the single-launch cluster path;
+    large or non-star plans and LORA_NO_SMALL=1 do not (host-only planning, no GPU needed)."""
+    W, c = synth.config("heat2d-256")
+    assert L.Stencil(W, c["shape"]).info()["single_launch"] == 1
+    assert L.Stencil(W, c["shape"], engine="tc").info()["single_launch"] == 0
+    assert L.Stencil(W, (257, 256)).info()["single_launch"] == 0          # 257 rows: no cluster divides it
+    assert L.Stencil(W, (4096, 4096)).info()["single_launch"] == 0        # does not fit shared memory
+    W2, c2 = synth.config("box2d49p-10240")
+    assert L.Stencil(W2, (256, 256)).info()["single_launch"] == 0         # not a star
+    monkeypatch.setenv("LORA_NO_SMALL", "1")
+    assert L.Stencil(W, c["shape"]).info()["single_launch"] == 0

@@ -40,6 +40,9 @@ def main():
             ops[d["op"]] = d
     load = [s for s in samples if s > 500]
     maxmhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+    med = statistics.median(load) if load else maxmhz
+    for o in ops.values():   # per-SM rate at the NVML clock (the pipe: 64 FP64 lanes/clk/SM)
+        o["lane_ops_per_clk_per_sm_at_nvml_clock"] = o["lane_ops_per_s"] / (med * 1e6) / lines[0]["sms"]
     best = max(o["lane_ops_per_s"] for o in ops.values())
     res = {"what": "FP64 pipe peak on this B200 (tools/ubench/fp64_peak.cu): 16 independent chains per thread, "
                    "2 CTAs x 512 threads per SM, best of 2 runs per op; one DFMA/DADD/DMUL = one FP64 lane-op",

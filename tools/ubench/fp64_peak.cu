@@ -6,7 +6,8 @@
 //   dfma_v : d = fma(d, x, y) with x, y per-thread registers (three vector operands)
 //   dadd   : d = d + a ;  dmul : d = d * a
 // Prints one JSON line per op: FP64 lane-ops/s (one DFMA = one lane-op = 2 flops), elapsed ms
-// (CUDA events), and the SM clock the kernel saw (clock64 cycles / elapsed time).
+// (CUDA events).  The SM clock comes from NVML in tools/fp64_peak.py (clock64 on B200 does not tick at
+// the SM clock: cycles / elapsed time gives ~1.47 GHz while NVML reports 1965 MHz under load).
 // Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o fp64_peak fp64_peak.cu
 #include <cstdio>
 #include <cuda_runtime.h>
@@ -60,10 +61,8 @@ int run(const char* name, int nsm, int iters) {
   avg /= blocks;
   const double lane_ops = 16.0 * iters * (double)blocks * threads;
   const double rate = lane_ops / (ms * 1e-3);
-  const double mhz = avg / (ms * 1e3);
-  printf("{\"op\":\"%s\",\"ms\":%.3f,\"lane_ops_per_s\":%.6e,\"tflops_fma2\":%.3f,\"kernel_mhz\":%.0f,"
-         "\"lane_ops_per_clk_per_sm\":%.2f}\n",
-         name, ms, rate, (OP <= 1 ? 2.0 : 1.0) * rate / 1e12, mhz, rate / (mhz * 1e6) / nsm);
+  printf("{\"op\":\"%s\",\"ms\":%.3f,\"lane_ops_per_s\":%.6e,\"tflops\":%.3f,\"clock64_per_us\":%.0f}\n",
+         name, ms, rate, (OP <= 1 ? 2.0 : 1.0) * rate / 1e12, avg / (ms * 1e3));
   fflush(stdout);
   delete[] h;
   cudaFree(out); cudaFree(cyc);
