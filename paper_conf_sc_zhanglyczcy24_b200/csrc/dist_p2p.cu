@@ -156,8 +156,10 @@ int lora_stencil_p2p_create(lora_p2p** out, const lora_plan* p, int nranks, int 
   c->ndim = p->ndim;
   c->R = p->R;
   c->engine = p->engine;
-  // fused launches: 2D CUDA-core engine only (the 3D fused kernel has no exchange hooks)
-  c->k = (p->ndim == 2 && p->engine == LORA_ENGINE_RDG_CUDA) ? std::max(1, p->fuse_k) : 1;
+  // fused launches: the CUDA-core engine keeps the plan's fusion depth (2D stream kernel, 3D radius-1
+  // fused kernel); the direct comparison kernel steps unfused
+  c->k = (p->engine == LORA_ENGINE_RDG_CUDA && (p->ndim == 2 || (p->ndim == 3 && rdg3d_fused_supported(*p))))
+             ? std::max(1, p->fuse_k) : 1;
   c->H = c->k * p->R;
   if (nranks > 1 && p->N[0] < c->H) {
     delete c;
@@ -383,7 +385,7 @@ int lora_stencil_run_dist_p2p(lora_plan* p, lora_p2p* c, const double* in_local,
   d.store_hi = (int)(c->hl + n0);
   d.lo_end = (int)(c->hl + H);
   d.hi_begin = (int)(c->hl + n0 - H);
-  auto units_of = [&](int kk) { return p->ndim == 2 ? p2p_units_k(v, kk) : U; };
+  auto units_of = [&](int kk) { return p2p_units_k(v, kk); };
   for (int64_t j = 1; j <= L; ++j) {
     const int kk = steps[j - 1];
     d.dst_lo = c->lo.present ? c->lo.buf[j % 2] : nullptr;

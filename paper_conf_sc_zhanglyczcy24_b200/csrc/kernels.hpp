@@ -102,7 +102,9 @@ bool rdg3d_supported(const Plan& p);
 int rdg3d_p2p_units(const Plan& p, int* nux);
 cudaError_t launch_rdg3d_p2p(const Plan& p, const double* src, double* dst, cudaStream_t s, const P2PArgs& d);
 // k = 2, 3 fused 3D steps (radius 1), kernels_rdg3df.cu.
-cudaError_t launch_rdg3d_fused(const Plan& p, const double* src, double* dst, cudaStream_t s, int k);
+cudaError_t launch_rdg3d_fused(const Plan& p, const double* src, double* dst, cudaStream_t s, int k,
+                               const P2PArgs* d = nullptr);
+int rdg3d_fused_units(const Plan& p, int k, int* nux);   // flag units (columns) of the k-fused 3D kernel
 bool rdg3d_fused_supported(const Plan& p);
 bool rdg2d_supported(const Plan& p);
 

@@ -1014,7 +1014,10 @@ int p2p_units(const Plan& p, int* nux) {
 }
 
 cudaError_t launch_step_p2p(const Plan& p, const double* src, double* dst, cudaStream_t s, const P2PArgs& d, int k) {
-  if (p.ndim == 3) return k == 1 ? launch_rdg3d_p2p(p, src, dst, s, d) : cudaErrorNotSupported;
+  if (p.ndim == 3) {
+    if (k == 1) return launch_rdg3d_p2p(p, src, dst, s, d);
+    return p.engine == LORA_ENGINE_RDG_CUDA ? launch_rdg3d_fused(p, src, dst, s, k, &d) : cudaErrorNotSupported;
+  }
   if (p.ndim != 2) return cudaErrorNotSupported;
   if (p.engine == LORA_ENGINE_DIRECT) return k == 1 ? direct2d(p, src, dst, s, &d) : cudaErrorNotSupported;
   if (p.engine != LORA_ENGINE_RDG_CUDA) return cudaErrorNotSupported;
@@ -1042,6 +1045,7 @@ int band_stride(int k) {
 }  // namespace
 
 int p2p_units_k(const Plan& p, int k) {
+  if (p.ndim == 3 && k >= 2) return rdg3d_fused_units(p, k, nullptr);
   if (p.ndim != 2 || k <= 1) return p2p_units(p, nullptr);
   const int bs = p.R == 1 ? band_stride<1>(k) : p.R == 2 ? band_stride<2>(k) : p.R == 3 ? band_stride<3>(k) : band_stride<4>(k);
   return (int)((p.N[1] + bs - 1) / bs);

@@ -225,8 +225,10 @@ __global__ void __launch_bounds__(R3_WARPS * 32, RDG3_MINB) rdg3d_kernel(const d
   // device-initiated exchange: the z-chunk holding the first (last) R interior planes of the slab
   // touches the lower (upper) neighbour (the host keeps it unique per column)
   auto touches = [&](int bz0, bool& lo, bool& hi) {
-    lo = dp.active && dp.dst_lo != nullptr && bz0 < R;
-    hi = dp.active && dp.dst_hi != nullptr && int64_t(bz0) + ZC > N0 - R;
+    // (view padded planes: the chunk's outputs are planes bz0 + R .. bz0 + R + ZC - 1; with a deep-halo
+    // view (fused endpoint, remainder launch) only [store_lo, store_hi) are this rank's)
+    lo = dp.active && dp.dst_lo != nullptr && bz0 + R < dp.lo_end;
+    hi = dp.active && dp.dst_hi != nullptr && int64_t(bz0) + R + ZC > dp.hi_begin;
   };
   auto issue_next = [&](int slot) {
     double* dst = reinterpret_cast<double*>(ring + slot * G::STAGE);
@@ -323,10 +325,10 @@ __global__ void __launch_bounds__(R3_WARPS * 32, RDG3_MINB) rdg3d_kernel(const d
       // output plane zi = (input plane) - 2R is complete: slot (I - 2R) mod n == (I + 1) mod n
       constexpr int s = (I + 1) % n;
       const int zi = cz + cj - 2 * R;
-      if (cj >= 2 * R && zi < zend) {
+      if (cj >= 2 * R && zi < zend && (!dp.active || (zi + R >= dp.store_lo && zi + R < dp.store_hi))) {
         // the plane goes to this slab and, for the first / last R interior planes of a slab with a
         // neighbour there, into that neighbour's halo as well (peer memory, csrc/dist_p2p.cu)
-        const bool rlo = t_lo && zi < R, rhi = t_hi && zi >= N0 - R;
+        const bool rlo = t_lo && zi + R < dp.lo_end, rhi = t_hi && zi + R >= dp.hi_begin;
         const int nd = 1 + (rlo ? 1 : 0) + (rhi ? 1 : 0);
         for (int d = 0; d < nd; ++d) {
           double* o = obase + int64_t(zi) * P1 * P2;
@@ -442,15 +444,19 @@ cudaError_t rdg3d_launch(const Plan& p, const double* src, double* dst, cudaStre
     const int64_t zc2 = (p.N[0] + nch - 1) / nch;
     if (zc2 >= 8 && zc2 <= 2 * R3_ZC && cols * ((p.N[0] + zc2 - 1) / zc2) <= rounds * TWmax) zc = zc2;
   }
-  if (d && d->active && zc < p.N[0]) {
-    // device-initiated exchange: exactly one z-chunk per column may hold the last R interior
-    // planes (the last chunk must have >= R planes)
-    int64_t ok = 0;
-    for (int64_t c = zc; c <= zc + 64 && !ok; ++c) {
-      const int64_t rem = p.N[0] % c;
-      if (rem == 0 || rem >= R) ok = c;
+  if (d && d->active) {
+    // device-initiated exchange: exactly one z-chunk per column and side may touch a neighbour — the
+    // first chunk holds view planes [R, lo_end), the last one starts at or below hi_begin
+    const int64_t N0v = p.N[0], need_lo = d->lo_end - R, need_hi = N0v + R - d->hi_begin;
+    zc = std::max<int64_t>(zc, need_lo);
+    if (zc < N0v) {
+      int64_t ok = 0;
+      for (int64_t c = zc; c <= zc + 64 && !ok; ++c) {
+        const int64_t rem = N0v % c;
+        if ((rem == 0 ? c : rem) >= need_hi) ok = c;
+      }
+      zc = ok ? ok : N0v;
     }
-    zc = ok ? ok : p.N[0];
   }
   const int ZC = (int)zc;
   const int SI = (int)(((ZC + 2 * R) + G::n - 1) / G::n * G::n);

@@ -23,6 +23,7 @@
 #include <vector>
 
 #include "kernels.hpp"
+#include "p2p.cuh"
 #include "pipe.cuh"
 
 namespace lora {
@@ -263,7 +264,8 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
                                                                  int64_t N0, int64_t N1, int64_t N2, int nbx, int nby,
                                                                  int nitems, int ZC, int SI,
                                                                  const __grid_constant__ CUtensorMap tmap,
-                                                                 const __grid_constant__ FParams prm) {
+                                                                 const __grid_constant__ FParams prm,
+                                                                 const __grid_constant__ P2PArgs dp) {
   constexpr int STAGE = ((F_IN * F_BW * 8 + 127) / 128) * 128;
   constexpr int F_NS = SG::ns;
   constexpr int S1B = F_S1 * F_S1W;          // doubles per intermediate plane buffer
@@ -285,17 +287,46 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
   }
   __syncthreads();
   // item -> lane column 0 at padded X0, final rows from padded Y0, final planes from padded Z0
+  const int nbz = nitems / (nbx * nby);
   auto geom = [&](int item, int& X0, int& Y0, int& Z0) {
-    const int bx = item % nbx, rest = item / nbx, by = rest % nby, bz = rest / nby;
+    const int bx = item % nbx, rest = item / nbx, by = rest % nby;
+    const int bz = dp.active ? p2p_chunk_order(rest / nby, nbz) : rest / nby;
     X0 = 1 + bx * BS - (K - 1) - SG1;   // R + b*BS - R(K-1) - SG   (X0 - R even)
     Y0 = 1 + by * TY;
     Z0 = 1 + bz * ZC;
+  };
+  // device-initiated exchange (csrc/dist_p2p.cu; the launch sees the slab buffer as a taller "view"
+  // whose deep-halo planes count as interior): the z-chunk holding the slab's first (last) H own
+  // planes touches the lower (upper) neighbour — it waits for the neighbour's step counter of the
+  // 3 x 3 units around its column before staging, stores those planes into the neighbour's halo as
+  // well, and publishes its own counter when done.  The host keeps that chunk unique per column.
+  auto touches = [&](int Z0_, bool& lo, bool& hi) {
+    lo = dp.active && dp.dst_lo != nullptr && Z0_ < dp.lo_end;
+    hi = dp.active && dp.dst_hi != nullptr && Z0_ + ZC > dp.hi_begin;
   };
   int pitem = blockIdx.x, pj = 0, pX = 0, pY = 0, pZ = 0;
   if (pitem < nitems) geom(pitem, pX, pY, pZ);
   auto issue_next = [&](int slot) {
     double* dst = reinterpret_cast<double*>(ring + slot * STAGE);
     const int x = pX - 1, y = pY - K, z = pZ - K + pj;
+    if (dp.active && pj == 0 && tid == 0) {   // this column's halo planes come from a neighbour
+      bool lo, hi;
+      touches(pZ, lo, hi);
+      if (lo || hi) {
+        if (dp.wait_units > 0) {   // the neighbour's previous launch had another geometry: every unit
+          if (lo) p2p_wait_units(dp.wait_lo, 0, dp.wait_units - 1, dp.wait_val, dp.err);
+          if (hi) p2p_wait_units(dp.wait_hi, 0, dp.wait_units - 1, dp.wait_val, dp.err);
+        } else {
+          const int u = pitem % (nbx * nby), ux = u % nbx, uy = u / nbx;
+          for (int yy = max(uy - 1, 0); yy <= min(uy + 1, nby - 1); ++yy) {
+            const int u0 = yy * nbx + max(ux - 1, 0), u1 = yy * nbx + min(ux + 1, nbx - 1);
+            if (lo) p2p_wait_units(dp.wait_lo, u0, u1, dp.wait_val, dp.err);
+            if (hi) p2p_wait_units(dp.wait_hi, u0, u1, dp.wait_val, dp.err);
+          }
+        }
+        fence_proxy_async_global();
+      }
+    }
     if constexpr (TMA) {  // x even by construction; negative origins are zero-filled by TMA
       if (tid == 0) {
         fence_proxy_async();
@@ -303,6 +334,7 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
         tma_load_3d(dst, &tmap, x, y, z, &bar[slot]);
       }
     } else {  // no TMA (row pitch not a multiple of 16 B): the CTA fills the box itself
+      if (dp.active && pj == 0) __syncthreads();   // after tid 0's wait for the neighbour
       for (int i = tid; i < F_IN * F_BW; i += blockDim.x) {
         const int r = i / F_BW, c = i - r * F_BW;
         const int gy = y + r, gx = x + c;
@@ -323,6 +355,7 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
   double acc[K][3][2][2];
   int citem = blockIdx.x, cj = 0, slot = 0, phase = 0;
   int X0 = 0, Y0 = 0, Z0 = 0, zend = 0;
+  bool t_lo = false, t_hi = false;   // the current item touches the lower / upper neighbour
   const int c0 = 2 * lane;  // lane's first column (relative to X0)
   // per item: intermediate stage S rows/columns of this lane strictly inside (publish fast path);
   // final elements of this lane to store (row / column validity, the z test is per plane)
@@ -336,7 +369,8 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
       else __syncthreads();
       if (cj == 0) {
         geom(citem, X0, Y0, Z0);
-        zend = min(Z0 + ZC, P0 - 1);
+        zend = min(Z0 + ZC, dp.active ? dp.store_hi : P0 - 1);
+        touches(Z0, t_lo, t_hi);
         const bool xs_in = X0 + c0 >= 1 && X0 + c0 + 1 < P2 - 1;
 #pragma unroll
         for (int S = 1; S < K; ++S) {
@@ -401,13 +435,20 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
           // final plane zf = p - K complete: ring slot (IS + 1) % 3
           constexpr int s = (IS + 1) % 3;
           const int zf = p - K;
-          if (cj >= 2 * K && zf >= Z0 && zf < zend) {
-            double* o = out + (int64_t(zf) * P1 + Y0 + 2 * w) * P2 + X0 + c0;
+          if (cj >= 2 * K && zf >= Z0 && zf < zend && (!dp.active || zf >= dp.store_lo)) {
+            // the plane goes to this slab and, for the first / last H own planes of a slab with a
+            // neighbour there, into that neighbour's halo as well (peer memory)
+            const int64_t e0 = (int64_t(zf) * P1 + Y0 + 2 * w) * P2 + X0 + c0;
+            const bool rlo = t_lo && zf < dp.lo_end, rhi = t_hi && zf >= dp.hi_begin;
+            const int nd = 1 + (rlo ? 1 : 0) + (rhi ? 1 : 0);
+            for (int d = 0; d < nd; ++d) {
+              double* o = d == 0 ? out + e0 : ((rlo && d == 1) ? dp.dst_lo + (e0 + dp.off_lo) : dp.dst_hi + (e0 + dp.off_hi));
 #pragma unroll
-            for (int y = 0; y < 2; ++y)
+              for (int y = 0; y < 2; ++y)
 #pragma unroll
-              for (int e = 0; e < 2; ++e)
-                if (st_ok[y][e]) o[y * P2 + e] = acc[K - 1][s][y][e];
+                for (int e = 0; e < 2; ++e)
+                  if (st_ok[y][e]) o[y * P2 + e] = acc[K - 1][s][y][e];
+            }
           }
           if constexpr (!SG::assign0) {
 #pragma unroll
@@ -419,7 +460,17 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
         (stage(std::integral_constant<int, Ss + 2>{}), ...);
       }(std::make_integer_sequence<int, K - 1>{});
       if (++slot == F_NS) { slot = 0; phase ^= 1; }
-      if (++cj == SI) { cj = 0; citem += gridDim.x; }
+      if (++cj == SI) {
+        if (t_lo || t_hi) {   // CTA-uniform: every thread's stores of the item are visible system-wide,
+          __threadfence_system();   // then one release per neighbour
+          __syncthreads();
+          const int u = citem % (nbx * nby);
+          if (tid == 0 && t_lo) p2p_st_release(dp.sig_lo + u, dp.sig_val);
+          if (tid == 0 && t_hi) p2p_st_release(dp.sig_hi + u, dp.sig_val);
+        }
+        cj = 0;
+        citem += gridDim.x;
+      }
     };
     [&]<int... Is>(std::integer_sequence<int, Is...>) {
       (one(std::integral_constant<int, Is>{}), ...);
@@ -469,7 +520,7 @@ bool make_fparams(const Plan& p, FParams& prm) {
 
 template <class SG, int K, bool TMA>
 cudaError_t launch_f(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
-                     const FParams& prm) {
+                     const FParams& prm, const P2PArgs* d) {
   constexpr int STAGE = ((F_IN * F_BW * 8 + 127) / 128) * 128;
   const int smem = 128 + SG::ns * STAGE + 2 * (K - 1) * F_S1 * F_S1W * 8;
   int max_grid = 0;
@@ -477,6 +528,7 @@ cudaError_t launch_f(const Plan& p, const double* src, double* dst, cudaStream_t
     cudaError_t e = kernel_setup((const void*)rdg3df_kernel<SG, K, TMA>, F_WARPS * 32, smem, &max_grid);
     if (e != cudaSuccess) return e;
   }
+  if (d && d->prepare_only) return cudaSuccess;
   constexpr int TY = F_S1 - 2 * (K - 1), BS = 64 - 2 * (K - 1) - 2 * ((K - 1) & 1);
   const int nbx = (int)((p.N[2] + BS - 1) / BS), nby = (int)((p.N[1] + TY - 1) / TY);
   int64_t zc = F_ZC;
@@ -487,18 +539,35 @@ cudaError_t launch_f(const Plan& p, const double* src, double* dst, cudaStream_t
     const int64_t zc2 = (p.N[0] + nch - 1) / nch;
     if (zc2 >= 8 && zc2 <= 2 * F_ZC && cols * ((p.N[0] + zc2 - 1) / zc2) <= rounds * max_grid) zc = zc2;
   }
+  if (d && d->active) {
+    // device-initiated exchange: exactly one z-chunk per column and side may touch a neighbour —
+    // the first chunk holds view planes [1, lo_end) (ZC >= lo_end - 1) and the last one starts at or
+    // below hi_begin (it has >= P0 - 1 - hi_begin planes)
+    const int64_t N0v = p.N[0], need_lo = d->lo_end - 1, need_hi = (N0v + 1) - d->hi_begin;
+    zc = std::max<int64_t>(zc, need_lo);
+    if (zc < N0v) {
+      int64_t ok = 0;
+      for (int64_t c = zc; c <= zc + 64 && !ok; ++c) {
+        const int64_t rem = N0v % c;
+        if ((rem == 0 ? c : rem) >= need_hi) ok = c;
+      }
+      zc = ok ? ok : N0v;
+    }
+  }
   const int ZC = (int)zc;
   const int SI = ((ZC + 2 * K) + 2) / 3 * 3;
   const int nbz = (int)((p.N[0] + ZC - 1) / ZC);
   const int64_t nitems = int64_t(nbx) * nby * nbz;
   const int grid = (int)std::min<int64_t>(max_grid, nitems);
+  static const P2PArgs none{};
   rdg3df_kernel<SG, K, TMA><<<grid, F_WARPS * 32, smem, s>>>(src, dst, p.N[0], p.N[1], p.N[2], nbx, nby, (int)nitems, ZC, SI,
-                                                     map, prm);
+                                                     map, prm, d ? *d : none);
   return cudaGetLastError();
 }
 
 template <int K>
-cudaError_t launch_fk(const Plan& p, const double* src, double* dst, cudaStream_t s, const FParams& prm) {
+cudaError_t launch_fk(const Plan& p, const double* src, double* dst, cudaStream_t s, const FParams& prm,
+                      const P2PArgs* d = nullptr) {
   CUtensorMap map;
   const int64_t padded[3] = {p.P[0], p.P[1], p.P[2]};
   const int box[3] = {1, F_IN, F_BW};
@@ -506,13 +575,13 @@ cudaError_t launch_fk(const Plan& p, const double* src, double* dst, cudaStream_
   if (!tma) std::memset(&map, 0, sizeof(map));
   // specialisations: Box-3D27P-like (PMA planes, z-mirrored) and Heat-3D-like (point / star, mirrored)
   if (prm.mode[0] == PM_PMA1 && prm.mode[1] == PM_PMA1 && prm.mirror[0])
-    return tma ? launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, K, true>(p, src, dst, s, map, prm)
-               : launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, K, false>(p, src, dst, s, map, prm);
+    return tma ? launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, K, true>(p, src, dst, s, map, prm, d)
+               : launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, K, false>(p, src, dst, s, map, prm, d);
   if (prm.mode[0] == PM_POINT && prm.mode[1] == PM_STAR && prm.mirror[0])
-    return tma ? launch_f<Sig3<PM_POINT, PM_STAR, 1>, K, true>(p, src, dst, s, map, prm)
-               : launch_f<Sig3<PM_POINT, PM_STAR, 1>, K, false>(p, src, dst, s, map, prm);
-  return tma ? launch_f<Sig3<-1, -1, -1>, K, true>(p, src, dst, s, map, prm)
-             : launch_f<Sig3<-1, -1, -1>, K, false>(p, src, dst, s, map, prm);
+    return tma ? launch_f<Sig3<PM_POINT, PM_STAR, 1>, K, true>(p, src, dst, s, map, prm, d)
+               : launch_f<Sig3<PM_POINT, PM_STAR, 1>, K, false>(p, src, dst, s, map, prm, d);
+  return tma ? launch_f<Sig3<-1, -1, -1>, K, true>(p, src, dst, s, map, prm, d)
+             : launch_f<Sig3<-1, -1, -1>, K, false>(p, src, dst, s, map, prm, d);
 }
 
 }  // namespace
@@ -522,12 +591,20 @@ bool rdg3d_fused_supported(const Plan& p) {
   return make_fparams(p, prm);
 }
 
-cudaError_t launch_rdg3d_fused(const Plan& p, const double* src, double* dst, cudaStream_t s, int k) {
+cudaError_t launch_rdg3d_fused(const Plan& p, const double* src, double* dst, cudaStream_t s, int k, const P2PArgs* d) {
   FParams prm;
   if (!make_fparams(p, prm)) return cudaErrorNotSupported;
-  if (k == 2) return launch_fk<2>(p, src, dst, s, prm);
-  if (k == 3) return launch_fk<3>(p, src, dst, s, prm);
+  if (k == 2) return launch_fk<2>(p, src, dst, s, prm, d);
+  if (k == 3) return launch_fk<3>(p, src, dst, s, prm, d);
   return cudaErrorNotSupported;
+}
+
+int rdg3d_fused_units(const Plan& p, int k, int* nux) {
+  if (k < 2 || k > 3 || !rdg3d_fused_supported(p)) return 0;
+  const int TY = F_S1 - 2 * (k - 1), BS = 64 - 2 * (k - 1) - 2 * ((k - 1) & 1);
+  const int bx = (int)((p.N[2] + BS - 1) / BS), by = (int)((p.N[1] + TY - 1) / TY);
+  if (nux) *nux = bx;
+  return bx * by;
 }
 
 }  // namespace lora

@@ -93,12 +93,12 @@ class _DevBuf:
                                          "version": 3, "strides": None}
 
 
-def _global(W, g, T, engine):
+def _global(W, g, T, engine, fuse_k=1):
     import torch
     import paper_conf_sc_zhanglyczcy24_b200 as L
     h = (W.shape[0] - 1) // 2
     shape = tuple(s - 2 * h for s in g.shape)
-    st = L.Stencil(W, shape, engine=engine, fuse_k=1)
+    st = L.Stencil(W, shape, engine=engine, fuse_k=fuse_k)
     x = torch.from_numpy(g).cuda()
     y = torch.empty_like(x)
     st.run(x, y, T)
@@ -161,6 +161,36 @@ def test_p2p_fused_deep_halo_bitwise(case):
         assert np.array_equal(out, ref), (T, float(np.nanmax(np.abs(out - ref))))
     out = _run_local(W, g, h, shape, 5, "rdg_cuda", counts, fuse_k=k, repeat=2)
     assert np.array_equal(out, _global(W, g, 5, "rdg_cuda"))
+
+
+FUSED3D = [
+    # kind, global interior shape (z, y, x), slab plane counts, fusion depth k (deep halos H = k)
+    ("rsym", (96, 20, 66), [48, 48], 2),                 # Box-3D27P signature, the planner default k = 2
+    ("heat3d", (130, 12, 40), [64, 2, 64], 2),           # Heat-3D signature; a slab of exactly H planes
+    ("rsym", (64, 33, 130), [16, 16, 16, 16], 2),        # 4 ranks, several x bands / y blocks per slab
+    ("asym", (60, 17, 70), [20, 21, 19], 3),             # general plane signature, k = 3
+    ("rsym", (400, 30, 62), [200, 200], 2),              # several z chunks per column (interior chunks)
+]
+
+
+@pytest.mark.parametrize("case", FUSED3D)
+def test_p2p_fused3d_deep_halo_bitwise(case):
+    """3D: the fused radius-1 kernel (rdg3df, k steps per launch) with the in-kernel exchange: internal
+    slab edges carry H = k deep halo planes, the boundary z-chunks wait on / publish the per-column
+    step counters; T covers remainder launches (the unfused kernel, another column geometry).  Bitwise
+    against the single-GPU run of the global grid at the same fusion depth and unfused."""
+    kind, shape, counts, k = case
+    W = _weights(kind, 3, 1, 47)
+    g = synth.grid(tuple(n + 2 for n in shape), 53)
+    for T in sorted({1, k, k + 1, 2 * k + 1, 6}):
+        ref = _global(W, g, T, "rdg_cuda", fuse_k=k)
+        out = _run_local(W, g, 1, shape, T, "rdg_cuda", counts, fuse_k=k)
+        assert np.array_equal(out, ref), (T, float(np.nanmax(np.abs(out - ref))))
+        assert np.array_equal(ref, _global(W, g, T, "rdg_cuda", fuse_k=1)), T
+    out = _run_local(W, g, 1, shape, 5, "rdg_cuda", counts, fuse_k=k, repeat=2)
+    assert np.array_equal(out, _global(W, g, 5, "rdg_cuda", fuse_k=k))
+    if int(np.prod(shape)) <= 200000:
+        assert rel_err(out, oracle.run(W, g, 5)) <= 1e-12
 
 
 def test_p2p_repeated_runs_and_zero_copy():
