@@ -39,7 +39,11 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="box2d49p-10240")
+    ap.add_argument("--workload", default=None,
+                    help="synth config; default box2d49p-10240 at N = 1, box2d49p-40960 (BASELINE's multi-GPU shape) at N > 1")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="multi-GPU shapes (40960^2, 1024^3): weak = fixed local slab (SURVEY §8(e): 5120 x 40960 / "
+                         "128 x 1024^2, the global shape at N = 8), strong = the global shape split N ways")
     ap.add_argument("--engine", default="auto")
     ap.add_argument("--fuse", type=int, default=0)
     ap.add_argument("--per-stencil", action="store_true", help="also time the other Table II kernels (NEXT-3)")
@@ -198,6 +202,24 @@ def host_info():
 
 
 # ------------------------------------------------------------------ reference arm: the CPU oracle
+# multi-GPU shapes (BASELINE.json configs[4]) and their weak-scaling local slabs
+WEAK_SLAB = {"box2d49p-40960": (5120, 40960), "box3d27p-1024": (128, 1024, 1024)}
+
+
+def local_shape(name, cfg, world, rank, scaling):
+    """This rank's interior slab and the global interior shape.  Multi-GPU configs: weak = the fixed
+    §8(e) slab per rank (global grows with N), strong = the global shape split along the slowest axis
+    (uneven splits allowed).  Other configs: every rank owns the config's shape (weak)."""
+    g = tuple(cfg["shape"])
+    if name in WEAK_SLAB and (world > 1 or scaling == "strong"):
+        if scaling == "weak":
+            loc = WEAK_SLAB[name]
+            return loc, (loc[0] * world,) + tuple(loc[1:])
+        n0 = g[0] // world + (1 if rank < g[0] % world else 0)
+        return (n0,) + g[1:], g
+    return g, (g[0] * world,) + g[1:]
+
+
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -238,6 +260,8 @@ def run_reference(args):
 # ------------------------------------------------------------------ our arm
 def main():
     args = parse()
+    if args.workload is None:
+        args.workload = "box2d49p-40960" if int(os.environ.get("WORLD_SIZE", "1")) > 1 else "box2d49p-10240"
     if args.impl == "reference":
         return run_reference(args)
     import torch
@@ -257,7 +281,7 @@ def main():
     W, cfg = synth.config(args.workload)
     cfg["name"] = args.workload
     h, T = cfg["radius"], cfg["T"]
-    shape = tuple(cfg["shape"])                      # per-rank local interior (weak scaling)
+    shape, gshape = local_shape(args.workload, cfg, world, rank, args.scaling)   # this rank's slab, global grid
     padded = tuple(n + 2 * h for n in shape)
     st = L.Stencil(W, shape, engine=args.engine, fuse_k=args.fuse)
     info = st.info()
@@ -298,16 +322,16 @@ def main():
             uid = b"\0" * L.lora_stencil_comm_id_size()
         comm = L.lora_stencil_comm_init(world, rank, uid)
 
-    # seeded synthetic input (SplitMix64 over the padded array; each rank its own seed offset)
-    g = synth.grid(padded, cfg["seed"] + 1000 * rank)
-    host_in = torch.from_numpy(g).pin_memory()
-    host_out = torch.empty_like(host_in).pin_memory()
-    x = host_in.to(dev)
+    # seeded synthetic input (SplitMix64 over the padded array, generated on the device — bit-identical
+    # to synth.grid; each rank its own seed offset); pinned host copies for the e2e leg
+    x = synth.grid_torch(padded, cfg["seed"] + 1000 * rank, device=dev)
     y = torch.empty_like(x)
+    host_in = x.cpu().pin_memory()
+    host_out = torch.empty_like(host_in).pin_memory()
     stream = torch.cuda.current_stream(dev)
     sptr = stream.cuda_stream
 
-    zero_copy = ep is not None and (info["fuse_k"] == 1 or cfg["ndim"] == 3)
+    zero_copy = ep is not None and info["fuse_k"] == 1
     if zero_copy:
         # zero-copy use of the exchange buffers (unfused launches keep the caller's layout): the slab
         # lives in buffer 0, the result lands in buffer T % 2 (T even: buffer 0 again, so each timed
@@ -353,10 +377,13 @@ def main():
         tt = torch.tensor([t], device=dev, dtype=torch.float64)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         t = float(tt.item())
-    pts_per_step = float(np.prod(shape)) * T * world
+    npts = torch.tensor([float(np.prod(shape))], device=dev, dtype=torch.float64)
+    if world > 1:
+        dist.all_reduce(npts)          # uneven strong-scaling splits: the points all ranks processed
+    pts_per_step = float(npts.item()) * T
     value = pts_per_step * args.steps / t / 1e9
-    # the NCCL path steps unfused; the P2P path runs the plan's fused depth in 2D (deep halos)
-    fuse = 1 if (comm is not None or (ep is not None and cfg["ndim"] == 3)) else info["fuse_k"]
+    # the NCCL path steps unfused; the P2P path runs the plan's fused depth (deep halos, 2D and 3D)
+    fuse = 1 if comm is not None else info["fuse_k"]
     launches_per_step = -(-T // fuse) + 2      # stencil launches + 2 halo-copy launches
     if ep is not None:   # ceil(T/k) stencil launches + 1 halo copy + per neighbour: 2 publish, 2 wait, 1 push
         nb = (1 if rank > 0 else 0) + (1 if rank < world - 1 else 0)
@@ -414,6 +441,64 @@ def main():
                "serial": {"value": pts_per_step * args.steps / te_serial / 1e9,
                           "api": "lora_stencil_run_host, one synchronous call per step"},
                "clock": "host wall clock around the K steps"}
+    elif not args.no_e2e:
+        # multi-GPU e2e: every step copies this rank's slab in from pinned host memory, runs the
+        # distributed sweep (the exchange path of the timed region) and copies the result back; host
+        # wall clock, max over ranks
+        nbytes = host_in.numel() * 8
+        xin, yout = x.data_ptr(), y.data_ptr()
+
+        def dstep():
+            x.copy_(host_in, non_blocking=True)
+            if ep is not None:
+                L.lora_stencil_run_dist_p2p(st.plan, ep, xin, yout, T, sptr)
+            else:
+                L.lora_stencil_run_dist(st.plan, comm, xin, yout, T, sptr)
+            host_out.copy_(y, non_blocking=True)
+        dstep()
+        torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            dstep()
+        torch.cuda.synchronize(dev)
+        te = torch.tensor([time.perf_counter() - t0], device=dev, dtype=torch.float64)
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e = {"value": pts_per_step * args.steps / float(te.item()) / 1e9, "unit": UNIT, "h2d_bytes_per_step": nbytes,
+               "d2h_bytes_per_step": nbytes,
+               "api": "torch copy_ from pinned host -> lora_stencil_run_dist" + ("_p2p" if ep is not None else "") +
+                      " -> copy_ to pinned host, per rank, one stream",
+               "clock": "host wall clock around the K steps, max over ranks"}
+
+    # multi-GPU: the single-GPU run the efficiency is measured against (rank 0, no exchange): weak = the
+    # same local slab on one GPU, strong = the whole global grid on one GPU
+    scaling_check = None
+    if (world > 1 or args.force_dist) and rank == 0:
+        ref_shape = shape if (args.scaling == "weak" or args.workload not in WEAK_SLAB) else gshape
+        s1 = L.Stencil(W, ref_shape, engine=args.engine, fuse_k=args.fuse)
+        x1 = synth.grid_torch(tuple(n + 2 * h for n in ref_shape), cfg["seed"], device=dev)
+        y1 = torch.empty_like(x1)
+        L.lora_stencil_run(s1.plan, x1.data_ptr(), y1.data_ptr(), T, sptr)
+        torch.cuda.synchronize(dev)
+        b0, b1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        b0.record(stream)
+        for _ in range(max(2, min(args.steps, 5))):
+            L.lora_stencil_run(s1.plan, x1.data_ptr(), y1.data_ptr(), T, sptr)
+        b1.record(stream)
+        torch.cuda.synchronize(dev)
+        t1 = b0.elapsed_time(b1) / 1e3 / max(2, min(args.steps, 5))
+        v1 = float(np.prod(ref_shape)) * T / t1 / 1e9
+        scaling_check = {"single_gpu_value": v1, "single_gpu_grid": list(ref_shape), "scaling": args.scaling,
+                         "efficiency": value / (world * v1),
+                         "note": "weak: value / (N x one GPU on the same local slab); strong: value / (N x one GPU on "
+                                 "the global grid) — informational, the driver computes its own from the per-N values"}
+        s1.close()
+        del x1, y1
+        torch.cuda.empty_cache()
+    if world > 1:
+        dist.barrier()
 
     # per-config records: every BASELINE single-GPU config (configs[0..3]), planner defaults, seeded
     # SplitMix64 inputs generated on the device (bit-identical to synth.grid), CUDA events around each
@@ -509,10 +594,10 @@ def main():
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": 1e3 * t / args.steps, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "scaling": args.scaling if args.workload in WEAK_SLAB else "weak", "vs_baseline": None, "dtype": "f64",
                 "data": "synthetic: SplitMix64 grid in [0.5,1.5) over the padded array, seeded radially symmetric weights",
                 "config": {"workload": args.workload, "grid_per_rank": list(shape), "T": T, "radius": h,
-                           "ndim": cfg["ndim"], "global_grid": [shape[0] * world] + list(shape[1:]),
+                           "ndim": cfg["ndim"], "global_grid": list(gshape),
                            "engine": info["engine_name"], "fuse_k": fuse, "n_terms": info["n_terms"],
                            "parallelism": f"slab{world}" if (comm is not None or ep is not None) else "single",
                            "exchange": exchange,
@@ -524,6 +609,8 @@ def main():
                 "host": host_info()}
         if per_config:
             line["configs"] = per_config
+        if scaling_check:
+            line["scaling_check"] = scaling_check
         if engines:
             line["engines"] = engines
         print(json.dumps(line), flush=True)

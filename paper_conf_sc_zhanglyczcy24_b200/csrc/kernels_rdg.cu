@@ -133,9 +133,10 @@ __device__ __forceinline__ void row_compute(const double (&x)[2 * R + 2], double
     acc[s0][1] = fma(P.c, x[R + 1], acc[s0][1]);
   } else if constexpr (SIG == SIG_ROWS) {
     // row-pair rank-1 split of a doubly reflection-symmetric W (Plan::rdg_rows): term a has
-    // u_a = e_{R+a} + e_{R-a} and v_a = W[R+a,:] (palindromic), so the horizontal gather is
-    // v_a[0] x_0 + sum_b v_a[b] (x_{-b} + x_{+b}) on the shared pair sums and the vertical gather
-    // is one add into each of the (at most two) output rows R+a, R-a away.
+    // u_a = c_a (e_{R+a} + e_{R-a}) and v_a = W[R+a,:] / c_a with c_a = W[R+a,R] (unit centre tap),
+    // so the horizontal gather is t_a = x_0 + sum_b v_a[b] (x_{-b} + x_{+b}) on the shared pair
+    // sums (R DFMA, no DMUL) and the vertical gather is one DFMA c_a t_a into each of the (at most
+    // two) output rows R+a, R-a away; the first term of an output row is the product c_R t_R.
     double sp0[R + 1], sp1[R + 1];
 #pragma unroll
     for (int b = 1; b <= R; ++b) {
@@ -144,22 +145,23 @@ __device__ __forceinline__ void row_compute(const double (&x)[2 * R + 2], double
     }
 #pragma unroll
     for (int a = 0; a <= R; ++a) {
-      double t0 = P.v[a][R] * x[R], t1 = P.v[a][R] * x[R + 1];
+      double t0 = x[R], t1 = x[R + 1];   // v_a[R] == 1
 #pragma unroll
       for (int b = 1; b <= R; ++b) {
         t0 = fma(P.v[a][R + b], sp0[b], t0);
         t1 = fma(P.v[a][R + b], sp1[b], t1);
       }
+      const double ca = P.u[a][0];
       const int s = pmod(I - R - a, n);
-      acc[s][0] += t0;
-      acc[s][1] += t1;
+      acc[s][0] = fma(ca, t0, acc[s][0]);
+      acc[s][1] = fma(ca, t1, acc[s][1]);
       if (a == R) {   // slot I mod n was emptied after the previous row: this is its first term
-        acc[pmod(I, n)][0] = t0;
-        acc[pmod(I, n)][1] = t1;
+        acc[pmod(I, n)][0] = ca * t0;
+        acc[pmod(I, n)][1] = ca * t1;
       } else if (a > 0) {
         const int s2 = pmod(I - R + a, n);
-        acc[s2][0] += t0;
-        acc[s2][1] += t1;
+        acc[s2][0] = fma(ca, t0, acc[s2][0]);
+        acc[s2][1] = fma(ca, t1, acc[s2][1]);
       }
     }
   } else if constexpr (SIG == SIG_STAR) {
@@ -235,7 +237,7 @@ __device__ __forceinline__ void row_shift(const double (&x)[2 * R + 2], double (
     double t[R + 1][2];
 #pragma unroll
     for (int a = 0; a <= R; ++a) {
-      double t0 = P.v[a][R] * x[R], t1 = P.v[a][R] * x[R + 1];
+      double t0 = x[R], t1 = x[R + 1];   // unit centre tap (row_compute SIG_ROWS)
 #pragma unroll
       for (int b = 1; b <= R; ++b) {
         t0 = fma(P.v[a][R + b], sp0[b], t0);
@@ -247,11 +249,11 @@ __device__ __forceinline__ void row_shift(const double (&x)[2 * R + 2], double (
 #pragma unroll
     for (int j = 0; j < 2 * R; ++j) {
       const int a = j < R ? R - j : j - R;
-      p[j][0] = p[j + 1][0] + t[a][0];
-      p[j][1] = p[j + 1][1] + t[a][1];
+      p[j][0] = fma(P.u[a][0], t[a][0], p[j + 1][0]);
+      p[j][1] = fma(P.u[a][0], t[a][1], p[j + 1][1]);
     }
-    p[2 * R][0] = t[R][0];
-    p[2 * R][1] = t[R][1];
+    p[2 * R][0] = P.u[R][0] * t[R][0];
+    p[2 * R][1] = P.u[R][0] * t[R][1];
   } else if constexpr (SIG == SIG_PMA) {
     double t[R][2];
 #pragma unroll
@@ -818,9 +820,14 @@ int signature(const Plan& p, RdgParams& prm) {
   std::memset(&prm, 0, sizeof(prm));
   const int R = p.R, n = 2 * R + 1;
   if (p.rdg_rows && p.ndim == 2) {
+    // row pairs with a unit centre tap: v_a = W[R+a,:] / c_a, c_a = W[R+a,R] (nonzero: planner.cpp)
     prm.K = R + 1;
-    for (int a = 0; a <= R; ++a)
-      for (int j = 0; j < n; ++j) prm.v[a][j] = p.W[size_t(R + a) * n + j];
+    for (int a = 0; a <= R; ++a) {
+      const double ca = p.W[size_t(R + a) * n + R];
+      for (int j = 0; j < n; ++j) prm.v[a][j] = p.W[size_t(R + a) * n + j] / ca;
+      prm.v[a][R] = 1.0;
+      prm.u[a][0] = ca;
+    }
     return SIG_ROWS;
   }
   // PMA pyramid: chains of radius R, R-1, ..., 1 (in that order) + centre scalar

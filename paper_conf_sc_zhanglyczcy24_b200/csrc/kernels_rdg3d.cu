@@ -237,11 +237,17 @@ __global__ void __launch_bounds__(R3_WARPS * 32, RDG3_MINB) rdg3d_kernel(const d
       bool lo, hi;
       touches(pz, lo, hi);
       if (lane == 0 && (lo || hi)) {
-        const int u = pitem % (nbx * nby), ux = u % nbx, uy = u / nbx;
-        for (int yy = max(uy - 1, 0); yy <= min(uy + 1, nby - 1); ++yy) {
-          const int u0 = yy * nbx + max(ux - 1, 0), u1 = yy * nbx + min(ux + 1, nbx - 1);
-          if (lo) p2p_wait_units(dp.wait_lo, u0, u1, dp.wait_val, dp.err);
-          if (hi) p2p_wait_units(dp.wait_hi, u0, u1, dp.wait_val, dp.err);
+        if (dp.wait_units > 0) {   // the neighbour's previous launch had another geometry (the fused
+                                   // kernel before a remainder launch): wait on every unit it signalled
+          if (lo) p2p_wait_units(dp.wait_lo, 0, dp.wait_units - 1, dp.wait_val, dp.err);
+          if (hi) p2p_wait_units(dp.wait_hi, 0, dp.wait_units - 1, dp.wait_val, dp.err);
+        } else {
+          const int u = pitem % (nbx * nby), ux = u % nbx, uy = u / nbx;
+          for (int yy = max(uy - 1, 0); yy <= min(uy + 1, nby - 1); ++yy) {
+            const int u0 = yy * nbx + max(ux - 1, 0), u1 = yy * nbx + min(ux + 1, nbx - 1);
+            if (lo) p2p_wait_units(dp.wait_lo, u0, u1, dp.wait_val, dp.err);
+            if (hi) p2p_wait_units(dp.wait_hi, u0, u1, dp.wait_val, dp.err);
+          }
         }
         fence_proxy_async_global();
       }

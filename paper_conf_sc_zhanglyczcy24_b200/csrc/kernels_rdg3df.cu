@@ -256,7 +256,7 @@ __device__ __forceinline__ void publish_ip(double (&acc)[K][3][2][2], double* __
 
 // K fused steps (K = 2, 3).  Stage s computes 16 - 2(s-1) rows (warps w < 8 - (s-1)); final rows
 // TY = 16 - 2(K-1); one __syncthreads per stage boundary per plane.
-template <class SG, int K, bool TMA>
+template <class SG, int K, bool TMA, bool P2P>
 #ifndef RDG3F_MINB
 #define RDG3F_MINB 2
 #endif
@@ -288,9 +288,11 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
   __syncthreads();
   // item -> lane column 0 at padded X0, final rows from padded Y0, final planes from padded Z0
   const int nbz = nitems / (nbx * nby);
+  // P2P: the instantiation with the exchange hooks (single-GPU launches use P2P = false: no hook code)
+  const bool act = P2P && dp.active;
   auto geom = [&](int item, int& X0, int& Y0, int& Z0) {
     const int bx = item % nbx, rest = item / nbx, by = rest % nby;
-    const int bz = dp.active ? p2p_chunk_order(rest / nby, nbz) : rest / nby;
+    const int bz = act ? p2p_chunk_order(rest / nby, nbz) : rest / nby;
     X0 = 1 + bx * BS - (K - 1) - SG1;   // R + b*BS - R(K-1) - SG   (X0 - R even)
     Y0 = 1 + by * TY;
     Z0 = 1 + bz * ZC;
@@ -301,15 +303,15 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
   // 3 x 3 units around its column before staging, stores those planes into the neighbour's halo as
   // well, and publishes its own counter when done.  The host keeps that chunk unique per column.
   auto touches = [&](int Z0_, bool& lo, bool& hi) {
-    lo = dp.active && dp.dst_lo != nullptr && Z0_ < dp.lo_end;
-    hi = dp.active && dp.dst_hi != nullptr && Z0_ + ZC > dp.hi_begin;
+    lo = act && dp.dst_lo != nullptr && Z0_ < dp.lo_end;
+    hi = act && dp.dst_hi != nullptr && Z0_ + ZC > dp.hi_begin;
   };
   int pitem = blockIdx.x, pj = 0, pX = 0, pY = 0, pZ = 0;
   if (pitem < nitems) geom(pitem, pX, pY, pZ);
   auto issue_next = [&](int slot) {
     double* dst = reinterpret_cast<double*>(ring + slot * STAGE);
     const int x = pX - 1, y = pY - K, z = pZ - K + pj;
-    if (dp.active && pj == 0 && tid == 0) {   // this column's halo planes come from a neighbour
+    if (act && pj == 0 && tid == 0) {   // this column's halo planes come from a neighbour
       bool lo, hi;
       touches(pZ, lo, hi);
       if (lo || hi) {
@@ -334,7 +336,7 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
         tma_load_3d(dst, &tmap, x, y, z, &bar[slot]);
       }
     } else {  // no TMA (row pitch not a multiple of 16 B): the CTA fills the box itself
-      if (dp.active && pj == 0) __syncthreads();   // after tid 0's wait for the neighbour
+      if (act && pj == 0) __syncthreads();   // after tid 0's wait for the neighbour
       for (int i = tid; i < F_IN * F_BW; i += blockDim.x) {
         const int r = i / F_BW, c = i - r * F_BW;
         const int gy = y + r, gx = x + c;
@@ -369,7 +371,7 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
       else __syncthreads();
       if (cj == 0) {
         geom(citem, X0, Y0, Z0);
-        zend = min(Z0 + ZC, dp.active ? dp.store_hi : P0 - 1);
+        zend = min(Z0 + ZC, act ? dp.store_hi : P0 - 1);
         touches(Z0, t_lo, t_hi);
         const bool xs_in = X0 + c0 >= 1 && X0 + c0 + 1 < P2 - 1;
 #pragma unroll
@@ -435,7 +437,7 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
           // final plane zf = p - K complete: ring slot (IS + 1) % 3
           constexpr int s = (IS + 1) % 3;
           const int zf = p - K;
-          if (cj >= 2 * K && zf >= Z0 && zf < zend && (!dp.active || zf >= dp.store_lo)) {
+          if (cj >= 2 * K && zf >= Z0 && zf < zend && (!act || zf >= dp.store_lo)) {
             // the plane goes to this slab and, for the first / last H own planes of a slab with a
             // neighbour there, into that neighbour's halo as well (peer memory)
             const int64_t e0 = (int64_t(zf) * P1 + Y0 + 2 * w) * P2 + X0 + c0;
@@ -518,14 +520,14 @@ bool make_fparams(const Plan& p, FParams& prm) {
   return true;
 }
 
-template <class SG, int K, bool TMA>
+template <class SG, int K, bool TMA, bool P2P>
 cudaError_t launch_f(const Plan& p, const double* src, double* dst, cudaStream_t s, const CUtensorMap& map,
                      const FParams& prm, const P2PArgs* d) {
   constexpr int STAGE = ((F_IN * F_BW * 8 + 127) / 128) * 128;
   const int smem = 128 + SG::ns * STAGE + 2 * (K - 1) * F_S1 * F_S1W * 8;
   int max_grid = 0;
   {
-    cudaError_t e = kernel_setup((const void*)rdg3df_kernel<SG, K, TMA>, F_WARPS * 32, smem, &max_grid);
+    cudaError_t e = kernel_setup((const void*)rdg3df_kernel<SG, K, TMA, P2P>, F_WARPS * 32, smem, &max_grid);
     if (e != cudaSuccess) return e;
   }
   if (d && d->prepare_only) return cudaSuccess;
@@ -560,12 +562,12 @@ cudaError_t launch_f(const Plan& p, const double* src, double* dst, cudaStream_t
   const int64_t nitems = int64_t(nbx) * nby * nbz;
   const int grid = (int)std::min<int64_t>(max_grid, nitems);
   static const P2PArgs none{};
-  rdg3df_kernel<SG, K, TMA><<<grid, F_WARPS * 32, smem, s>>>(src, dst, p.N[0], p.N[1], p.N[2], nbx, nby, (int)nitems, ZC, SI,
+  rdg3df_kernel<SG, K, TMA, P2P><<<grid, F_WARPS * 32, smem, s>>>(src, dst, p.N[0], p.N[1], p.N[2], nbx, nby, (int)nitems, ZC, SI,
                                                      map, prm, d ? *d : none);
   return cudaGetLastError();
 }
 
-template <int K>
+template <int K, bool P2P>
 cudaError_t launch_fk(const Plan& p, const double* src, double* dst, cudaStream_t s, const FParams& prm,
                       const P2PArgs* d = nullptr) {
   CUtensorMap map;
@@ -575,13 +577,13 @@ cudaError_t launch_fk(const Plan& p, const double* src, double* dst, cudaStream_
   if (!tma) std::memset(&map, 0, sizeof(map));
   // specialisations: Box-3D27P-like (PMA planes, z-mirrored) and Heat-3D-like (point / star, mirrored)
   if (prm.mode[0] == PM_PMA1 && prm.mode[1] == PM_PMA1 && prm.mirror[0])
-    return tma ? launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, K, true>(p, src, dst, s, map, prm, d)
-               : launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, K, false>(p, src, dst, s, map, prm, d);
+    return tma ? launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, K, true, P2P>(p, src, dst, s, map, prm, d)
+               : launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, K, false, P2P>(p, src, dst, s, map, prm, d);
   if (prm.mode[0] == PM_POINT && prm.mode[1] == PM_STAR && prm.mirror[0])
-    return tma ? launch_f<Sig3<PM_POINT, PM_STAR, 1>, K, true>(p, src, dst, s, map, prm, d)
-               : launch_f<Sig3<PM_POINT, PM_STAR, 1>, K, false>(p, src, dst, s, map, prm, d);
-  return tma ? launch_f<Sig3<-1, -1, -1>, K, true>(p, src, dst, s, map, prm, d)
-             : launch_f<Sig3<-1, -1, -1>, K, false>(p, src, dst, s, map, prm, d);
+    return tma ? launch_f<Sig3<PM_POINT, PM_STAR, 1>, K, true, P2P>(p, src, dst, s, map, prm, d)
+               : launch_f<Sig3<PM_POINT, PM_STAR, 1>, K, false, P2P>(p, src, dst, s, map, prm, d);
+  return tma ? launch_f<Sig3<-1, -1, -1>, K, true, P2P>(p, src, dst, s, map, prm, d)
+             : launch_f<Sig3<-1, -1, -1>, K, false, P2P>(p, src, dst, s, map, prm, d);
 }
 
 }  // namespace
@@ -594,8 +596,13 @@ bool rdg3d_fused_supported(const Plan& p) {
 cudaError_t launch_rdg3d_fused(const Plan& p, const double* src, double* dst, cudaStream_t s, int k, const P2PArgs* d) {
   FParams prm;
   if (!make_fparams(p, prm)) return cudaErrorNotSupported;
-  if (k == 2) return launch_fk<2>(p, src, dst, s, prm, d);
-  if (k == 3) return launch_fk<3>(p, src, dst, s, prm, d);
+  if (d) {
+    if (k == 2) return launch_fk<2, true>(p, src, dst, s, prm, d);
+    if (k == 3) return launch_fk<3, true>(p, src, dst, s, prm, d);
+  } else {
+    if (k == 2) return launch_fk<2, false>(p, src, dst, s, prm, nullptr);
+    if (k == 3) return launch_fk<3, false>(p, src, dst, s, prm, nullptr);
+  }
   return cudaErrorNotSupported;
 }
 

@@ -20,6 +20,7 @@
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdlib>
 #include <cstring>
 #include <map>
@@ -38,63 +39,85 @@ struct StarArms {
   double v[kMaxN];   // vertical arm (u of term 1; its centre is 0 when the horizontal arm has it)
 };
 
+// Buffer row j of CTA c holds padded row c*rp + R - HK + j (HK = k R: the halo depth of a block of
+// k steps); own rows are j in [HK, HK + rp).  Rows outside the array are zero and never feed a
+// stored value; rows of the global Dirichlet halo are loaded into both buffers and never written.
 template <int R>
 __global__ void __launch_bounds__(SM_TX * SM_TY, 1)
-small2d_star_kernel(const double* __restrict__ in, double* __restrict__ out, int N0, int N1, int rp, int T,
+small2d_star_kernel(const double* __restrict__ in, double* __restrict__ out, int N0, int N1, int rp, int T, int kb,
                     const __grid_constant__ StarArms w) {
   cg::cluster_group cl = cg::this_cluster();
   const int c = (int)cl.block_rank(), CS = (int)cl.num_blocks();
   extern __shared__ __align__(16) double sm[];
-  const int P1 = N1 + 2 * R, SR = rp + 2 * R;
-  double* buf0 = sm;
-  double* buf1 = sm + size_t(SR) * P1;
-  const int tid = threadIdx.y * SM_TX + threadIdx.x;
-  const int64_t g0 = int64_t(c) * rp;   // padded row of buffer row 0 (own rows are buffer rows R .. R+rp-1)
-  // stage the slab (own rows + R halo rows each side, all columns) into both buffers
-  const double* src = in + g0 * P1;
-  for (int i = tid; i < SR * P1; i += SM_TX * SM_TY) {
-    const double v = src[i];
+  const int P1 = N1 + 2 * R, P0 = N0 + 2 * R, HK = kb * R, SR = rp + 2 * HK;
+  double* const buf0 = sm;
+  double* const buf1 = sm + size_t(SR) * P1;
+  double* mbox = sm + 2 * size_t(SR) * P1;   // [parity][side 0: from c-1 (top), 1: from c+1 (bottom)][HK][P1]
+  const size_t MB = size_t(HK) * P1;
+  const int tid = threadIdx.y * SM_TX + threadIdx.x, NT = SM_TX * SM_TY;
+  const int pr0 = c * rp + R - HK;          // padded row of buffer row 0
+  for (int i = tid; i < SR * P1; i += NT) {
+    const int pr = pr0 + i / P1;
+    const double v = (pr >= 0 && pr < P0) ? in[int64_t(pr0) * P1 + i] : 0.0;
     buf0[i] = v;
     buf1[i] = v;
   }
-  // neighbours' buffers (DSMEM): my first R own rows are rows rp+R.. of CTA c-1, my last R own
-  // rows are rows 0..R-1 of CTA c+1
-  double* lo0 = c > 0 ? cl.map_shared_rank(buf0, c - 1) : nullptr;
-  double* lo1 = c > 0 ? cl.map_shared_rank(buf1, c - 1) : nullptr;
-  double* hi0 = c < CS - 1 ? cl.map_shared_rank(buf0, c + 1) : nullptr;
-  double* hi1 = c < CS - 1 ? cl.map_shared_rank(buf1, c + 1) : nullptr;
-  cl.sync();   // every CTA staged its slab before anyone stores into a neighbour's halo
-  for (int t = 0; t < T; ++t) {
-    const double* cur = (t & 1) ? buf1 : buf0;
-    double* nxt = (t & 1) ? buf0 : buf1;
-    double* lo = (t & 1) ? lo0 : lo1;
-    double* hi = (t & 1) ? hi0 : hi1;
-    for (int j = R + threadIdx.y; j < R + rp; j += SM_TY) {
-      for (int x = R + threadIdx.x; x < R + N1; x += SM_TX) {
-        const double* cx = cur + size_t(j) * P1 + x;
-        double th = 0.0;
+  // the neighbours' mailboxes (DSMEM): my first HK own rows fill the bottom side of CTA c-1's, my
+  // last HK own rows the top side of CTA c+1's
+  double* lo_mb = c > 0 ? cl.map_shared_rank(mbox, c - 1) : nullptr;
+  double* hi_mb = c < CS - 1 ? cl.map_shared_rank(mbox, c + 1) : nullptr;
+  const int jlo = max(R, R - pr0), jhi = min(SR - R, P0 - R - pr0);   // buffer rows inside the interior
+  cl.sync();   // every CTA staged its slab before any mailbox store
+  int cur = 0;
+  for (int t0 = 0, blk = 0; t0 < T; t0 += kb, ++blk) {
+    const int ks = min(kb, T - t0);
+    const int par = blk & 1;
+    for (int st = 1; st <= ks; ++st) {
+      const double* src = cur ? buf1 : buf0;
+      double* dst = cur ? buf0 : buf1;
+      const bool last = st == ks;
+      // rows valid after this step: shrink by R per step from the block's HK-deep halo
+      const int j0 = max(jlo, R * st + (HK - R * ks)), j1 = min(jhi, SR - R * st - (HK - R * ks));
+      for (int j = j0 + threadIdx.y; j < j1; j += SM_TY) {
+        const bool to_lo = last && lo_mb && j >= HK && j < 2 * HK;               // my first HK own rows
+        const bool to_hi = last && hi_mb && j >= rp && j < rp + HK;               // my last HK own rows
+        for (int x = R + threadIdx.x; x < R + N1; x += SM_TX) {
+          const double* cx = src + size_t(j) * P1 + x;
+          double th = 0.0;
 #pragma unroll
-        for (int b = -R; b <= R; ++b) th = fma(w.h[R + b], cx[b], th);
-        double acc = 0.0;
+          for (int b = -R; b <= R; ++b) th = fma(w.h[R + b], cx[b], th);
+          double acc = 0.0;
 #pragma unroll
-        for (int a = -R; a <= R; ++a) {
-          if (a == 0) acc += th;
-          acc = fma(w.v[R + a], cx[a * P1], acc);
+          for (int a = -R; a <= R; ++a) {
+            if (a == 0) acc += th;
+            acc = fma(w.v[R + a], cx[a * P1], acc);
+          }
+          dst[size_t(j) * P1 + x] = acc;
+          if (to_lo) lo_mb[(2 * par + 1) * MB + size_t(j - HK) * P1 + x] = acc;
+          if (to_hi) hi_mb[(2 * par + 0) * MB + size_t(j - rp) * P1 + x] = acc;
         }
-        nxt[size_t(j) * P1 + x] = acc;
-        if (lo && j < 2 * R) lo[size_t(rp + j) * P1 + x] = acc;
-        if (hi && j >= rp) hi[size_t(j - rp) * P1 + x] = acc;
       }
+      cur ^= 1;
+      if (!last) __syncthreads();
     }
-    cl.sync();   // release my rows (local and remote), acquire the neighbours' rows of my halo
+    cl.sync();   // release my mailbox stores, acquire the neighbours' rows of my halo
+    if (t0 + ks < T) {   // unpack the mailbox into the halo rows of the block's result buffer
+      // (interior columns only: the column halo of every row is the fixed Dirichlet value loaded at
+      // the start, and the mailbox holds only the columns the neighbour computed)
+      double* dst = cur ? buf1 : buf0;
+      for (int j = threadIdx.y; j < HK; j += SM_TY)
+        for (int x = R + threadIdx.x; x < R + N1; x += SM_TX) {
+          if (c > 0) dst[size_t(j) * P1 + x] = mbox[(2 * par + 0) * MB + size_t(j) * P1 + x];
+          if (c < CS - 1) dst[size_t(HK + rp + j) * P1 + x] = mbox[(2 * par + 1) * MB + size_t(j) * P1 + x];
+        }
+      __syncthreads();
+    }
   }
   // write back: own rows (all columns: the column halo is the input's), plus the grid's top / bottom
   // halo rows from the first / last CTA
-  const double* res = (T & 1) ? buf1 : buf0;
-  const int j0 = c == 0 ? 0 : R, j1 = c == CS - 1 ? SR : R + rp;
-  double* dst = out + g0 * P1;
-  for (int i = j0 * P1 + tid; i < j1 * P1; i += SM_TX * SM_TY) dst[i] = res[i];
-  (void)N0;
+  const double* res = cur ? buf1 : buf0;
+  const int w0 = c == 0 ? HK - R : HK, w1 = c == CS - 1 ? HK + rp + R : HK + rp;
+  for (int i = w0 * P1 + tid; i < w1 * P1; i += NT) out[int64_t(pr0) * P1 + i] = res[i];
 }
 
 // The two-arm star signature of the streaming engine (kernels_rdg.cu signature(), SIG_STAR).
@@ -127,17 +150,29 @@ const void* kernel_for(int R) {
 }
 
 constexpr size_t kMaxSmem = 227 * 1024;
+constexpr int kMaxBlock = 8;   // steps per exchange (redundant halo rows grow with it)
+
+// Shared memory of one CTA: two slab buffers of rp + 2kR rows plus the double-buffered two-sided
+// mailbox of kR rows.
+size_t smem_bytes(const Plan& p, int64_t rp, int k) {
+  const size_t P1 = size_t(p.P[1]), HK = size_t(k) * p.R;
+  return (2 * (size_t(rp) + 2 * HK) * P1 + 4 * HK * P1) * sizeof(double);
+}
+
+// Steps per exchange for cluster size cs: the largest k <= kMaxBlock with kR <= rp that fits.
+int block_steps(const Plan& p, int cs) {
+  if (p.N[0] % cs) return 0;
+  const int64_t rp = p.N[0] / cs;
+  for (int k = kMaxBlock; k >= 1; --k)
+    if (int64_t(k) * p.R <= rp && smem_bytes(p, rp, k) <= kMaxSmem) return k;
+  return 0;
+}
 
 // Cluster size for the plan: the largest CS in {16, 8, 4, 2} that divides N0 with >= R rows per CTA
-// and whose slab pair fits the shared memory of one CTA; 0 = the plan does not fit.
+// and whose buffers fit the shared memory of one CTA; 0 = the plan does not fit.
 int cluster_size(const Plan& p) {
-  for (int cs : {16, 8, 4, 2}) {
-    if (p.N[0] % cs) continue;
-    const int64_t rp = p.N[0] / cs;
-    if (rp < p.R) continue;
-    const size_t smem = 2 * size_t(rp + 2 * p.R) * size_t(p.P[1]) * sizeof(double);
-    if (smem <= kMaxSmem) return cs;
-  }
+  for (int cs : {16, 8, 4, 2})
+    if (block_steps(p, cs) > 0) return cs;
   return 0;
 }
 
@@ -193,12 +228,11 @@ cudaError_t launch_small2d(const Plan& p, const double* in, double* out, int64_t
   if (cs == 0) return cudaErrorInvalidValue;
   const void* k = kernel_for(p.R);
   // fall back to smaller clusters if the device cannot schedule this one
-  while (cs >= 2 && setup(k, 2 * size_t(p.N[0] / cs + 2 * p.R) * size_t(p.P[1]) * 8, cs) == 0) {
-    do { cs /= 2; } while (cs >= 2 && p.N[0] % cs);
-  }
+  while (cs >= 2 && (block_steps(p, cs) == 0 || setup(k, kMaxSmem, cs) == 0)) cs /= 2;
   if (cs < 2) return cudaErrorNotSupported;
   const int rp = (int)(p.N[0] / cs);
-  const size_t smem = 2 * size_t(rp + 2 * p.R) * size_t(p.P[1]) * sizeof(double);
+  const int kb = (int)std::min<int64_t>(block_steps(p, cs), T);
+  const size_t smem = smem_bytes(p, rp, kb);
   if (smem > kMaxSmem) return cudaErrorNotSupported;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(cs, 1, 1);
@@ -212,10 +246,10 @@ cudaError_t launch_small2d(const Plan& p, const double* in, double* out, int64_t
   cfg.numAttrs = 1;
   const int N0 = (int)p.N[0], N1 = (int)p.N[1], Ti = (int)T;
   switch (p.R) {
-    case 1: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<1>, in, out, N0, N1, rp, Ti, w);
-    case 2: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<2>, in, out, N0, N1, rp, Ti, w);
-    case 3: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<3>, in, out, N0, N1, rp, Ti, w);
-    case 4: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<4>, in, out, N0, N1, rp, Ti, w);
+    case 1: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<1>, in, out, N0, N1, rp, Ti, kb, w);
+    case 2: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<2>, in, out, N0, N1, rp, Ti, kb, w);
+    case 3: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<3>, in, out, N0, N1, rp, Ti, kb, w);
+    case 4: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<4>, in, out, N0, N1, rp, Ti, kb, w);
   }
   return cudaErrorInvalidValue;
 }

@@ -43,9 +43,10 @@ struct Plan {
   int tc_no_bvs = 0;
   int no_small = 0;       // LORA_NO_SMALL=1: no single-launch cluster path for small 2D grids (tests)      // LORA_TC_NO_BVS=1: the Fig. 9 ablation (shuffle-based stage 2) in the TC engine
   int n_planes_point = 0;
-  // CUDA-core engine, 2D, radius >= 3, W reflection-symmetric in both axes: evaluate W as the
-  // row-pair rank-1 split u_a = e_{R+a} + e_{R-a}, v_a = W[R+a,:] (a = 0..R; exact, growth 1),
-  // which issues R + (R+1)^2 + 2R FP64 ops per point against PMA's (28 vs 25 at R = 3).
+  // CUDA-core engine, 2D, radius >= 3, W reflection-symmetric in both axes with a nonzero centre
+  // column: evaluate W as the row-pair rank-1 split u_a = c_a (e_{R+a} + e_{R-a}), v_a = W[R+a,:] / c_a
+  // (c_a = W[R+a,R], a = 0..R; exact up to the rounding of v_a, growth 1), which issues
+  // R + R(R+1) + 2R + 1 FP64 ops per point against PMA's (22 vs 25 at R = 3).
   // LORA_RDG_PMA=1 keeps the PMA factors on that engine (ablation).
   int rdg_rows = 0;
   double recon_err = 0, growth = 0;

@@ -202,7 +202,9 @@ double cuda_fma_per_point(const Plan& p) {
   };
   if (p.ndim == 2) {
     const int R = p.R;
-    if (p.rdg_rows) return R + (R + 1) * (R + 1) + 2 * R;   // SIG_ROWS (kernels_rdg.cu; the fresh ring slot is assigned)
+    // SIG_ROWS (kernels_rdg.cu): R shared pair sums, R DFMA per row term (unit centre tap), 2R DFMA
+    // for the vertical gather and one DMUL for the fresh ring slot
+    if (p.rdg_rows) return R + (R + 1) * R + 2 * R + 1;
     // PMA pyramid (SIG_PMA): R shared tap-pair sums, then per chain of radius H a palindromic
     // horizontal gather (H: the chain is rescaled to a unit centre tap of v, kernels_rdg.cu
     // signature()) and a vertical scatter (2H+1), plus the scalar C_{h+1}
@@ -307,6 +309,7 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
 
   {  // row-pair split for the CUDA-core engine (Plan::rdg_rows)
     bool rows = ndim == 2 && radius >= 3;
+    for (int a = 0; rows && a <= radius; ++a) rows = weights[size_t(radius + a) * n + radius] != 0.0;   // unit centre taps
     for (int i = 0; rows && i < n; ++i)
       for (int j = 0; j < n; ++j)
         if (weights[size_t(i) * n + j] != weights[size_t(n - 1 - i) * n + j] ||
@@ -317,9 +320,7 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
     if (rows) {  // only where it issues less than the planner's own factors (not for star arms)
       const double f_terms = cuda_fma_per_point(p);
       p.rdg_rows = 1;
-      // a tie goes to the row pairs: their vertical gather is DADDs, which the FP64 pipe sustains at
-      // its full rate, the PMA scatter DFMAs with three register operands (~75 %,
-      // tools/ubench/fp64_operands.cu) — Box-2D49P: 25 vs 25
+      // Box-2D49P: 22 (row pairs, unit centre taps) vs 25 (PMA pyramid, unit centre taps)
       if (cuda_fma_per_point(p) > f_terms) p.rdg_rows = 0;
     }
   }

@@ -216,12 +216,14 @@ def test_default_engine_and_fusion_choices(L):
 
 def test_cuda_core_rank1_forms(L, monkeypatch):
     """CUDA-core engine: doubly reflection-symmetric W at radius >= 3 is evaluated as the row-pair
-    split (R + (R+1)^2 + 2R FP64 ops per point: 25 for Box-2D49P; it wins the tie with the PMA
-    pyramid, whose chains are rescaled to a unit centre tap: R + 1 + sum_H (H + 2H + 1) = 25), PMA
-    with LORA_RDG_PMA=1; an asymmetric W or radius <= 2 keeps the planner's factors."""
+    split with unit centre taps (R + R(R+1) + 2R + 1 FP64 ops per point: 22 for Box-2D49P, against
+    the PMA pyramid's R + 1 + sum_H (H + 2H + 1) = 25), PMA with LORA_RDG_PMA=1 or when a centre-
+    column weight is zero; an asymmetric W or radius <= 2 keeps the planner's factors."""
     W = synth.rsym_weights(2, 3, 4)
-    assert L.Stencil(W, (64, 64), engine="rdg_cuda").info()["fma_per_point_issued"] == 25
-    assert L.Stencil(synth.rsym_weights(2, 4, 4), (64, 64), engine="rdg_cuda").info()["fma_per_point_issued"] == 37
+    assert L.Stencil(W, (64, 64), engine="rdg_cuda").info()["fma_per_point_issued"] == 22
+    assert L.Stencil(synth.rsym_weights(2, 4, 4), (64, 64), engine="rdg_cuda").info()["fma_per_point_issued"] == 33
+    Wz = W.copy(); Wz[0, 3] = Wz[6, 3] = 0.0   # a zero centre-column weight: no unit centre tap for row pair 3
+    assert L.Stencil(Wz, (64, 64), engine="rdg_cuda").info()["fma_per_point_issued"] != 22
     assert L.Stencil(synth.rsym_weights(2, 1, 4), (64, 64), engine="rdg_cuda").info()["fma_per_point_issued"] == 6
     monkeypatch.setenv("LORA_RDG_PMA", "1")
     assert L.Stencil(W, (64, 64), engine="rdg_cuda").info()["fma_per_point_issued"] == 25
