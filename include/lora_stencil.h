@@ -197,10 +197,11 @@ int lora_stencil_dist_exchange_plan(const lora_plan* p, int rank, int nranks, in
  * single-GPU run of the global grid (same kernels, same per-point arithmetic).
  *
  * Engines: the CUDA-core engine (2D, 3D radius <= 2) and the direct comparison kernel; other
- * plans return LORA_ERR_UNSUPPORTED.  2D CUDA-core plans keep their fusion depth k (plan fuse_k):
- * each launch advances k steps and internal slab edges carry k*r-deep halos (every slab needs
- * >= k*r rows, else LORA_ERR_INVALID_ARG); 3D and direct plans step unfused.  Every rank's plan has
- * the same trailing extents, radius and fuse_k (the local n0 may differ).
+ * plans return LORA_ERR_UNSUPPORTED.  CUDA-core plans keep their fusion depth k (plan fuse_k; 2D,
+ * and 3D radius 1): each launch advances k steps and internal slab edges carry k*r-deep halos
+ * (every slab needs >= k*r rows/planes, else LORA_ERR_INVALID_ARG); direct plans and 3D radius-2
+ * plans step unfused.  Every rank's plan has the same trailing extents, radius and fuse_k (the
+ * local n0 may differ).
  *
  * Exchange buffers: the communicator owns two padded slabs (the ping-pong pair the neighbours
  * write into; rows = lower halo depth + n0 + upper halo depth) plus the flag words, allocated with

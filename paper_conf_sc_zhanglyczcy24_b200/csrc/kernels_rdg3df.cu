@@ -329,6 +329,9 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
         fence_proxy_async_global();
       }
     }
+    // warp 0 reconverges here: lane 0 may have spun above, and the CTA barriers that follow are
+    // .aligned (a diverged warp 0 would let lane 0 run on alone and deadlock at the next __syncwarp)
+    if (act) __syncwarp();
     if constexpr (TMA) {  // x even by construction; negative origins are zero-filled by TMA
       if (tid == 0) {
         fence_proxy_async();
@@ -354,6 +357,8 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
   // prologue (uniform across the CTA: issue_next may contain __syncthreads)
   for (int q = 0; q < F_NS - 1; ++q)
     if (q < nstages) issue_next(q);
+  __shared__ unsigned sig_count;   // warps done with the current boundary item (P2P signal)
+  if (tid == 0) sig_count = 0u;
   double acc[K][3][2][2];
   int citem = blockIdx.x, cj = 0, slot = 0, phase = 0;
   int X0 = 0, Y0 = 0, Z0 = 0, zend = 0;
@@ -463,12 +468,22 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
       }(std::make_integer_sequence<int, K - 1>{});
       if (++slot == F_NS) { slot = 0; phase ^= 1; }
       if (++cj == SI) {
-        if (t_lo || t_hi) {   // CTA-uniform: every thread's stores of the item are visible system-wide,
-          __threadfence_system();   // then one release per neighbour
-          __syncthreads();
-          const int u = citem % (nbx * nby);
-          if (tid == 0 && t_lo) p2p_st_release(dp.sig_lo + u, dp.sig_val);
-          if (tid == 0 && t_hi) p2p_st_release(dp.sig_hi + u, dp.sig_val);
+        if (t_lo || t_hi) {
+          // every warp makes its item stores visible system-wide and counts itself in; the last warp
+          // to arrive publishes the step counter to the neighbour(s) (no CTA-wide barrier here)
+          __threadfence_system();
+          __syncwarp();
+          if (lane == 0) {
+            const unsigned prev = atomicAdd(&sig_count, 1u);
+            if (prev == F_WARPS - 1) {
+              sig_count = 0u;
+              __threadfence_system();
+              const int u = citem % (nbx * nby);
+              if (t_lo) p2p_st_release(dp.sig_lo + u, dp.sig_val);
+              if (t_hi) p2p_st_release(dp.sig_hi + u, dp.sig_val);
+            }
+          }
+          __syncwarp();
         }
         cj = 0;
         citem += gridDim.x;

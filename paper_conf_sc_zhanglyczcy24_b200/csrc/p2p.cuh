@@ -41,13 +41,19 @@ __device__ __forceinline__ unsigned long long p2p_clock_ns() {
 // Spin (one thread) until flags[u] >= val for u in [u0, u1].  Gives up after kP2PTimeoutNs and
 // raises the device error word instead of hanging the GPU (the result is then invalid and
 // lora_stencil_p2p_status reports it).
-constexpr unsigned long long kP2PTimeoutNs = 20ull * 1000 * 1000 * 1000;
+#ifndef LORA_P2P_TIMEOUT_S
+#define LORA_P2P_TIMEOUT_S 20
+#endif
+constexpr unsigned long long kP2PTimeoutNs = LORA_P2P_TIMEOUT_S * 1000ull * 1000 * 1000;
 
 __device__ __forceinline__ void p2p_wait_units(const unsigned long long* flags, int u0, int u1,
                                                unsigned long long val, int* err) {
   unsigned long long t0 = 0;
   for (int u = u0; u <= u1; ++u) {
     while (p2p_ld_acquire(flags + u) < val) {
+      // once any wait of this endpoint has timed out the run is void: fail fast instead of paying
+      // the timeout again in every later wait
+      if (*reinterpret_cast<volatile int*>(err)) return;
       const unsigned long long now = p2p_clock_ns();
       if (t0 == 0) t0 = now;
       else if (now - t0 > kP2PTimeoutNs) { atomicExch(err, 1); return; }
