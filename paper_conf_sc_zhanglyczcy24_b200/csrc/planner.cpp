@@ -310,6 +310,11 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
   {  // row-pair split for the CUDA-core engine (Plan::rdg_rows)
     bool rows = ndim == 2 && radius >= 3;
     for (int a = 0; rows && a <= radius; ++a) rows = weights[size_t(radius + a) * n + radius] != 0.0;   // unit centre taps
+    // integer-valued W (the integer-exact mode, pin P9): the unit-centre rescale W[R+a,:] / c_a is
+    // not exact in general (c_a = 31 for the integer pyramid), so keep the planner's exact factors
+    bool integral = true;
+    for (size_t i = 0; integral && i < nw; ++i) integral = weights[i] == std::nearbyint(weights[i]);
+    if (integral) rows = false;
     for (int i = 0; rows && i < n; ++i)
       for (int j = 0; j < n; ++j)
         if (weights[size_t(i) * n + j] != weights[size_t(n - 1 - i) * n + j] ||
