@@ -42,7 +42,75 @@ struct StarArms {
 // Buffer row j of CTA c holds padded row c*rp + R - HK + j (HK = k R: the halo depth of a block of
 // k steps); own rows are j in [HK, HK + rp).  Rows outside the array are zero and never feed a
 // stored value; rows of the global Dirichlet halo are loaded into both buffers and never written.
-template <int R>
+// Radius 1, even padded width: one step of rows [j0, j1) with each thread walking a strip of rows of
+// one column pair (16-byte shared loads), the three rows of the vertical arm in registers and the
+// horizontal neighbours from the adjacent lanes (shuffles; warp-edge lanes load theirs).  Same
+// per-point arithmetic, in the same order, as the scalar loop below (and the streaming kernel).
+__device__ __forceinline__ void star1_step_vec(const double* __restrict__ src, double* __restrict__ dst, int P1, int N1,
+                                               int j0, int j1, const StarArms& w, double* lo_mb, double* hi_mb,
+                                               int HK, int rp, bool last, size_t lo_off, size_t hi_off) {
+  constexpr int NT = SM_TX * SM_TY;
+  const int tid = threadIdx.y * SM_TX + threadIdx.x;
+  const int NPR = P1 / 2;                       // column pairs (2q, 2q+1), q < NPR
+  const int QW = (NPR + 31) / 32 * 32;          // lanes per strip (whole warps)
+  const int S = NT / QW;                        // strips
+  const int q = tid % QW, sidx = tid / QW;
+  if (sidx >= S) return;                        // whole warps only: shuffles stay warp-uniform
+  const int lane = tid & 31;
+  const int nr = j1 - j0, per = (nr + S - 1) / S;
+  const int ra = j0 + sidx * per, rb = min(j1, ra + per);
+  const bool act = q < NPR;
+  const int x0 = 2 * q;
+  const bool in0 = x0 >= 1 && x0 <= N1, in1 = x0 + 1 <= N1;
+  double2 xm = make_double2(0.0, 0.0), xc = xm;
+  if (act && ra < rb) {
+    xm = *reinterpret_cast<const double2*>(src + size_t(ra - 1) * P1 + x0);
+    xc = *reinterpret_cast<const double2*>(src + size_t(ra) * P1 + x0);
+  }
+  for (int j = ra; j < rb; ++j) {
+    double2 xp = make_double2(0.0, 0.0);
+    if (act) xp = *reinterpret_cast<const double2*>(src + size_t(j + 1) * P1 + x0);
+    double left = __shfl_up_sync(0xffffffffu, xc.y, 1);
+    double right = __shfl_down_sync(0xffffffffu, xc.x, 1);
+    const double* row = src + size_t(j) * P1;
+    if (act && lane == 0 && x0 >= 1) left = row[x0 - 1];
+    if (act && (lane == 31 || q == NPR - 1) && x0 + 2 < P1) right = row[x0 + 2];
+    double th = fma(w.h[0], left, 0.0);
+    th = fma(w.h[1], xc.x, th);
+    th = fma(w.h[2], xc.y, th);
+    double a0 = fma(w.v[0], xm.x, 0.0);
+    a0 += th;
+    a0 = fma(w.v[1], xc.x, a0);
+    a0 = fma(w.v[2], xp.x, a0);
+    th = fma(w.h[0], xc.x, 0.0);
+    th = fma(w.h[1], xc.y, th);
+    th = fma(w.h[2], right, th);
+    double a1 = fma(w.v[0], xm.y, 0.0);
+    a1 += th;
+    a1 = fma(w.v[1], xc.y, a1);
+    a1 = fma(w.v[2], xp.y, a1);
+    if (act) {
+      double* o = dst + size_t(j) * P1 + x0;
+      if (in0 && in1) *reinterpret_cast<double2*>(o) = make_double2(a0, a1);
+      else if (in1) o[1] = a1;
+      else if (in0) o[0] = a0;
+      if (last && lo_mb && j >= HK && j < 2 * HK) {
+        double* m = lo_mb + lo_off + size_t(j - HK) * P1 + x0;
+        if (in0) m[0] = a0;
+        if (in1) m[1] = a1;
+      }
+      if (last && hi_mb && j >= rp && j < rp + HK) {
+        double* m = hi_mb + hi_off + size_t(j - rp) * P1 + x0;
+        if (in0) m[0] = a0;
+        if (in1) m[1] = a1;
+      }
+    }
+    xm = xc;
+    xc = xp;
+  }
+}
+
+template <int R, bool VEC>
 __global__ void __launch_bounds__(SM_TX * SM_TY, 1)
 small2d_star_kernel(const double* __restrict__ in, double* __restrict__ out, int N0, int N1, int rp, int T, int kb,
                     const __grid_constant__ StarArms w) {
@@ -78,6 +146,9 @@ small2d_star_kernel(const double* __restrict__ in, double* __restrict__ out, int
       const bool last = st == ks;
       // rows valid after this step: shrink by R per step from the block's HK-deep halo
       const int j0 = max(jlo, R * st + (HK - R * ks)), j1 = min(jhi, SR - R * st - (HK - R * ks));
+      if constexpr (VEC) {
+        star1_step_vec(src, dst, P1, N1, j0, j1, w, lo_mb, hi_mb, HK, rp, last, (2 * par + 1) * MB, (2 * par + 0) * MB);
+      } else
       for (int j = j0 + threadIdx.y; j < j1; j += SM_TY) {
         const bool to_lo = last && lo_mb && j >= HK && j < 2 * HK;               // my first HK own rows
         const bool to_hi = last && hi_mb && j >= rp && j < rp + HK;               // my last HK own rows
@@ -137,20 +208,26 @@ bool star_arms(const Plan& p, StarArms& w) {
 }
 
 template <int R>
-const void* kernel_of() { return (const void*)small2d_star_kernel<R>; }
+const void* kernel_of(bool vec) {
+  if constexpr (R == 1) { if (vec) return (const void*)small2d_star_kernel<1, true>; }
+  return (const void*)small2d_star_kernel<R, false>;
+}
 
-const void* kernel_for(int R) {
+const void* kernel_for(int R, bool vec) {
   switch (R) {
-    case 1: return kernel_of<1>();
-    case 2: return kernel_of<2>();
-    case 3: return kernel_of<3>();
-    case 4: return kernel_of<4>();
+    case 1: return kernel_of<1>(vec);
+    case 2: return kernel_of<2>(vec);
+    case 3: return kernel_of<3>(vec);
+    case 4: return kernel_of<4>(vec);
   }
   return nullptr;
 }
 
 constexpr size_t kMaxSmem = 227 * 1024;
-constexpr int kMaxBlock = 8;   // steps per exchange (redundant halo rows grow with it)
+#ifndef SMALL_MAX_BLOCK
+#define SMALL_MAX_BLOCK 8
+#endif
+constexpr int kMaxBlock = SMALL_MAX_BLOCK;   // steps per exchange (redundant halo rows grow with it)
 
 // Shared memory of one CTA: two slab buffers of rp + 2kR rows plus the double-buffered two-sided
 // mailbox of kR rows.
@@ -226,7 +303,8 @@ cudaError_t launch_small2d(const Plan& p, const double* in, double* out, int64_t
   if (!star_arms(p, w) || T < 1 || T > (int64_t(1) << 30)) return cudaErrorInvalidValue;
   int cs = cluster_size(p);
   if (cs == 0) return cudaErrorInvalidValue;
-  const void* k = kernel_for(p.R);
+  const bool vec = p.R == 1 && (p.P[1] % 2) == 0;   // 16-byte rows: the register-walking R = 1 step
+  const void* k = kernel_for(p.R, vec);
   // fall back to smaller clusters if the device cannot schedule this one
   while (cs >= 2 && (block_steps(p, cs) == 0 || setup(k, kMaxSmem, cs) == 0)) cs /= 2;
   if (cs < 2) return cudaErrorNotSupported;
@@ -246,10 +324,11 @@ cudaError_t launch_small2d(const Plan& p, const double* in, double* out, int64_t
   cfg.numAttrs = 1;
   const int N0 = (int)p.N[0], N1 = (int)p.N[1], Ti = (int)T;
   switch (p.R) {
-    case 1: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<1>, in, out, N0, N1, rp, Ti, kb, w);
-    case 2: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<2>, in, out, N0, N1, rp, Ti, kb, w);
-    case 3: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<3>, in, out, N0, N1, rp, Ti, kb, w);
-    case 4: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<4>, in, out, N0, N1, rp, Ti, kb, w);
+    case 1: return vec ? cudaLaunchKernelEx(&cfg, small2d_star_kernel<1, true>, in, out, N0, N1, rp, Ti, kb, w)
+                       : cudaLaunchKernelEx(&cfg, small2d_star_kernel<1, false>, in, out, N0, N1, rp, Ti, kb, w);
+    case 2: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<2, false>, in, out, N0, N1, rp, Ti, kb, w);
+    case 3: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<3, false>, in, out, N0, N1, rp, Ti, kb, w);
+    case 4: return cudaLaunchKernelEx(&cfg, small2d_star_kernel<4, false>, in, out, N0, N1, rp, Ti, kb, w);
   }
   return cudaErrorInvalidValue;
 }

@@ -172,7 +172,8 @@ def test_rows_and_pma_forms(h, shape, monkeypatch):
         for T in (1, 2, 5):
             a, info = run_gpu(W, g, T, engine="rdg_cuda", fuse_k=1)
             n = h + 1
-            want = (h + n * n + 2 * h) if pma == "0" else (h + 1 + sum((h - k) + (2 * (h - k) + 1) for k in range(h)))
+            # row pairs with unit centre taps: h pair sums + h DFMA per row term + 2h DFMA + 1 DMUL
+            want = (h + n * h + 2 * h + 1) if pma == "0" else (h + 1 + sum((h - k) + (2 * (h - k) + 1) for k in range(h)))
             assert info["fma_per_point_issued"] == want
             assert rel_err(a, oracle.run(W, g, T)) <= 1e-12
             b, _ = run_gpu(W, g, T, engine="rdg_cuda", fuse_k=2)
