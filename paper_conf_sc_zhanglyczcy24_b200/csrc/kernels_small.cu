@@ -59,22 +59,25 @@ __device__ __forceinline__ void star1_step_vec(const double* __restrict__ src, d
   const int lane = tid & 31;
   const int nr = j1 - j0, per = (nr + S - 1) / S;
   const int ra = j0 + sidx * per, rb = min(j1, ra + per);
+  if (ra >= rb) return;                         // uniform per warp (a strip is whole warps)
   const bool act = q < NPR;
-  const int x0 = 2 * q;
-  const bool in0 = x0 >= 1 && x0 <= N1, in1 = x0 + 1 <= N1;
-  double2 xm = make_double2(0.0, 0.0), xc = xm;
-  if (act && ra < rb) {
-    xm = *reinterpret_cast<const double2*>(src + size_t(ra - 1) * P1 + x0);
-    xc = *reinterpret_cast<const double2*>(src + size_t(ra) * P1 + x0);
-  }
-  for (int j = ra; j < rb; ++j) {
-    double2 xp = make_double2(0.0, 0.0);
-    if (act) xp = *reinterpret_cast<const double2*>(src + size_t(j + 1) * P1 + x0);
+  const int x0 = act ? 2 * q : 0;               // idle lanes read column pair 0 (any row): finite values
+  const bool in0 = act && x0 >= 1 && x0 <= N1, in1 = act && x0 + 1 <= N1;
+  const bool ld_left = act && lane == 0 && x0 >= 1, ld_right = act && (lane == 31 || q == NPR - 1) && x0 + 2 < P1;
+  const double* sp = src + ra * P1 + x0;        // row j, this pair
+  double* op = dst + ra * P1 + x0;
+  // mailbox rows: the block's last step stores my first / last HK own rows for the neighbours
+  const bool mlo = last && lo_mb != nullptr, mhi = last && hi_mb != nullptr;
+  double* lop = mlo ? lo_mb + lo_off + (ra - HK) * P1 + x0 : nullptr;
+  double* hip = mhi ? hi_mb + hi_off + (ra - rp) * P1 + x0 : nullptr;
+  double2 xm = *reinterpret_cast<const double2*>(sp - P1);
+  double2 xc = *reinterpret_cast<const double2*>(sp);
+  for (int j = ra; j < rb; ++j, sp += P1, op += P1, lop += P1, hip += P1) {
+    const double2 xp = *reinterpret_cast<const double2*>(sp + P1);
     double left = __shfl_up_sync(0xffffffffu, xc.y, 1);
     double right = __shfl_down_sync(0xffffffffu, xc.x, 1);
-    const double* row = src + size_t(j) * P1;
-    if (act && lane == 0 && x0 >= 1) left = row[x0 - 1];
-    if (act && (lane == 31 || q == NPR - 1) && x0 + 2 < P1) right = row[x0 + 2];
+    if (ld_left) left = sp[-1];
+    if (ld_right) right = sp[2];
     double th = fma(w.h[0], left, 0.0);
     th = fma(w.h[1], xc.x, th);
     th = fma(w.h[2], xc.y, th);
@@ -89,21 +92,16 @@ __device__ __forceinline__ void star1_step_vec(const double* __restrict__ src, d
     a1 += th;
     a1 = fma(w.v[1], xc.y, a1);
     a1 = fma(w.v[2], xp.y, a1);
-    if (act) {
-      double* o = dst + size_t(j) * P1 + x0;
-      if (in0 && in1) *reinterpret_cast<double2*>(o) = make_double2(a0, a1);
-      else if (in1) o[1] = a1;
-      else if (in0) o[0] = a0;
-      if (last && lo_mb && j >= HK && j < 2 * HK) {
-        double* m = lo_mb + lo_off + size_t(j - HK) * P1 + x0;
-        if (in0) m[0] = a0;
-        if (in1) m[1] = a1;
-      }
-      if (last && hi_mb && j >= rp && j < rp + HK) {
-        double* m = hi_mb + hi_off + size_t(j - rp) * P1 + x0;
-        if (in0) m[0] = a0;
-        if (in1) m[1] = a1;
-      }
+    if (in0 && in1) *reinterpret_cast<double2*>(op) = make_double2(a0, a1);
+    else if (in1) op[1] = a1;
+    else if (in0) op[0] = a0;
+    if (mlo && j < 2 * HK) {
+      if (in0) lop[0] = a0;
+      if (in1) lop[1] = a1;
+    }
+    if (mhi && j >= rp) {
+      if (in0) hip[0] = a0;
+      if (in1) hip[1] = a1;
     }
     xm = xc;
     xc = xp;
@@ -225,7 +223,7 @@ const void* kernel_for(int R, bool vec) {
 
 constexpr size_t kMaxSmem = 227 * 1024;
 #ifndef SMALL_MAX_BLOCK
-#define SMALL_MAX_BLOCK 8
+#define SMALL_MAX_BLOCK 4
 #endif
 constexpr int kMaxBlock = SMALL_MAX_BLOCK;   // steps per exchange (redundant halo rows grow with it)
 
