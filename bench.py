@@ -382,8 +382,9 @@ def main():
         dist.all_reduce(npts)          # uneven strong-scaling splits: the points all ranks processed
     pts_per_step = float(npts.item()) * T
     value = pts_per_step * args.steps / t / 1e9
-    # the NCCL path steps unfused; the P2P path runs the plan's fused depth (deep halos, 2D and 3D)
-    fuse = 1 if comm is not None else info["fuse_k"]
+    # the P2P path runs the plan's fused depth (deep halos, 2D and 3D); the NCCL path too for the
+    # CUDA-core engine at N > 1 (comm-owned deep-halo buffers), else it steps unfused
+    fuse = info["fuse_k"] if (comm is None or (world > 1 and info["engine_name"] == "rdg_cuda")) else 1
     launches_per_step = -(-T // fuse) + 2      # stencil launches + 2 halo-copy launches
     if ep is not None:   # ceil(T/k) stencil launches + 1 halo copy + per neighbour: 2 publish, 2 wait, 1 push
         nb = (1 if rank > 0 else 0) + (1 if rank < world - 1 else 0)

@@ -169,7 +169,11 @@ int lora_stencil_comm_get_id(void* id_out);
 /* Collective over `nranks` processes, one GPU each (current device). */
 int lora_stencil_comm_init(lora_comm** c, int nranks, int rank, const void* nccl_unique_id);
 /* Collective: every rank calls with the same timesteps.  `p` is planned with this rank's
- * LOCAL interior shape (n0_local, N1[, N2]) — uneven splits are allowed.  in_local/out_local
+ * LOCAL interior shape (n0_local, N1[, N2]) — uneven splits are allowed.  CUDA-core plans with
+ * fuse_k > 1 keep their fusion depth: the communicator then owns two deep-halo slab buffers
+ * (fuse_k * radius rows/planes at internal edges; every slab needs at least that many) and the
+ * exchange runs once per fused launch (after it, not overlapped); other plans step unfused with the
+ * edge strips computed first and the exchange overlapped with the interior strip.  in_local/out_local
  * are device padded arrays of that local shape.  Rank 0's low halo and rank n-1's high halo
  * are the physical Dirichlet boundary; the other slab-edge halos are overwritten each step
  * by the neighbours' edge rows/planes.  Ordered on `stream`. */
@@ -184,6 +188,13 @@ void lora_stencil_comm_destroy(lora_comm* c);
  * (elements, contiguous).  Returns the number of entries (0..4) or a negative lora_status. */
 int lora_stencil_dist_exchange_plan(const lora_plan* p, int rank, int nranks, int64_t* kind, int64_t* peer,
                                     int64_t* offset, int64_t* count);
+/* The same for a slab buffer whose internal edges carry halo_depth (>= radius) rows/planes: rows
+ * [0, hl) low halo, [hl, hl + n0) own, then hh high-halo rows, with hl = halo_depth below a neighbour
+ * and radius at the physical boundary (likewise hh).  lora_stencil_run_dist uses halo_depth =
+ * fuse_k * radius for CUDA-core plans with fuse_k > 1 (comm-owned deep-halo buffers, one exchange
+ * per fused launch); halo_depth = radius is lora_stencil_dist_exchange_plan. */
+int lora_stencil_dist_exchange_plan_ex(const lora_plan* p, int rank, int nranks, int64_t halo_depth, int64_t* kind,
+                                       int64_t* peer, int64_t* offset, int64_t* count);
 
 /* ---- multi-GPU: the same slab decomposition with a DEVICE-INITIATED halo exchange ----
  * (north star (d) "halo exchange over NVLink ... overlapped with interior

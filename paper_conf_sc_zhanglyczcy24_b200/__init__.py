@@ -80,6 +80,7 @@ _sig = {
     "lora_stencil_run_dist": (ctypes.c_int, [_P, _P, _P, _P, ctypes.c_int64, _P]),
     "lora_stencil_comm_destroy": (None, [_P]),
     "lora_stencil_dist_exchange_plan": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_int, _P, _P, _P, _P]),
+    "lora_stencil_dist_exchange_plan_ex": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_int, ctypes.c_int64, _P, _P, _P, _P]),
     "lora_stencil_p2p_create": (ctypes.c_int, [_P, _P, ctypes.c_int, ctypes.c_int]),
     "lora_stencil_p2p_handle_size": (ctypes.c_size_t, []),
     "lora_stencil_p2p_get_handle": (ctypes.c_int, [_P, _P]),
@@ -277,10 +278,15 @@ def lora_stencil_p2p_destroy(c) -> None:
     _lib.lora_stencil_p2p_destroy(c)
 
 
-def lora_stencil_dist_exchange_plan(plan, rank: int, nranks: int):
-    """[(kind 'send'|'recv', peer, element offset, element count)] in NCCL-group issue order."""
+def lora_stencil_dist_exchange_plan(plan, rank: int, nranks: int, halo_depth: int | None = None):
+    """[(kind 'send'|'recv', peer, element offset, element count)] in NCCL-group issue order; with
+    halo_depth, the plan for a deep-halo slab buffer (lora_stencil_dist_exchange_plan_ex)."""
     a = [np.zeros(4, np.int64) for _ in range(4)]
-    m = _lib.lora_stencil_dist_exchange_plan(plan, int(rank), int(nranks), *[x.ctypes.data for x in a])
+    if halo_depth is None:
+        m = _lib.lora_stencil_dist_exchange_plan(plan, int(rank), int(nranks), *[x.ctypes.data for x in a])
+    else:
+        m = _lib.lora_stencil_dist_exchange_plan_ex(plan, int(rank), int(nranks), int(halo_depth),
+                                                    *[x.ctypes.data for x in a])
     if m < 0:
         raise LoraError(m, lora_stencil_last_error())
     return [("send" if a[0][i] == 0 else "recv", int(a[1][i]), int(a[2][i]), int(a[3][i])) for i in range(m)]

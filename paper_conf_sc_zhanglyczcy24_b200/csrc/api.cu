@@ -52,6 +52,9 @@ cudaError_t step(const Plan& p, const double* src, double* dst, cudaStream_t s, 
 int step_launch(const Plan& p, const double* src, double* dst, void* stream) {
   return (int)step(p, src, dst, static_cast<cudaStream_t>(stream));
 }
+int step_launch_k(const Plan& p, const double* src, double* dst, void* stream, int k) {
+  return (int)step(p, src, dst, static_cast<cudaStream_t>(stream), k);
+}
 int copy_halo_launch(const Plan& p, const double* in, double* dst, void* stream) {
   return (int)launch_copy_halo(p, in, dst, static_cast<cudaStream_t>(stream));
 }

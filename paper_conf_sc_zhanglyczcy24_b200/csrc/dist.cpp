@@ -81,30 +81,38 @@ struct lora_comm {
   int rank = 0, nranks = 1, device = -1;
   cudaStream_t comm_stream = nullptr;   // halo exchange runs here, overlapped with interior compute
   cudaEvent_t ev_edge = nullptr, ev_comm = nullptr;
+  double* dbuf[2] = {nullptr, nullptr}; // fused runs: deep-halo slab buffers (hl + n0 + hh rows)
+  size_t dbuf_elems = 0;
 };
 
 namespace {
-int exchange_plan(const lora_plan* p, int rank, int nranks, int64_t* kind, int64_t* peer, int64_t* off, int64_t* cnt) {
-  const int R = p->R;
+// The halo exchange of a slab buffer whose internal edges carry H-deep halos (H = R: the caller's
+// layout; H = k R: the fused path's deep-halo buffers).  Buffer rows: [0, hl) low halo, [hl, hl + n0)
+// own rows, [hl + n0, hl + n0 + hh) high halo, with hl = H below a neighbour (R at the physical
+// boundary), likewise hh.  My first H own rows go to rank - 1's high halo, my last H to rank + 1's
+// low halo; the neighbours' rows fill mine.  All transfers are whole contiguous rows / planes.
+int exchange_plan(const lora_plan* p, int rank, int nranks, int64_t H, int64_t* kind, int64_t* peer, int64_t* off,
+                  int64_t* cnt) {
   const int64_t row = p->ndim == 2 ? p->P[1] : p->P[1] * p->P[2];   // elements per padded row/plane
   const int64_t n0 = p->N[0];
+  const int64_t hl = rank > 0 ? H : p->R;
   int k = 0;
-  if (rank > 0) {  // my first R interior rows go down; the neighbour's last R fill my low halo
-    kind[k] = 0; peer[k] = rank - 1; off[k] = R * row; cnt[k] = R * row; ++k;
-    kind[k] = 1; peer[k] = rank - 1; off[k] = 0; cnt[k] = R * row; ++k;
+  if (rank > 0) {  // my first H own rows go down; the neighbour's last H fill my low halo
+    kind[k] = 0; peer[k] = rank - 1; off[k] = hl * row; cnt[k] = H * row; ++k;
+    kind[k] = 1; peer[k] = rank - 1; off[k] = 0; cnt[k] = H * row; ++k;
   }
-  if (rank < nranks - 1) {  // my last R interior rows go up; the neighbour's first R fill my high halo
-    kind[k] = 0; peer[k] = rank + 1; off[k] = n0 * row; cnt[k] = R * row; ++k;
-    kind[k] = 1; peer[k] = rank + 1; off[k] = (n0 + R) * row; cnt[k] = R * row; ++k;
+  if (rank < nranks - 1) {  // my last H own rows go up; the neighbour's first H fill my high halo
+    kind[k] = 0; peer[k] = rank + 1; off[k] = (hl + n0 - H) * row; cnt[k] = H * row; ++k;
+    kind[k] = 1; peer[k] = rank + 1; off[k] = (hl + n0) * row; cnt[k] = H * row; ++k;
   }
   return k;
 }
 
-// Fills buf's slab-edge halos from the neighbours (one NCCL group, stream-ordered).
-int exchange(const lora_plan* p, lora_comm* c, double* buf, cudaStream_t s) {
+// Fills buf's slab-edge halos (depth H) from the neighbours (one NCCL group, stream-ordered).
+int exchange(const lora_plan* p, lora_comm* c, double* buf, cudaStream_t s, int64_t H = 0) {
   if (c->nranks == 1) return LORA_OK;
   int64_t kind[4], peer[4], off[4], cnt[4];
-  const int m = exchange_plan(p, c->rank, c->nranks, kind, peer, off, cnt);
+  const int m = exchange_plan(p, c->rank, c->nranks, H > 0 ? H : p->R, kind, peer, off, cnt);
   Nccl& n = nccl();
   ncclResult_t r = n.GroupStart();
   if (r) return nccl_fail(r, "ncclGroupStart");
@@ -127,7 +135,16 @@ int lora_stencil_dist_exchange_plan(const lora_plan* p, int rank, int nranks, in
   if (!p || !kind || !peer || !offset || !count || nranks < 1 || rank < 0 || rank >= nranks)
     return lora::fail(LORA_ERR_INVALID_ARG, "bad exchange-plan arguments");
   if (nranks > 1 && p->N[0] < p->R) return lora::fail(LORA_ERR_INVALID_ARG, "each slab needs >= radius rows/planes");
-  return exchange_plan(p, rank, nranks, kind, peer, offset, count);
+  return exchange_plan(p, rank, nranks, p->R, kind, peer, offset, count);
+}
+
+int lora_stencil_dist_exchange_plan_ex(const lora_plan* p, int rank, int nranks, int64_t halo_depth, int64_t* kind,
+                                       int64_t* peer, int64_t* offset, int64_t* count) {
+  if (!p || !kind || !peer || !offset || !count || nranks < 1 || rank < 0 || rank >= nranks || halo_depth < p->R)
+    return lora::fail(LORA_ERR_INVALID_ARG, "bad exchange-plan arguments (halo_depth must be >= radius)");
+  if (nranks > 1 && p->N[0] < halo_depth)
+    return lora::fail(LORA_ERR_INVALID_ARG, "each slab needs >= halo_depth rows/planes");
+  return exchange_plan(p, rank, nranks, halo_depth, kind, peer, offset, count);
 }
 
 int lora_stencil_comm_get_id(void* id_out) {
@@ -168,6 +185,63 @@ int lora_stencil_comm_init(lora_comm** c, int nranks, int rank, const void* nccl
   return LORA_OK;
 }
 
+}  // extern "C"
+
+namespace {
+// Fused run (the plan's fusion depth k > 1, CUDA-core engine): the slab lives in two comm-owned
+// buffers with H = k R deep halos at internal edges, presented to the plan's own fused kernels as a
+// taller padded array (the "view": its deep-halo rows count as interior and are recomputed
+// redundantly; after j fused sub-steps only rows within jR of the view's R-deep edge are wrong, and
+// jR <= H never reaches an own row).  Per launch: k steps on the view, then one NCCL group refills
+// the H-deep halos of the result with the neighbours' rows (what the kernel wrote there is
+// discarded).  Every own point is computed exactly as in a single-GPU run (pin P10).
+int run_fused(lora_plan* p, lora_comm* c, const double* in_local, double* out_local, int64_t T, cudaStream_t s) {
+  using namespace lora;
+  const int R = p->R, k = p->fuse_k;
+  const int64_t H = int64_t(k) * R, n0 = p->N[0];
+  if (c->nranks > 1 && n0 < H)
+    return fail(LORA_ERR_INVALID_ARG, "each slab needs >= fuse_k * radius rows/planes (plan with a smaller fuse_k)");
+  const int64_t hl = c->rank > 0 ? H : R, hh = c->rank < c->nranks - 1 ? H : R;
+  const int64_t row = p->ndim == 1 ? 1 : (p->ndim == 2 ? p->P[1] : p->P[1] * p->P[2]);
+  const size_t elems = size_t(hl + n0 + hh) * size_t(row);
+  if (c->dbuf_elems < elems) {
+    for (double*& b : c->dbuf) { if (b) cudaFree(b); b = nullptr; }
+    c->dbuf_elems = 0;
+    for (double*& b : c->dbuf)
+      if (cudaMalloc(&b, elems * sizeof(double)) != cudaSuccess) { cudaGetLastError(); return fail(LORA_ERR_OOM, "cudaMalloc(deep-halo slab buffers)"); }
+    c->dbuf_elems = elems;
+  }
+  lora::Plan v = *p;   // the view: hl + n0 + hh rows with an R-deep halo
+  v.N[0] = n0 + (hl - R) + (hh - R);
+  v.P[0] = v.N[0] + 2 * R;
+  v.elems = elems;
+  v.graph_exec = nullptr;
+  v.scratch = nullptr;
+  v.dev_in = v.dev_out = nullptr;
+  const int64_t shift = (hl - R) * row;   // caller row 0 -> buffer row hl - R
+  const size_t bytes = p->elems * sizeof(double);
+  cudaError_t ce = cudaMemcpyAsync(c->dbuf[0] + shift, in_local, bytes, cudaMemcpyDeviceToDevice, s);
+  if (ce != cudaSuccess) return cuda_fail(ce, "copy-in");
+  int e = copy_halo_launch(*p, in_local, c->dbuf[1] + shift, s);   // the Dirichlet ring of the own rows
+  if (e) return cuda_fail(e, "copy_halo launch");
+  int rc = exchange(p, c, c->dbuf[0], s, H);                        // step-0 deep halos
+  if (rc) return rc;
+  int cur = 0;
+  for (int64_t done = 0; done < T;) {
+    const int kk = (int)std::min<int64_t>(k, T - done);
+    if ((e = step_launch_k(v, c->dbuf[cur], c->dbuf[cur ^ 1], s, kk))) return cuda_fail(e, "fused stencil launch");
+    cur ^= 1;
+    if ((rc = exchange(p, c, c->dbuf[cur], s, H))) return rc;
+    done += kk;
+  }
+  ce = cudaMemcpyAsync(out_local, c->dbuf[cur] + shift, bytes, cudaMemcpyDeviceToDevice, s);
+  if (ce != cudaSuccess) return cuda_fail(ce, "copy-out");
+  return LORA_OK;
+}
+}  // namespace
+
+extern "C" {
+
 int lora_stencil_run_dist(lora_plan* p, lora_comm* c, const double* in_local, double* out_local, int64_t timesteps,
                           void* stream) {
   using namespace lora;
@@ -185,6 +259,15 @@ int lora_stencil_run_dist(lora_plan* p, lora_comm* c, const double* in_local, do
   }
   int rc = ensure_device(*p, timesteps >= 2);
   if (rc) return rc;
+  const char* ff = std::getenv("LORA_DIST_FUSED");   // tests: the fused path on one rank
+  if (p->engine == LORA_ENGINE_RDG_CUDA && p->fuse_k > 1 && (c->nranks > 1 || (ff && ff[0] == '1'))) {
+    rc = run_fused(p, c, in_local, out_local, timesteps, s);
+    if (rc == LORA_OK && sync_check()) {
+      cudaError_t ce = cudaStreamSynchronize(s);
+      if (ce != cudaSuccess) return cuda_fail(ce, "LORA_SYNC_CHECK stream sync");
+    }
+    return rc;
+  }
   int e = copy_halo_launch(*p, in_local, out_local, s);
   if (e) return cuda_fail(e, "copy_halo launch");
   if (timesteps >= 2) {
@@ -238,6 +321,8 @@ int lora_stencil_run_dist(lora_plan* p, lora_comm* c, const double* in_local, do
 
 void lora_stencil_comm_destroy(lora_comm* c) {
   if (!c) return;
+  for (double* b : c->dbuf)
+    if (b) cudaFree(b);
   if (c->comm && nccl().ok) nccl().CommDestroy(c->comm);
   if (c->ev_edge) cudaEventDestroy(c->ev_edge);
   if (c->ev_comm) cudaEventDestroy(c->ev_comm);

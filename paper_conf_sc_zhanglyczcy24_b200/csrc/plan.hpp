@@ -76,6 +76,7 @@ int fail(int code, const std::string& msg);
 int cuda_fail(int /*cudaError_t*/ e, const char* what);
 int ensure_device(Plan& p, bool want_scratch);
 int step_launch(const Plan& p, const double* src, double* dst, void* stream);       // cudaError_t
+int step_launch_k(const Plan& p, const double* src, double* dst, void* stream, int k);   // k fused steps
 int copy_halo_launch(const Plan& p, const double* in, double* dst, void* stream);   // cudaError_t
 bool sync_check();
 

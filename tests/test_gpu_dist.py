@@ -54,6 +54,30 @@ def test_run_dist_split_strips_bitwise(d, h, shape, engine, monkeypatch):
     L.lora_stencil_comm_destroy(comm)
 
 
+@pytest.mark.parametrize("d,h,shape", [(2, 3, (200, 130)), (2, 1, (150, 97)), (3, 1, (40, 20, 66))])
+def test_run_dist_fused_path_one_rank(d, h, shape, monkeypatch):
+    """The fused NCCL path (comm-owned deep-halo buffers, one exchange per fused launch; csrc/dist.cpp
+    run_fused) on one rank (LORA_DIST_FUSED=1): equal to lora_stencil_run bitwise for T covering
+    remainder launches, and repeated runs reuse the buffers."""
+    import torch
+    import paper_conf_sc_zhanglyczcy24_b200 as L
+    monkeypatch.setenv("LORA_DIST_FUSED", "1")
+    W = synth.rsym_weights(d, h, 23)
+    g = synth.grid(tuple(n + 2 * h for n in shape), 24)
+    st = L.Stencil(W, shape)
+    k = st.info()["fuse_k"]
+    assert k > 1
+    x = torch.from_numpy(g).cuda()
+    comm = L.lora_stencil_comm_init(1, 0, b"\0" * L.lora_stencil_comm_id_size())
+    for T in sorted({1, k, k + 1, 2 * k + 1}):
+        a = torch.empty_like(x); b = torch.full_like(x, float("nan"))
+        st.run(x, a, T)
+        L.lora_stencil_run_dist(st.plan, comm, x.data_ptr(), b.data_ptr(), T, torch.cuda.current_stream().cuda_stream)
+        torch.cuda.synchronize()
+        assert torch.equal(a, b), T
+    L.lora_stencil_comm_destroy(comm)
+
+
 def _rank(rank, world, case, q, idq):
     try:
         import sys
