@@ -32,6 +32,11 @@ namespace {
 #ifndef RDG3F_NS
 #define RDG3F_NS 0   // TMA ring stages; 0: per signature (f_ns)
 #endif
+#ifndef RDG3F_LAG
+#define RDG3F_LAG 0   // 1: stage S consumes the plane stage S-1 published in the PREVIOUS iteration (one
+#endif                // CTA barrier at the end of the iteration, the stages of an iteration independent).
+                      // Measured slower (r02m, same box): Box-3D27P k = 2 393 -> 379 GS/s, Heat-3D 449 -> 416
+constexpr int F_LAG = RDG3F_LAG;
 constexpr int F_WARPS = 8;
 constexpr int F_S1 = 16;             // stage-1 rows per CTA column (2 per warp); stage s: 16 - 2(s-1)
 constexpr int F_IN = 18;             // staged input rows
@@ -420,29 +425,35 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
           publish_ip<K, 1, (I + 1) % 3, !SG::assign0>(acc, sbuf + (0 * 2 + par) * S1B, w, lane, Y0, X0, p - 1, P0, P1, P2, in,
                                                       fast1);
       }
-      __syncthreads();  // stage-1 plane visible; every warp is done with the input slot
-      if (q + F_NS - 1 < nstages) issue_next((slot + F_NS - 1) % F_NS);
-      // ---------------- stages 2 .. K
+      if constexpr (!F_LAG) {
+        __syncthreads();  // stage-1 plane visible; every warp is done with the input slot
+        if (q + F_NS - 1 < nstages) issue_next((slot + F_NS - 1) % F_NS);
+      }
+      // ---------------- stages 2 .. K (F_LAG: stage S runs L = S - 1 iterations behind stage 1 and
+      // reads the plane stage S-1 published in the previous iteration, from the other parity buffer)
       auto stage = [&](auto Sc) {
         constexpr int S = decltype(Sc)::value;
-        constexpr int IS = pm3(I - (S - 1));       // ring position of the stage-(S-1) plane consumed
-        const bool active = w < F_S1 / 2 - (S - 1) && cj >= 2 * (S - 1);
+        constexpr int LG = F_LAG ? S - 1 : 0;                  // iterations stage S lags stage 1
+        constexpr int IS = pm3(I - (S - 1) - LG);              // ring position of the stage-(S-1) plane consumed
+        const bool active = w < F_S1 / 2 - (S - 1) && cj >= 2 * (S - 1) + LG;
+        const int rpar = F_LAG ? (par ^ 1) : par;              // parity of the buffer stage S reads
         if (active) {
-          const double* Sb = sbuf + ((S - 2) * 2 + par) * S1B;
+          const double* Sb = sbuf + ((S - 2) * 2 + rpar) * S1B;
           double x[4][4];
           load_rows(Sb + (2 * w) * F_S1W, F_S1W, lane, x);
           planes2<SG, IS, 0>(x, prm, acc[S - 1]);
         }
         if constexpr (S < K) {
           // (S < K only for K = 3: in-place Dirichlet loads)
-          if (active) publish_ip<K, S, (IS + 1) % 3, !SG::assign0>(acc, sbuf + ((S - 1) * 2 + par) * S1B, w, lane, Y0, X0, p - S,
-                                                                  P0, P1, P2, in, xy_in[S - 1] && p - S >= 1 && p - S < P0 - 1);
-          __syncthreads();
+          if (active) publish_ip<K, S, (IS + 1) % 3, !SG::assign0>(acc, sbuf + ((S - 1) * 2 + par) * S1B, w, lane, Y0, X0,
+                                                                  p - S - LG, P0, P1, P2, in,
+                                                                  xy_in[S - 1] && p - S - LG >= 1 && p - S - LG < P0 - 1);
+          if constexpr (!F_LAG) __syncthreads();
         } else if (active) {
-          // final plane zf = p - K complete: ring slot (IS + 1) % 3
+          // final plane zf = p - K - LG complete: ring slot (IS + 1) % 3
           constexpr int s = (IS + 1) % 3;
-          const int zf = p - K;
-          if (cj >= 2 * K && zf >= Z0 && zf < zend && (!act || zf >= dp.store_lo)) {
+          const int zf = p - K - LG;
+          if (cj >= 2 * K + LG && zf >= Z0 && zf < zend && (!act || zf >= dp.store_lo)) {
             // the plane goes to this slab and, for the first / last H own planes of a slab with a
             // neighbour there, into that neighbour's halo as well (peer memory)
             const int64_t e0 = (int64_t(zf) * P1 + Y0 + 2 * w) * P2 + X0 + c0;
@@ -466,6 +477,10 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
       [&]<int... Ss>(std::integer_sequence<int, Ss...>) {
         (stage(std::integral_constant<int, Ss + 2>{}), ...);
       }(std::make_integer_sequence<int, K - 1>{});
+      if constexpr (F_LAG) {
+        __syncthreads();  // this iteration's planes visible, last iteration's buffers and the input slot free
+        if (q + F_NS - 1 < nstages) issue_next((slot + F_NS - 1) % F_NS);
+      }
       if (++slot == F_NS) { slot = 0; phase ^= 1; }
       if (++cj == SI) {
         if (t_lo || t_hi) {
@@ -572,7 +587,7 @@ cudaError_t launch_f(const Plan& p, const double* src, double* dst, cudaStream_t
     }
   }
   const int ZC = (int)zc;
-  const int SI = ((ZC + 2 * K) + 2) / 3 * 3;
+  const int SI = ((ZC + 2 * K + F_LAG * (K - 1)) + 2) / 3 * 3;   // + the lag of the last stage
   const int nbz = (int)((p.N[0] + ZC - 1) / ZC);
   const int64_t nitems = int64_t(nbx) * nby * nbz;
   const int grid = (int)std::min<int64_t>(max_grid, nitems);
