@@ -206,12 +206,12 @@ def host_info():
 WEAK_SLAB = {"box2d49p-40960": (5120, 40960), "box3d27p-1024": (128, 1024, 1024)}
 
 
-def local_shape(name, cfg, world, rank, scaling):
+def local_shape(name, cfg, world, rank, scaling, force_dist=False):
     """This rank's interior slab and the global interior shape.  Multi-GPU configs: weak = the fixed
     §8(e) slab per rank (global grows with N), strong = the global shape split along the slowest axis
     (uneven splits allowed).  Other configs: every rank owns the config's shape (weak)."""
     g = tuple(cfg["shape"])
-    if name in WEAK_SLAB and (world > 1 or scaling == "strong"):
+    if name in WEAK_SLAB and (world > 1 or scaling == "strong" or force_dist):
         if scaling == "weak":
             loc = WEAK_SLAB[name]
             return loc, (loc[0] * world,) + tuple(loc[1:])
@@ -281,7 +281,7 @@ def main():
     W, cfg = synth.config(args.workload)
     cfg["name"] = args.workload
     h, T = cfg["radius"], cfg["T"]
-    shape, gshape = local_shape(args.workload, cfg, world, rank, args.scaling)   # this rank's slab, global grid
+    shape, gshape = local_shape(args.workload, cfg, world, rank, args.scaling, args.force_dist)   # this rank's slab, global grid
     padded = tuple(n + 2 * h for n in shape)
     st = L.Stencil(W, shape, engine=args.engine, fuse_k=args.fuse)
     info = st.info()
