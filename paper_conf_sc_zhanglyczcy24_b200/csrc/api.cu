@@ -201,6 +201,7 @@ void lora_stencil_plan_destroy(lora_plan* p) {
     if (p->scratch) cudaFree(p->scratch);
     if (p->dev_in) cudaFree(p->dev_in);
     if (p->dev_out) cudaFree(p->dev_out);
+    if (p->xbuf) cudaFree(p->xbuf);
     if (cur >= 0 && cur != p->device) cudaSetDevice(cur);
   }
   delete p;

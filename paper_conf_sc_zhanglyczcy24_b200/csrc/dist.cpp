@@ -218,6 +218,8 @@ int run_fused(lora_plan* p, lora_comm* c, const double* in_local, double* out_lo
   v.graph_exec = nullptr;
   v.scratch = nullptr;
   v.dev_in = v.dev_out = nullptr;
+  v.xbuf = nullptr;
+  v.xbuf_elems = 0;
   const int64_t shift = (hl - R) * row;   // caller row 0 -> buffer row hl - R
   const size_t bytes = p->elems * sizeof(double);
   cudaError_t ce = cudaMemcpyAsync(c->dbuf[0] + shift, in_local, bytes, cudaMemcpyDeviceToDevice, s);

@@ -131,6 +131,8 @@ lora::Plan view_of(const lora::Plan& p, const lora_p2p* c) {
   v.graph_exec = nullptr;
   v.scratch = nullptr;
   v.dev_in = v.dev_out = nullptr;
+  v.xbuf = nullptr;
+  v.xbuf_elems = 0;
   return v;
 }
 

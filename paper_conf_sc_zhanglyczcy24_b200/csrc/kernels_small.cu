@@ -48,9 +48,8 @@ struct StarArms {
 // per-point arithmetic, in the same order, as the scalar loop below (and the streaming kernel).
 __device__ __forceinline__ void star1_step_vec(const double* __restrict__ src, double* __restrict__ dst, int P1, int N1,
                                                int j0, int j1, const StarArms& w, double* lo_mb, double* hi_mb,
-                                               int HK, int rp, bool last, size_t lo_off, size_t hi_off) {
-  constexpr int NT = SM_TX * SM_TY;
-  const int tid = threadIdx.y * SM_TX + threadIdx.x;
+                                               int HK, int rp, bool last, size_t lo_off, size_t hi_off,
+                                               int tid, int NT) {
   const int NPR = P1 / 2;                       // column pairs (2q, 2q+1), q < NPR
   const int QW = (NPR + 31) / 32 * 32;          // lanes per strip (whole warps)
   const int S = NT / QW;                        // strips
@@ -72,6 +71,7 @@ __device__ __forceinline__ void star1_step_vec(const double* __restrict__ src, d
   double* hip = mhi ? hi_mb + hi_off + (ra - rp) * P1 + x0 : nullptr;
   double2 xm = *reinterpret_cast<const double2*>(sp - P1);
   double2 xc = *reinterpret_cast<const double2*>(sp);
+#pragma unroll 3
   for (int j = ra; j < rb; ++j, sp += P1, op += P1, lop += P1, hip += P1) {
     const double2 xp = *reinterpret_cast<const double2*>(sp + P1);
     double left = __shfl_up_sync(0xffffffffu, xc.y, 1);
@@ -92,9 +92,12 @@ __device__ __forceinline__ void star1_step_vec(const double* __restrict__ src, d
     a1 += th;
     a1 = fma(w.v[1], xc.y, a1);
     a1 = fma(w.v[2], xp.y, a1);
-    if (in0 && in1) *reinterpret_cast<double2*>(op) = make_double2(a0, a1);
-    else if (in1) op[1] = a1;
-    else if (in0) op[0] = a0;
+    if (in0 && in1) {
+      *reinterpret_cast<double2*>(op) = make_double2(a0, a1);
+    } else {
+      if (in1) op[1] = a1;
+      if (in0) op[0] = a0;
+    }
     if (mlo && j < 2 * HK) {
       if (in0) lop[0] = a0;
       if (in1) lop[1] = a1;
@@ -145,7 +148,8 @@ small2d_star_kernel(const double* __restrict__ in, double* __restrict__ out, int
       // rows valid after this step: shrink by R per step from the block's HK-deep halo
       const int j0 = max(jlo, R * st + (HK - R * ks)), j1 = min(jhi, SR - R * st - (HK - R * ks));
       if constexpr (VEC) {
-        star1_step_vec(src, dst, P1, N1, j0, j1, w, lo_mb, hi_mb, HK, rp, last, (2 * par + 1) * MB, (2 * par + 0) * MB);
+        star1_step_vec(src, dst, P1, N1, j0, j1, w, lo_mb, hi_mb, HK, rp, last, (2 * par + 1) * MB, (2 * par + 0) * MB,
+                       tid, SM_TX * SM_TY);
       } else
       for (int j = j0 + threadIdx.y; j < j1; j += SM_TY) {
         const bool to_lo = last && lo_mb && j >= HK && j < 2 * HK;               // my first HK own rows
@@ -187,6 +191,130 @@ small2d_star_kernel(const double* __restrict__ in, double* __restrict__ out, int
   const double* res = cur ? buf1 : buf0;
   const int w0 = c == 0 ? HK - R : HK, w1 = c == CS - 1 ? HK + rp + R : HK + rp;
   for (int i = w0 * P1 + tid; i < w1 * P1; i += NT) out[int64_t(pr0) * P1 + i] = res[i];
+}
+
+// Grid variant (the default when it applies): a cooperative grid of G = N0 / rp CTAs (co-resident,
+// all SMs instead of one cluster's 16) with the same slab / block / shrinking-row scheme; after each
+// block of k steps every CTA copies its first / last kR own rows into a global exchange buffer
+// (two parities x G CTAs x 2 sides), one grid-wide barrier (cooperative groups) publishes them, and
+// each CTA unpacks its neighbours' rows into its halo.  Same per-point arithmetic (bitwise equal).
+constexpr int GT_MAX = 512;
+#ifdef SMALL_TRACE
+__device__ unsigned long long g_small_trace[64];
+__device__ __forceinline__ void strace(int k) {
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    g_small_trace[k] = t;
+  }
+}
+#else
+__device__ __forceinline__ void strace(int) {}
+#endif
+
+template <int R, bool VEC>
+__global__ void __launch_bounds__(GT_MAX)
+small2d_grid_kernel(const double* __restrict__ in, double* __restrict__ out, double* __restrict__ xch,
+                    unsigned long long* __restrict__ flags, unsigned long long base, int N0, int N1, int rp, int T,
+                    int kb, const __grid_constant__ StarArms w) {
+  const int c = blockIdx.x, G = gridDim.x;
+  extern __shared__ __align__(16) double sm[];
+  const int P1 = N1 + 2 * R, P0 = N0 + 2 * R, HK = kb * R, SR = rp + 2 * HK;
+  double* const buf0 = sm;
+  double* const buf1 = sm + size_t(SR) * P1;
+  const int tid = threadIdx.x, NT = blockDim.x;
+  const int pr0 = c * rp + R - HK;          // padded row of buffer row 0
+  strace(0);
+  {  // stage the slab: rows inside the array only (the others stay zero); all loads of a thread first
+    const int r0 = max(0, -pr0), r1 = min(SR, P0 - pr0);
+    for (int i = tid; i < SR * P1; i += NT) { buf0[i] = 0.0; buf1[i] = 0.0; }
+    __syncthreads();
+    const double* src = in + int64_t(pr0 + r0) * P1;
+    const int n = (r1 - r0) * P1;
+    double* d0 = buf0 + r0 * P1;
+    double* d1 = buf1 + r0 * P1;
+    constexpr int U = 8;
+    for (int b = tid; b < n; b += NT * U) {
+      double v[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) v[u] = b + u * NT < n ? __ldg(src + b + u * NT) : 0.0;
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+        if (b + u * NT < n) { d0[b + u * NT] = v[u]; d1[b + u * NT] = v[u]; }
+    }
+  }
+  const size_t XB = size_t(HK) * P1;       // one side of one CTA in the exchange buffer
+  const int jlo = max(R, R - pr0), jhi = min(SR - R, P0 - R - pr0);
+  __syncthreads();
+  strace(1);
+  int cur = 0;
+  for (int t0 = 0, blk = 0; t0 < T; t0 += kb, ++blk) {
+    const int ks = min(kb, T - t0);
+    for (int st = 1; st <= ks; ++st) {
+      const double* src = cur ? buf1 : buf0;
+      double* dst = cur ? buf0 : buf1;
+      const int j0 = max(jlo, R * st + (HK - R * ks)), j1 = min(jhi, SR - R * st - (HK - R * ks));
+      if constexpr (VEC) {
+        star1_step_vec(src, dst, P1, N1, j0, j1, w, nullptr, nullptr, HK, rp, false, 0, 0, tid, NT);
+      } else {
+        const int nrow = j1 - j0;
+        for (int i = tid; i < nrow * N1; i += NT) {
+          const int j = j0 + i / N1, x = R + i % N1;
+          const double* cx = src + size_t(j) * P1 + x;
+          double th = 0.0;
+#pragma unroll
+          for (int b = -R; b <= R; ++b) th = fma(w.h[R + b], cx[b], th);
+          double acc = 0.0;
+#pragma unroll
+          for (int a = -R; a <= R; ++a) {
+            if (a == 0) acc += th;
+            acc = fma(w.v[R + a], cx[a * P1], acc);
+          }
+          dst[size_t(j) * P1 + x] = acc;
+        }
+      }
+      cur ^= 1;
+      __syncthreads();
+      strace(2 + t0 + st);
+    }
+    if (t0 + ks < T) {
+      double* res = cur ? buf1 : buf0;
+      double* mine = xch + (size_t(blk & 1) * G + c) * 2 * XB;
+      for (int i = tid; i < HK * N1; i += NT) {       // interior columns of my first / last HK own rows
+        const int r = i / N1, x = R + i % N1;
+        mine[size_t(r) * P1 + x] = res[size_t(HK + r) * P1 + x];
+        mine[XB + size_t(r) * P1 + x] = res[size_t(rp + r) * P1 + x];
+      }
+      // publish my rows (release), then wait only for the two neighbours' rows of this block (acquire):
+      // a CTA cannot run two blocks ahead of a neighbour, so two exchange parities suffice
+      __syncthreads();
+      if (tid == 0) {
+        __threadfence();
+        asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(flags + c), "l"(base + blk + 1) : "memory");
+        for (int nb = c - 1; nb <= c + 1; nb += 2) {
+          if (nb < 0 || nb >= G) continue;
+          unsigned long long v;
+          do {
+            asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(flags + nb) : "memory");
+          } while (v < base + blk + 1);
+        }
+      }
+      __syncthreads();
+      const double* lo = xch + (size_t(blk & 1) * G + (c - 1)) * 2 * XB + XB;   // c-1's last HK own rows
+      const double* hi = xch + (size_t(blk & 1) * G + (c + 1)) * 2 * XB;        // c+1's first HK own rows
+      for (int i = tid; i < HK * N1; i += NT) {
+        const int r = i / N1, x = R + i % N1;
+        if (c > 0) res[size_t(r) * P1 + x] = lo[size_t(r) * P1 + x];
+        if (c < G - 1) res[size_t(HK + rp + r) * P1 + x] = hi[size_t(r) * P1 + x];
+      }
+      __syncthreads();
+      strace(40 + blk);
+    }
+  }
+  const double* res = cur ? buf1 : buf0;
+  const int w0 = c == 0 ? HK - R : HK, w1 = c == G - 1 ? HK + rp + R : HK + rp;
+  for (int i = w0 * P1 + tid; i < w1 * P1; i += NT) out[int64_t(pr0) * P1 + i] = res[i];
+  strace(60);
 }
 
 // The two-arm star signature of the streaming engine (kernels_rdg.cu signature(), SIG_STAR).
@@ -296,9 +424,103 @@ bool small2d_eligible(const Plan& p) {
          star_arms(p, w) && cluster_size(p) > 0;
 }
 
+namespace {
+// Grid variant: rows per CTA (a divisor of N0, >= R) and the resulting CTA count; 0 if none fits.
+int grid_rows(const Plan& p, int maxG) {
+  int want = 4;
+  if (const char* e = std::getenv("LORA_SMALL_RP")) want = std::max(1, std::atoi(e));
+  int best = 0;
+  for (int rp = std::max(want, p.R); rp <= 64 && !best; ++rp)
+    if (p.N[0] % rp == 0 && p.N[0] / rp <= maxG && p.N[0] / rp >= 2) best = rp;
+  return best;
+}
+
+template <int R, bool VEC>
+cudaError_t grid_launch(const Plan& p, const double* in, double* out, double* xch, unsigned long long* flags,
+                        unsigned long long base, int rp, int kb, int T, int threads, size_t smem, const StarArms& w,
+                        cudaStream_t s) {
+  const void* k = (const void*)small2d_grid_kernel<R, VEC>;
+  if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) {
+    cudaGetLastError();
+    return cudaErrorNotSupported;
+  }
+  const int G = (int)(p.N[0] / rp);
+  int occ = 0, dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, threads, smem) != cudaSuccess || occ * sms < G) {
+    cudaGetLastError();
+    return cudaErrorNotSupported;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(G, 1, 1);
+  cfg.blockDim = dim3(threads, 1, 1);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at;
+  at.id = cudaLaunchAttributeCooperative;
+  at.val.cooperative = 1;
+  cfg.attrs = &at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, small2d_grid_kernel<R, VEC>, in, out, xch, flags, base, (int)p.N[0], (int)p.N[1], rp,
+                            T, kb, w);
+}
+
+cudaError_t launch_grid_variant(const Plan& p, const double* in, double* out, int64_t T, cudaStream_t s,
+                                const StarArms& w) {
+  if (const char* e = std::getenv("LORA_SMALL_MODE"); e && std::strcmp(e, "cluster") == 0) return cudaErrorNotSupported;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int rp = grid_rows(p, sms);
+  if (rp == 0) return cudaErrorNotSupported;
+  const int kb = (int)std::min<int64_t>(std::min(kMaxBlock, rp / p.R), T);
+  const int HK = kb * p.R, G = (int)(p.N[0] / rp);
+  const size_t smem = 2 * size_t(rp + 2 * HK) * size_t(p.P[1]) * sizeof(double);
+  if (smem > kMaxSmem) return cudaErrorNotSupported;
+  // exchange buffer [parity][CTA][side][HK][P1] followed by one 64-bit step counter per CTA
+  const size_t xdata = size_t(2) * G * 2 * HK * size_t(p.P[1]);
+  const size_t xelems = xdata + size_t(G);
+  Plan& mp = const_cast<Plan&>(p);
+  if (mp.xbuf_elems != xelems) {   // (re)allocated per geometry: the counters start at 0 again
+    if (mp.xbuf) cudaFree(mp.xbuf);
+    mp.xbuf = nullptr;
+    mp.xbuf_elems = 0;
+    if (cudaMalloc(&mp.xbuf, xelems * sizeof(double)) != cudaSuccess) { cudaGetLastError(); mp.xbuf = nullptr; return cudaErrorNotSupported; }
+    if (cudaMemsetAsync(mp.xbuf, 0, xelems * sizeof(double), s) != cudaSuccess) { cudaGetLastError(); return cudaErrorNotSupported; }
+    mp.xbuf_elems = xelems;
+    mp.xflag_base = 0;
+  }
+  // counters are monotonic across launches: this launch publishes base + 1 .. base + nblocks
+  unsigned long long* flags = reinterpret_cast<unsigned long long*>(mp.xbuf + (mp.xbuf_elems - size_t(G)));
+  const unsigned long long base = mp.xflag_base;
+  mp.xflag_base += (unsigned long long)((T + kb - 1) / kb) + 1;
+  const bool vec = p.R == 1 && (p.P[1] % 2) == 0;
+  const int qw = ((int)(p.P[1] / 2) + 31) / 32 * 32;
+  const int threads = vec ? std::max(1, GT_MAX / qw) * qw : 256;
+  if (vec && qw > GT_MAX) return cudaErrorNotSupported;
+  const int Ti = (int)T;
+  switch (p.R) {
+    case 1: return vec ? grid_launch<1, true>(p, in, out, mp.xbuf, flags, base, rp, kb, Ti, threads, smem, w, s)
+                       : grid_launch<1, false>(p, in, out, mp.xbuf, flags, base, rp, kb, Ti, threads, smem, w, s);
+    case 2: return grid_launch<2, false>(p, in, out, mp.xbuf, flags, base, rp, kb, Ti, threads, smem, w, s);
+    case 3: return grid_launch<3, false>(p, in, out, mp.xbuf, flags, base, rp, kb, Ti, threads, smem, w, s);
+    case 4: return grid_launch<4, false>(p, in, out, mp.xbuf, flags, base, rp, kb, Ti, threads, smem, w, s);
+  }
+  return cudaErrorNotSupported;
+}
+}  // namespace
+
+#ifdef SMALL_TRACE
+extern "C" int lora_small_trace(unsigned long long* h) { return (int)cudaMemcpyFromSymbol(h, g_small_trace, sizeof(unsigned long long) * 64); }
+#endif
 cudaError_t launch_small2d(const Plan& p, const double* in, double* out, int64_t T, cudaStream_t s) {
   StarArms w;
   if (!star_arms(p, w) || T < 1 || T > (int64_t(1) << 30)) return cudaErrorInvalidValue;
+  {
+    const cudaError_t eg = launch_grid_variant(p, in, out, T, s, w);
+    if (eg != cudaErrorNotSupported) return eg;
+  }
   int cs = cluster_size(p);
   if (cs == 0) return cudaErrorInvalidValue;
   const bool vec = p.R == 1 && (p.P[1] % 2) == 0;   // 16-byte rows: the register-walking R = 1 step

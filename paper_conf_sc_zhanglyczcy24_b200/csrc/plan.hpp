@@ -56,6 +56,9 @@ struct Plan {
   double* scratch = nullptr;      // one padded buffer for the ping-pong
   double* dev_in = nullptr;       // run_host staging (device copies of host in/out)
   double* dev_out = nullptr;
+  double* xbuf = nullptr;         // small-grid kernel: exchange buffer of the cooperative-grid variant
+  size_t xbuf_elems = 0;
+  unsigned long long xflag_base = 0;   // its per-CTA step counters are monotonic across launches
   size_t elems = 0;               // padded element count
   void* graph_exec = nullptr;     // cudaGraphExec_t of the cached time loop (small grids)
   const double* g_in = nullptr;   // its key

@@ -424,11 +424,15 @@ def test_small_cluster_path_bitwise(kind, h, shape, monkeypatch):
     W = synth.preset("heat2d") if kind == "heat2d" else synth.star_weights(2, h, 11 + h)
     g = synth.grid(tuple(n + 2 * h for n in shape), 20240101 + h)
     for T in (1, 2, 5, 10):
-        out, info = run_gpu(W, g, T)
+        out, info = run_gpu(W, g, T)                      # cooperative-grid variant (default)
         assert info["single_launch"] == 1, info
+        monkeypatch.setenv("LORA_SMALL_MODE", "cluster")  # the thread-block-cluster (DSMEM) variant
+        out_cl, _ = run_gpu(W, g, T)
+        monkeypatch.delenv("LORA_SMALL_MODE")
         monkeypatch.setenv("LORA_NO_SMALL", "1")
         ref_stream, info2 = run_gpu(W, g, T)
         monkeypatch.delenv("LORA_NO_SMALL")
         assert info2["single_launch"] == 0
         assert np.array_equal(out, ref_stream), (T, float(np.max(np.abs(out - ref_stream))))
+        assert np.array_equal(out_cl, ref_stream), (T, float(np.max(np.abs(out_cl - ref_stream))))
         assert rel_err(out, oracle.run(W, g, T)) <= 1e-12
