@@ -37,9 +37,12 @@ namespace {
 #endif                // CTA barrier at the end of the iteration, the stages of an iteration independent).
                       // Measured slower (r02m, same box): Box-3D27P k = 2 393 -> 379 GS/s, Heat-3D 449 -> 416
 constexpr int F_LAG = RDG3F_LAG;
-constexpr int F_WARPS = 8;
-constexpr int F_S1 = 16;             // stage-1 rows per CTA column (2 per warp); stage s: 16 - 2(s-1)
-constexpr int F_IN = 18;             // staged input rows
+#ifndef RDG3F_WARPS
+#define RDG3F_WARPS 8
+#endif
+constexpr int F_WARPS = RDG3F_WARPS;
+constexpr int F_S1 = 2 * F_WARPS;    // stage-1 rows per CTA column (2 per warp); stage s: F_S1 - 2(s-1)
+constexpr int F_IN = F_S1 + 2;       // staged input rows
 constexpr int F_BW = 66;             // staged columns (64 + 2R)
 constexpr int F_S1W = 72;            // step-1 plane buffer row pitch (doubles): data at [1, 65)
 constexpr int F_ZC = 64;
