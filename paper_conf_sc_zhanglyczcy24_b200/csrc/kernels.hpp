@@ -97,7 +97,7 @@ bool tc2d_supported(const Plan& p);
 // plans of the CUDA-core engine whose grid fits.  Bitwise equal to the streaming engine.
 // launch_small2d returns cudaErrorNotSupported when the device cannot schedule the cluster.
 bool small2d_eligible(const Plan& p);
-cudaError_t launch_small2d(const Plan& p, const double* in, double* out, int64_t T, cudaStream_t s);
+cudaError_t launch_small2d(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s);   // may allocate p.xbuf
 bool rdg3d_supported(const Plan& p);
 int rdg3d_p2p_units(const Plan& p, int* nux);
 cudaError_t launch_rdg3d_p2p(const Plan& p, const double* src, double* dst, cudaStream_t s, const P2PArgs& d);

@@ -427,8 +427,7 @@ bool small2d_eligible(const Plan& p) {
 namespace {
 // Grid variant: rows per CTA (a divisor of N0, >= R) and the resulting CTA count; 0 if none fits.
 int grid_rows(const Plan& p, int maxG) {
-  int want = 4;
-  if (const char* e = std::getenv("LORA_SMALL_RP")) want = std::max(1, std::atoi(e));
+  const int want = std::max(1, p.small_rp);
   int best = 0;
   for (int rp = std::max(want, p.R); rp <= 64 && !best; ++rp)
     if (p.N[0] % rp == 0 && p.N[0] / rp <= maxG && p.N[0] / rp >= 2) best = rp;
@@ -466,9 +465,9 @@ cudaError_t grid_launch(const Plan& p, const double* in, double* out, double* xc
                             T, kb, w);
 }
 
-cudaError_t launch_grid_variant(const Plan& p, const double* in, double* out, int64_t T, cudaStream_t s,
+cudaError_t launch_grid_variant(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s,
                                 const StarArms& w) {
-  if (const char* e = std::getenv("LORA_SMALL_MODE"); e && std::strcmp(e, "cluster") == 0) return cudaErrorNotSupported;
+  if (p.small_cluster_only) return cudaErrorNotSupported;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
@@ -481,7 +480,7 @@ cudaError_t launch_grid_variant(const Plan& p, const double* in, double* out, in
   // exchange buffer [parity][CTA][side][HK][P1] followed by one 64-bit step counter per CTA
   const size_t xdata = size_t(2) * G * 2 * HK * size_t(p.P[1]);
   const size_t xelems = xdata + size_t(G);
-  Plan& mp = const_cast<Plan&>(p);
+  Plan& mp = p;
   if (mp.xbuf_elems != xelems) {   // (re)allocated per geometry: the counters start at 0 again
     if (mp.xbuf) cudaFree(mp.xbuf);
     mp.xbuf = nullptr;
@@ -514,7 +513,7 @@ cudaError_t launch_grid_variant(const Plan& p, const double* in, double* out, in
 #ifdef SMALL_TRACE
 extern "C" int lora_small_trace(unsigned long long* h) { return (int)cudaMemcpyFromSymbol(h, g_small_trace, sizeof(unsigned long long) * 64); }
 #endif
-cudaError_t launch_small2d(const Plan& p, const double* in, double* out, int64_t T, cudaStream_t s) {
+cudaError_t launch_small2d(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s) {
   StarArms w;
   if (!star_arms(p, w) || T < 1 || T > (int64_t(1) << 30)) return cudaErrorInvalidValue;
   {

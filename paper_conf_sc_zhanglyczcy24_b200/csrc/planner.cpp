@@ -423,6 +423,10 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
     p.tc_no_bvs = (b && b[0] == '1') ? 1 : 0;
     const char* sm = std::getenv("LORA_NO_SMALL");
     p.no_small = (sm && sm[0] == '1') ? 1 : 0;
+    const char* smode = std::getenv("LORA_SMALL_MODE");   // tests: "cluster" = the DSMEM cluster variant
+    p.small_cluster_only = (smode && std::strcmp(smode, "cluster") == 0) ? 1 : 0;
+    const char* srp = std::getenv("LORA_SMALL_RP");       // experiments: rows per CTA of the grid variant
+    p.small_rp = srp ? std::max(1, std::atoi(srp)) : 4;
   }
   p.tile_m = eng == LORA_ENGINE_TC ? 64 : (p.ndim == 2 ? 64 : 8);
   p.tile_n = eng == LORA_ENGINE_TC ? 64 : 32;
