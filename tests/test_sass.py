@@ -57,7 +57,7 @@ def test_no_bvs_ablation_shuffles(sass):
 
 def test_tma_staging(sass):
     for pat in (r"tc2d_kernelILi\dELb1ELb0E", r"tc3d_kernelILi1ELb1E", r"rdg2d_kernelILi\dELi\dELi\dELb1E",
-                r"rdg3df_kernel.*ELb1E"):
+                r"rdg3df_kernel.*ELi\dELb1ELb[01]E"):
         for name, body in _pick(sass, pat).items():
             assert any(o.startswith("UTMALDG") for o in _ops(body)), name
 
