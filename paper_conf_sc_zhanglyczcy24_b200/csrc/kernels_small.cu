@@ -482,6 +482,11 @@ cudaError_t launch_grid_variant(Plan& p, const double* in, double* out, int64_t 
   const size_t xelems = xdata + size_t(G);
   Plan& mp = p;
   if (mp.xbuf_elems != xelems) {   // (re)allocated per geometry: the counters start at 0 again
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(s, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) {
+      cudaGetLastError();
+      return cudaErrorNotSupported;   // no allocation inside the caller's graph capture: cluster variant
+    }
     if (mp.xbuf) cudaFree(mp.xbuf);
     mp.xbuf = nullptr;
     mp.xbuf_elems = 0;
