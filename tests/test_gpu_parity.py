@@ -66,6 +66,21 @@ def test_integer_exact_bitwise(engine):
     assert np.array_equal(out, ref)
 
 
+@pytest.mark.parametrize("engine,fuse_k", [("rdg_cuda", 0), ("rdg_cuda", 1), ("direct", 0), ("tc", 0)])
+def test_integer_exact_bitwise_3d(engine, fuse_k):
+    """P9 in 3D (SURVEY §8(c) parity matrix: 64³): an integer 27-point box whose planes are rank-1 +
+    centre (PMA recovers them with dyadic unit-centre factors), inputs in {0..3}, T one below the
+    2^53 bound => every intermediate is exact and the GPU result equals the oracle bitwise, for the
+    fused (default k = 2) and unfused CUDA-core kernels, the direct kernel and the tensor-core chain."""
+    import math
+    W = np.array([[[1, 2, 1], [2, 4, 2], [1, 2, 1]], [[2, 4, 2], [4, 9, 4], [2, 4, 2]],
+                  [[1, 2, 1], [2, 4, 2], [1, 2, 1]]], dtype=np.float64)
+    T = int((53 - math.log2(3)) // math.log2(np.abs(W).sum())) - 1
+    g = synth.integer_grid((66, 66, 66), 98)
+    out, _ = run_gpu(W, g, T, engine=engine, fuse_k=fuse_k)
+    assert np.array_equal(out, oracle.run(W, g, T)), T
+
+
 ENGINES_3D = ["direct", "rdg_cuda", "tc"]
 
 
