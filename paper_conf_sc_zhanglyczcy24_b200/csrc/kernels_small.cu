@@ -25,6 +25,7 @@
 #include <cstring>
 #include <map>
 #include <mutex>
+#include <tuple>
 
 #include "kernels.hpp"
 
@@ -439,17 +440,24 @@ cudaError_t grid_launch(const Plan& p, const double* in, double* out, double* xc
                         unsigned long long base, int rp, int kb, int T, int threads, size_t smem, const StarArms& w,
                         cudaStream_t s) {
   const void* k = (const void*)small2d_grid_kernel<R, VEC>;
-  if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) {
-    cudaGetLastError();
-    return cudaErrorNotSupported;
-  }
   const int G = (int)(p.N[0] / rp);
-  int occ = 0, dev = 0, sms = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, threads, smem) != cudaSuccess || occ * sms < G) {
-    cudaGetLastError();
-    return cudaErrorNotSupported;
+  {  // per (device, threads, smem): the attribute and the co-residency bound, computed once
+    static std::mutex mu;
+    static std::map<std::tuple<int, int, size_t>, int> cap;   // -> resident CTAs on the device (0: unusable)
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return cudaErrorNotSupported; }
+    std::lock_guard<std::mutex> lock(mu);
+    auto it = cap.find({dev, threads, smem});
+    if (it == cap.end()) {
+      int occ = 0, sms = 0, resident = 0;
+      cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+      if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem) == cudaSuccess &&
+          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, threads, smem) == cudaSuccess)
+        resident = occ * sms;
+      cudaGetLastError();
+      it = cap.emplace(std::make_tuple(dev, threads, smem), resident).first;
+    }
+    if (it->second < G) return cudaErrorNotSupported;
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(G, 1, 1);
