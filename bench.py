@@ -397,6 +397,13 @@ def main():
     tr = ncu_traffic(args.workload, info["engine_name"])
     if tr and int(tr.get("fuse", 1)) != fuse:
         tr = None
+    if tr and tr.get("fp64_lane_ops"):
+        # EXECUTED FP64 lane-ops per launch (ncu op counters, incl. the redundant halo recomputation)
+        ex = float(tr["fp64_lane_ops"])
+        roof["views"]["fp64_executed"] = {"achieved": ex / roof["avg_launch_ms"] * 1e3 / 1e9, "peak": fp64_peak / 1e9,
+                                          "unit": "GFP64-op/s",
+                                          "frac": ex / (roof["avg_launch_ms"] * 1e-3) / fp64_peak,
+                                          "executed_ops_per_launch": ex, "source": tr.get("fp64_lane_ops_source")}
     roof.update({"traffic": tr["bytes"] if tr else None,       # dram read+write bytes per launch (ncu --set full)
                  "traffic_source": ({k: tr[k] for k in ("kernel", "source", "fuse")} if tr else None),
                  "kernel": f"{info['engine_name']} stencil step (fuse_k={fuse})",
@@ -605,8 +612,9 @@ def main():
                            "l2": "inputs (%.2f GB per buffer) larger than the 126 MB L2" % (8 * np.prod(padded) / 1e9)},
                 "clocks": clk.summary(), "gpu_launches": launches_per_step * args.steps,
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
-                "fma_per_point": {"issued": info["fma_per_point_issued"], "direct": info["fma_per_point_direct"],
-                                  "separable": info["fma_per_point_separable"]},
+                "fp64_ops_per_point_step": {"chosen_form": info["fma_per_point_issued"],
+                                            "direct_taps": info["fma_per_point_direct"],
+                                            "separable_terms": info["fma_per_point_separable"]},
                 "host": host_info()}
         if per_config:
             line["configs"] = per_config
