@@ -528,7 +528,8 @@ extern "C" int lora_small_trace(unsigned long long* h) { return (int)cudaMemcpyF
 #endif
 cudaError_t launch_small2d(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s) {
   StarArms w;
-  if (!star_arms(p, w) || T < 1 || T > (int64_t(1) << 30)) return cudaErrorInvalidValue;
+  if (!star_arms(p, w) || T < 1) return cudaErrorInvalidValue;
+  if (T > (int64_t(1) << 30)) return cudaErrorNotSupported;   // (int step counts) the per-step path runs it
   {
     const cudaError_t eg = launch_grid_variant(p, in, out, T, s, w);
     if (eg != cudaErrorNotSupported) return eg;
