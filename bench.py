@@ -566,8 +566,9 @@ def main():
                 if eng == "rdg_cuda_pma":   # the paper's PMA pyramid on the CUDA-core engine (LORA_RDG_PMA=1)
                     os.environ["LORA_RDG_PMA"] = "1"
                 try:
+                    # the PMA form at the headline's fusion depth (its own planner default is unfused)
                     s3 = L.Stencil(W, shape, engine=eng[:8] if eng.startswith("rdg_cuda") else eng,
-                                   fuse_k=1 if eng == "rdg_cuda_k1" else 0)
+                                   fuse_k=1 if eng == "rdg_cuda_k1" else (info["fuse_k"] if eng == "rdg_cuda_pma" else 0))
                 finally:
                     os.environ.pop("LORA_RDG_PMA", None)
             except L.LoraError as ex:
