@@ -255,6 +255,9 @@ int lora_stencil_run_dist(lora_plan* p, lora_comm* c, const double* in_local, do
   const char* b = reinterpret_cast<const char*>(out_local);
   if (a < b + bytes && b < a + bytes) return fail(LORA_ERR_ALIAS, "in and out overlap");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  int dev = -1;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev != c->device)
+    return fail(LORA_ERR_INVALID_ARG, "communicator is bound to another CUDA device");
   if (timesteps == 0) {
     cudaError_t e = cudaMemcpyAsync(out_local, in_local, bytes, cudaMemcpyDeviceToDevice, s);
     return e == cudaSuccess ? LORA_OK : cuda_fail(e, "cudaMemcpyAsync");
