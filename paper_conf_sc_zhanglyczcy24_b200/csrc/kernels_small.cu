@@ -199,7 +199,13 @@ small2d_star_kernel(const double* __restrict__ in, double* __restrict__ out, int
 // block of k steps every CTA copies its first / last kR own rows into a global exchange buffer
 // (two parities x G CTAs x 2 sides), one grid-wide barrier (cooperative groups) publishes them, and
 // each CTA unpacks its neighbours' rows into its halo.  Same per-point arithmetic (bitwise equal).
-constexpr int GT_MAX = 512;
+#ifndef SMALL_GT_MAX
+#define SMALL_GT_MAX 512
+#endif
+constexpr int GT_MAX = SMALL_GT_MAX;   // threads per CTA of the grid variant (whole strips of column pairs)
+#ifndef SMALL_ONE_BLOCK_MAX_HALO
+#define SMALL_ONE_BLOCK_MAX_HALO 16   // halo rows up to which a whole run is one block (no exchange)
+#endif
 #ifdef SMALL_TRACE
 __device__ unsigned long long g_small_trace[64];
 __device__ __forceinline__ void strace(int k) {
@@ -451,7 +457,14 @@ cudaError_t grid_launch(const Plan& p, const double* in, double* out, double* xc
     if (it == cap.end()) {
       int occ = 0, sms = 0, resident = 0;
       cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-      if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem) == cudaSuccess &&
+#ifndef SMALL_ATTR_EXACT
+#define SMALL_ATTR_EXACT 0
+#endif
+      const int attr = SMALL_ATTR_EXACT ? (int)smem : (int)kMaxSmem;
+#ifdef SMALL_CARVEOUT
+      cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, SMALL_CARVEOUT);
+#endif
+      if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, attr) == cudaSuccess &&
           cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, threads, smem) == cudaSuccess)
         resident = occ * sms;
       cudaGetLastError();
@@ -481,7 +494,11 @@ cudaError_t launch_grid_variant(Plan& p, const double* in, double* out, int64_t 
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const int rp = grid_rows(p, sms);
   if (rp == 0) return cudaErrorNotSupported;
-  const int kb = (int)std::min<int64_t>(std::min(kMaxBlock, rp / p.R), T);
+  // a short run in ONE block (halo T R rows deep, all of it staged from `in`: no exchange at all, the
+  // redundant halo rows are cheaper than a neighbour wait); longer runs in blocks of k <= rp / R steps
+  const size_t one_block = 2 * size_t(rp + 2 * T * p.R) * size_t(p.P[1]) * sizeof(double);
+  const int kb = (T * p.R <= SMALL_ONE_BLOCK_MAX_HALO && one_block <= kMaxSmem)
+                     ? (int)T : (int)std::min<int64_t>(std::min(kMaxBlock, rp / p.R), T);
   const int HK = kb * p.R, G = (int)(p.N[0] / rp);
   const size_t smem = 2 * size_t(rp + 2 * HK) * size_t(p.P[1]) * sizeof(double);
   if (smem > kMaxSmem) return cudaErrorNotSupported;

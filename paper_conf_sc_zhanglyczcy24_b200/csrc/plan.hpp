@@ -43,7 +43,7 @@ struct Plan {
   int tc_no_bvs = 0;
   int no_small = 0;       // LORA_NO_SMALL=1: no single-launch path for small 2D grids (tests)
   int small_cluster_only = 0;   // LORA_SMALL_MODE=cluster: the cluster variant of that path (tests)
-  int small_rp = 4;       // LORA_SMALL_RP: rows per CTA of its cooperative-grid variant (experiments)      // LORA_TC_NO_BVS=1: the Fig. 9 ablation (shuffle-based stage 2) in the TC engine
+  int small_rp = 2;       // LORA_SMALL_RP: rows per CTA of its cooperative-grid variant (experiments)      // LORA_TC_NO_BVS=1: the Fig. 9 ablation (shuffle-based stage 2) in the TC engine
   int n_planes_point = 0;
   // CUDA-core engine, 2D, radius >= 3, W reflection-symmetric in both axes with a nonzero centre
   // column: evaluate W as the row-pair rank-1 split u_a = c_a (e_{R+a} + e_{R-a}), v_a = W[R+a,:] / c_a

@@ -426,7 +426,7 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
     const char* smode = std::getenv("LORA_SMALL_MODE");   // tests: "cluster" = the DSMEM cluster variant
     p.small_cluster_only = (smode && std::strcmp(smode, "cluster") == 0) ? 1 : 0;
     const char* srp = std::getenv("LORA_SMALL_RP");       // experiments: rows per CTA of the grid variant
-    p.small_rp = srp ? std::max(1, std::atoi(srp)) : 4;
+    p.small_rp = srp ? std::max(1, std::atoi(srp)) : 2;   // Heat-2D 256^2 x 10: 2 -> 14.8 us, 4 -> 15.8, 8 -> 18.1
   }
   p.tile_m = eng == LORA_ENGINE_TC ? 64 : (p.ndim == 2 ? 64 : 8);
   p.tile_n = eng == LORA_ENGINE_TC ? 64 : 32;
