@@ -82,7 +82,10 @@ typedef struct {               /* filled by lora_stencil_plan_query             
                                   holding the grid in shared memory (DSMEM halo exchange)       */
   double recon_err;            /* max|sum u v^T - W| / max|W|                                 */
   double growth;               /* sum_k ||u_k||_1 ||v_k||_1 / ||W||_1                         */
-  double fma_per_point_issued; /* FP64 FMAs issued per point per step by the chosen engine    */
+  double fma_per_point_issued; /* FP64 work per point per step of the chosen engine's rank-1
+                                  form: DFMA/DADD/DMUL lane-ops (CUDA-core engines) or DMMA FMA
+                                  slots incl. band padding (tensor-core engine); halo recompute
+                                  of fused launches not counted                                  */
   double fma_per_point_direct; /* (2r+1)^d, nonzero weights only                              */
   double fma_per_point_separable; /* sum over terms of (len u + len v) + point-wise terms      */
   /* The paper's analytic cost model for its A100 tiling at the plan's radius h (host arithmetic on
