@@ -1,14 +1,21 @@
 // Small 2D grids (BASELINE configs[0], Heat-2D 256^2 x 10): ONE launch runs all T time steps.
 //
 // The per-step launches of the streaming engine leave a 0.5 MB problem launch- and latency-bound
-// (r01: 9.7 GStencil/s with CUDA-graph replay).  Here the whole padded grid lives in the shared
-// memory of one thread-block cluster (the B200 rules: distributed shared memory
-// between the CTAs of a cluster): CTA c of CS owns rp = N0 / CS interior rows plus an R-row halo on
-// each side, in two ping-pong buffers.  A step computes the CTA's own rows from buffer `cur` into
-// `nxt`; the first / last R of them are also stored straight into the neighbour CTA's halo rows of
-// `nxt` through DSMEM (st.shared::cluster via cluster.map_shared_rank); one cluster barrier per
-// step (release/acquire) publishes them.  The column halo and the top / bottom halo rows of the
-// grid are the Dirichlet values (loaded into both buffers, never written; Q1).
+// (r01: 9.7 GStencil/s with CUDA-graph replay).  Two single-launch variants:
+//
+// * cooperative grid (default, small2d_grid_kernel): G = N0 / rp co-resident CTAs, CTA c owns rp
+//   interior rows plus a kR-deep halo on each side in two shared-memory ping-pong buffers.  A block
+//   of k steps runs on a shrinking row range (step s of a block computes the rows that are still
+//   valid: own rows plus (k - s) R halo rows each side).  A short run (T R <= 16) is ONE block whose
+//   halo is staged from `in` (no exchange at all); longer runs exchange the first / last kR own rows
+//   through a global buffer after each block, each CTA waiting only for its two neighbours' step
+//   counters (release / acquire at gpu scope).
+// * thread-block cluster (fallback, small2d_star_kernel): the same slab / block scheme with the whole
+//   grid in the shared memory of one cluster of <= 16 CTAs and the exchange through the neighbours'
+//   DSMEM mailboxes (st.shared::cluster via cluster.map_shared_rank), one cluster barrier per block.
+//
+// The column halo and the top / bottom halo rows of the grid are the Dirichlet values (loaded into
+// both buffers, never written; Q1).
 //
 // Arithmetic: the two star arms of the planner (horizontal arm u = e_R, v = W[R,:]; vertical arm
 // u = W[:,R] with the centre in the horizontal arm, v = e_R — planner.cpp factor_plane (i)) in
