@@ -257,6 +257,9 @@ void lora_stencil_p2p_destroy(lora_p2p* c);
 
 /* Thread-local message for the last failure on this thread ("" if none). */
 const char* lora_stencil_last_error(void);
+/* Thread-local lora_status of the last failure on this thread (LORA_OK after a successful
+ * lora_stencil_plan / _plan_ex): the reason a plan call returned NULL. */
+int lora_stencil_last_status(void);
 /* Library version string. */
 const char* lora_stencil_version(void);
 

@@ -91,6 +91,7 @@ _sig = {
     "lora_stencil_p2p_status": (ctypes.c_int, [_P]),
     "lora_stencil_p2p_destroy": (None, [_P]),
     "lora_stencil_last_error": (ctypes.c_char_p, []),
+    "lora_stencil_last_status": (ctypes.c_int, []),
     "lora_stencil_version": (ctypes.c_char_p, []),
 }
 for _name, (_res, _args) in _sig.items():
@@ -130,7 +131,7 @@ def lora_stencil_plan_ex(weights, ndim: int, radius: int, grid_shape, engine=0, 
     opts = lora_plan_opts(engine=int(engine), fuse_k=int(fuse_k))
     h = _lib.lora_stencil_plan_ex(w.ctypes.data, int(ndim), int(radius), g.ctypes.data, ctypes.byref(opts))
     if not h:
-        raise LoraError(-1, lora_stencil_last_error())
+        raise LoraError(int(_lib.lora_stencil_last_status()), lora_stencil_last_error())
     return h
 
 

@@ -16,9 +16,11 @@
 
 namespace lora {
 thread_local std::string g_err;
-int fail(int code, const std::string& msg) { g_err = msg; return code; }
+thread_local int g_status = LORA_OK;   // status of the last failure on this thread (plan creation returns NULL)
+int fail(int code, const std::string& msg) { g_err = msg; g_status = code; return code; }
 int cuda_fail(int e, const char* what) {
   g_err = std::string(what) + ": " + cudaGetErrorString(static_cast<cudaError_t>(e));
+  g_status = LORA_ERR_CUDA;
   return LORA_ERR_CUDA;
 }
 bool sync_check() {
@@ -174,16 +176,18 @@ using namespace lora;
 extern "C" {
 
 const char* lora_stencil_last_error(void) { return g_err.c_str(); }
+int lora_stencil_last_status(void) { return g_status; }
 const char* lora_stencil_version(void) { return "lora_stencil_b200 0.1 (sm_100a)"; }
 
 lora_plan* lora_stencil_plan_ex(const double* weights, int ndim, int radius, const int64_t* grid_shape,
                                 const lora_plan_opts* opts) {
   lora_plan* p = new (std::nothrow) lora_plan();
-  if (!p) { g_err = "out of host memory"; return nullptr; }
+  if (!p) { g_err = "out of host memory"; g_status = LORA_ERR_OOM; return nullptr; }
   std::string err;
   int rc = plan_build(*p, weights, ndim, radius, grid_shape, opts, err);
-  if (rc != LORA_OK) { g_err = err; delete p; return nullptr; }
+  if (rc != LORA_OK) { g_err = err; g_status = rc; delete p; return nullptr; }
   g_err.clear();
+  g_status = LORA_OK;
   return p;
 }
 

@@ -254,3 +254,19 @@ def test_single_launch_path_selection(L, monkeypatch):
     assert L.Stencil(W2, (256, 256)).info()["single_launch"] == 0         # not a star
     monkeypatch.setenv("LORA_NO_SMALL", "1")
     assert L.Stencil(W, c["shape"]).info()["single_launch"] == 0
+
+
+def test_plan_failure_status_codes(L):
+    """lora_stencil_last_status reports why a plan call returned NULL (the binding raises it)."""
+    W = synth.rsym_weights(2, 1, 1)
+    with pytest.raises(L.LoraError) as e:
+        L.lora_stencil_plan(W, 2, 1, [0, 10])
+    assert e.value.code == L.LORA_ERR_INVALID_ARG
+    with pytest.raises(L.LoraError) as e:
+        L.lora_stencil_plan(np.zeros((11, 11)), 2, 5, [10, 10])
+    assert e.value.code == L.LORA_ERR_UNSUPPORTED
+    with pytest.raises(L.LoraError) as e:
+        L.Stencil(synth.preset("heat1d"), (100,), engine="tc")
+    assert e.value.code == L.LORA_ERR_UNSUPPORTED
+    L.lora_stencil_plan(W, 2, 1, [10, 10])
+    assert L._lib.lora_stencil_last_status() == L.LORA_OK
