@@ -50,7 +50,7 @@ def _weights(kind, d, h, seed):
     return W / W.sum()
 
 
-@pytest.mark.parametrize("i", range(60))
+@pytest.mark.parametrize("i", range(240))
 def test_random_case_matches_oracle(i, monkeypatch):
     d, h, kind, shape, T, engine, fuse, no_tma, seed = _case(i)
     W = _weights(kind, d, h, seed)
