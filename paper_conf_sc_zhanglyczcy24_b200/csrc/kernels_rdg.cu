@@ -631,7 +631,12 @@ constexpr int rdg_minb() {
                                                                                         : ((K == 1 || R == 1) ? 4 : 3)));
 }
 
-template <int R, int SIG, int K, bool TMA>
+// P2P: the device-initiated exchange hooks (csrc/dist_p2p.cu) are compiled in.  The single-GPU
+// instantiation has none: with the spin-wait code in the kernel ptxas keeps the stencil weights in
+// vector registers (three vector operands per DFMA); without it they live in uniform registers
+// (DFMA R, R, UR, R), which the FP64 pipe issues faster (tools/ubench/fp64_mix.cu: +20 % for this
+// instruction mix) and which frees 32 vector registers per thread.
+template <int R, int SIG, int K, bool TMA, bool P2P>
 __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d_kernel(const double* __restrict__ in, double* __restrict__ out,
                                                               int64_t N0, int64_t N1, int nbands, int nitems, int RC,
                                                               int SI, const __grid_constant__ CUtensorMap tmap,
@@ -643,6 +648,7 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
   constexpr int BS = 64 * NH - 2 * R * (K - 1) - 2 * SG;  // band stride (valid final columns per band)
   constexpr int BUFD = G::BUFD;
   extern __shared__ __align__(128) unsigned char smem_raw[];
+  const bool dact = P2P && dp.active;
   const int lane = threadIdx.x & 31;
   // the warp index through a shuffle from lane 0: ptxas then knows it (and all item geometry derived
   // from it) is warp-uniform — uniform branches and uniform-datapath address arithmetic
@@ -667,7 +673,7 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
   const int nch = nitems / nbands;
   auto geom = [&](int item, int& X0, int& A) {
     const int band = item % nbands;
-    const int chunk = dp.active ? p2p_chunk_order(item / nbands, nch) : item / nbands;
+    const int chunk = dact ? p2p_chunk_order(item / nbands, nch) : item / nbands;
     X0 = R + band * BS - R * (K - 1) - SG;
     A = R + chunk * RC;
   };
@@ -675,15 +681,15 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
   // lower (upper) neighbour — it stores them into the neighbour's halo and stages the halo the
   // neighbour wrote; the host keeps that item unique per band (RC >= 2H, last chunk >= 2H - R rows)
   auto touches = [&](int A_, bool& lo, bool& hi) {
-    lo = dp.active && dp.dst_lo != nullptr && A_ < dp.lo_end;
-    hi = dp.active && dp.dst_hi != nullptr && A_ + RC - 1 >= dp.hi_begin;
+    lo = dact && dp.dst_lo != nullptr && A_ < dp.lo_end;
+    hi = dact && dp.dst_hi != nullptr && A_ + RC - 1 >= dp.hi_begin;
   };
   // producer position (next stage to stage into the ring)
   int pitem = gw, pj = 0, pX0 = 0, pA = 0;
   if (gw < nitems) geom(pitem, pX0, pA);
   auto issue_next = [&](int slot) {
     const int x = pX0 - R, y = pA - K * R + pj * G::SROWS;
-    if (dp.active && pj == 0) {  // the halo this item stages was written by a neighbour: wait for it
+    if (dact && pj == 0) {  // the halo this item stages was written by a neighbour: wait for it
       bool lo, hi;
       touches(pA, lo, hi);
       if (lane == 0 && (lo || hi)) {
@@ -762,7 +768,7 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
         lc.vec[h] = lc.valid[h][0] && lc.valid[h][1] &&
                     ((reinterpret_cast<uintptr_t>(out + lc.c0 + 64 * h) & 15) == 0) && ((P1 & 1) == 0);
       }
-      rows_valid_end = min(A + RC, dp.active ? dp.store_hi : P0 - R);
+      rows_valid_end = min(A + RC, dact ? dp.store_hi : P0 - R);
       // FULL lanes: no halo columns; a pair is stored as a whole or not at all — one 16-byte store
       // for even R; for odd R the lane columns X0 + 2p are odd (the staged origin X0 - R is kept
       // even for TMA), so the pair is two 8-byte stores
@@ -778,7 +784,7 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
     const int yb = A - K * R + cj * G::SROWS;
     {
       const int yf = yb - K * R - (K - 1);  // final row produced by input row I = 0 (one-row lag per stage)
-      sc.lo = (dp.active ? max(A, dp.store_lo) : A) - yf;
+      sc.lo = (dact ? max(A, dp.store_lo) : A) - yf;
       sc.hi = rows_valid_end - yf;
       sc.ooff = int64_t(yf) * P1 + lc.c0;
       sc.rem_lo = t_lo ? dp.lo_end - yf : INT_MIN;       // rows [store_lo, lo_end)
@@ -878,7 +884,8 @@ cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream
   const int smem = 128 + RDG_WARPS * (G::WARP_BYTES + 2 * (K - 1) * BUFD * 8);
   int max_grid = 0;
   {
-    cudaError_t e = kernel_setup((const void*)rdg2d_kernel<R, SIG, K, TMA>, RDG_WARPS * 32, smem, &max_grid);
+    cudaError_t e = d && d->active ? kernel_setup((const void*)rdg2d_kernel<R, SIG, K, TMA, true>, RDG_WARPS * 32, smem, &max_grid)
+                                   : kernel_setup((const void*)rdg2d_kernel<R, SIG, K, TMA, false>, RDG_WARPS * 32, smem, &max_grid);
     if (e != cudaSuccess) return e;
   }
   if (d && d->prepare_only) return cudaSuccess;
@@ -919,8 +926,12 @@ cudaError_t rdg_launch(const Plan& p, const double* src, double* dst, cudaStream
   const int nitems = nbands * nchunks;
   const int grid = (int)std::min<int64_t>(max_grid, (nitems + RDG_WARPS - 1) / RDG_WARPS);
   static const P2PArgs none{};
-  rdg2d_kernel<R, SIG, K, TMA><<<grid, RDG_WARPS * 32, smem, s>>>(src, dst, p.N[0], p.N[1], nbands, nitems, RC, SI,
-                                                                   map, prm, d ? *d : none);
+  if (d && d->active)
+    rdg2d_kernel<R, SIG, K, TMA, true><<<grid, RDG_WARPS * 32, smem, s>>>(src, dst, p.N[0], p.N[1], nbands, nitems, RC, SI,
+                                                                         map, prm, *d);
+  else
+    rdg2d_kernel<R, SIG, K, TMA, false><<<grid, RDG_WARPS * 32, smem, s>>>(src, dst, p.N[0], p.N[1], nbands, nitems, RC,
+                                                                          SI, map, prm, none);
   return cudaGetLastError();
 }
 
