@@ -692,12 +692,12 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
     if (dact && pj == 0) {  // the halo this item stages was written by a neighbour: wait for it
       bool lo, hi;
       touches(pA, lo, hi);
-      if (lane == 0 && (lo || hi)) {
+      if (lo || hi) {   // warp-uniform
         const int b = pitem % nbands;
         const int u0 = dp.wait_units > 0 ? 0 : max(b - 1, 0), u1 = dp.wait_units > 0 ? dp.wait_units - 1 : min(b + 1, nbands - 1);
-        if (lo) p2p_wait_units(dp.wait_lo, u0, u1, dp.wait_val, dp.err);
-        if (hi) p2p_wait_units(dp.wait_hi, u0, u1, dp.wait_val, dp.err);
-        fence_proxy_async_global();
+        if (lo) p2p_wait_units_warp(dp.wait_lo, u0, u1, dp.wait_val, dp.err);
+        if (hi) p2p_wait_units_warp(dp.wait_hi, u0, u1, dp.wait_val, dp.err);
+        if (lane == 0) fence_proxy_async_global();
       }
       __syncwarp();
     }

@@ -62,6 +62,34 @@ __device__ __forceinline__ void p2p_wait_units(const unsigned long long* flags, 
   }
 }
 
+// Warp-uniform form of p2p_wait_units, called by EVERY lane of a warp: lane 0 does the acquire
+// loads and the timeout bookkeeping, the loop decisions are broadcast by shuffles, so the loop
+// exits are warp-uniform.  (A spin loop of lane 0 alone inside the 2D stream kernel made ptxas keep
+// the stencil weights in vector registers for the whole kernel: 364 vs 429 GS/s single-GPU.)
+__device__ __forceinline__ void p2p_wait_units_warp(const unsigned long long* flags, int u0, int u1,
+                                                    unsigned long long val, int* err) {
+  const bool l0 = (threadIdx.x & 31) == 0;
+  unsigned long long t0 = 0;
+  for (int u = u0; u <= u1; ++u) {
+    for (;;) {
+      int st = 0;   // 0: wait, 1: ready, 2: give up
+      if (l0) {
+        if (p2p_ld_acquire(flags + u) >= val) st = 1;
+        else if (*reinterpret_cast<volatile int*>(err)) st = 2;
+        else {
+          const unsigned long long now = p2p_clock_ns();
+          if (t0 == 0) t0 = now;
+          else if (now - t0 > kP2PTimeoutNs) { atomicExch(err, 1); st = 2; }
+        }
+      }
+      st = __shfl_sync(0xffffffffu, st, 0);
+      if (st == 2) return;
+      if (st == 1) break;
+      __nanosleep(128);
+    }
+  }
+}
+
 // Called by every lane of the warp after its last store of a boundary item: publishes `val` in the
 // peer's flag `u` once every lane's stores are visible system-wide.
 __device__ __forceinline__ void p2p_signal_warp(unsigned long long* peer_flags, int u, unsigned long long val) {
