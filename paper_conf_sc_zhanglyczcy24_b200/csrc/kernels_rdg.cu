@@ -488,11 +488,13 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
 }
 
 #ifndef RDG_PF
-#define RDG_PF 3   // fused kernels of radius >= RDG_PF: prefetch the next staged input row (0: never)
+#define RDG_PF 0   // fused kernels of radius >= RDG_PF: prefetch the next staged input row (0: never)
 #endif
 #ifndef RDG_PF2
 #define RDG_PF2 2  // K = 2: also load stage 2's input row before stage 1's work — 1: always, 2: star
 #endif             // arms only (Star-2D13P 435 -> 451 GS/s; Box-2D49P 322 -> 290: register spills), 0: never
+// Default off since the weights moved to uniform registers (r02v/r02w, same box): Box-2D49P k = 2
+// 428 -> 449 GS/s without the prefetch (202 instead of 230 registers).
 // Fused kernels with RDG_PF: stage 1 runs first on the row prefetched in the previous iteration,
 // then the next staged row (same TMA stage) is loaded into xq, then stages K .. 2 run — their FP64
 // work covers the shared-load latency of the next stage-1 row (which the per-row __syncwarp keeps
