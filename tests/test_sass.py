@@ -67,3 +67,17 @@ def test_cuda_core_engine_has_no_dmma(sass):
         ops = _ops(body)
         assert any(o.startswith("DFMA") for o in ops), name
         assert not any(o.startswith("DMMA") for o in ops), name
+
+
+def test_stencil_weights_in_uniform_registers(sass):
+    # DESIGN.md §6 "Uniform-register weights": every DFMA of the fused 2D row-pair / PMA / star kernels
+    # (single-GPU AND device-initiated-exchange instantiations) and of the fused 3D kernel takes its
+    # weight from a uniform register (DFMA R, R, URx, R); a lane-0-only spin loop in the kernel made
+    # ptxas keep the weights in vector registers (364 vs 429 GS/s on Box-2D49P)
+    pats = (r"rdg2d_kernelILi\dELi[014]ELi[234]ELb[01]ELb[01]E", r"rdg3df_kernel.*ELi2ELb1ELb[01]E")
+    for pat in pats:
+        for name, body in _pick(sass, pat).items():
+            dfma = [ln for ln in body.splitlines() if re.search(r"\bDFMA\b", ln)]
+            assert dfma, name
+            vec = [ln for ln in dfma if not re.search(r"\bUR\d+", ln)]
+            assert len(vec) <= len(dfma) // 50, (name, len(vec), len(dfma), vec[:3])
