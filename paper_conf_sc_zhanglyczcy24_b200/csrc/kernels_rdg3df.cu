@@ -37,6 +37,9 @@ namespace {
 #endif                // CTA barrier at the end of the iteration, the stages of an iteration independent).
                       // Measured slower (r02m, same box): Box-3D27P k = 2 393 -> 379 GS/s, Heat-3D 449 -> 416
 constexpr int F_LAG = RDG3F_LAG;
+#ifndef RDG3F_HALO_Z
+#define RDG3F_HALO_Z 1   // stage-1 Dirichlet fetch with the x/y masks precomputed per item (halo_fetch_z)
+#endif
 #ifndef RDG3F_WARPS
 #define RDG3F_WARPS 8
 #endif
@@ -208,6 +211,21 @@ __device__ __forceinline__ unsigned halo_fetch(int w, int lane, int Y0, int X0, 
   return m;
 }
 
+// The same with the x/y part precomputed per item (halo_xy: in_xy = elements inside the array's
+// x/y range, hal_xy = those of them on the x/y Dirichlet ring; base = the element (0, 0) offset
+// gy * P2 + cx within a plane): per plane only the z tests and the loads of flagged elements.
+__device__ __forceinline__ unsigned halo_fetch_z(int zs, int P0, int64_t P12, int P2, unsigned in_xy, unsigned hal_xy,
+                                                 int64_t base, const double* __restrict__ in, double (&hv)[2][2]) {
+  const bool zin = zs >= 0 && zs < P0, zh = zs < 1 || zs >= P0 - 1;
+  const unsigned ld = zin ? (zh ? in_xy : hal_xy) : 0u;        // elements taking an input value
+  const double* src = in + (int64_t(zs) * P12 + base);
+#pragma unroll
+  for (int y = 0; y < 2; ++y)
+#pragma unroll
+    for (int e = 0; e < 2; ++e) hv[y][e] = ((ld >> (2 * y + e)) & 1u) ? src[y * P2 + e] : 0.0;
+  return zin ? ((~in_xy | ld) & 0xFu) : 0xFu;                  // outside the array: every element is 0
+}
+
 // fast: every element of the lane is strictly inside the array (hm == 0): plain stores; otherwise
 // the elements flagged in hm take the prefetched Dirichlet values hv (halo_fetch).
 template <int K, int S, int CS, bool ZERO = true>
@@ -375,6 +393,8 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
   // per item: intermediate stage S rows/columns of this lane strictly inside (publish fast path);
   // final elements of this lane to store (row / column validity, the z test is per plane)
   bool xy_in[K > 1 ? K - 1 : 1];
+  unsigned in_xy1 = 0u, hal_xy1 = 0u;   // stage 1 (K = 2): halo_fetch_z's per-item x/y masks and offset
+  int64_t base1 = 0;
   bool st_ok[2][2];
   for (int q0 = 0; q0 < nstages; q0 += 3) {
     auto one = [&](auto Ic) {
@@ -391,6 +411,21 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
         for (int S = 1; S < K; ++S) {
           const int gy = Y0 - (K - S) + 2 * w;
           xy_in[S - 1] = xs_in && gy >= 1 && gy + 1 < P1 - 1;
+        }
+        if constexpr (K == 2) {
+          in_xy1 = hal_xy1 = 0u;
+          const int gy0 = Y0 - 1 + 2 * w;
+          base1 = int64_t(gy0) * P2 + X0 + c0;
+#pragma unroll
+          for (int y = 0; y < 2; ++y)
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+              const int gy = gy0 + y, cx = X0 + c0 + e;
+              const bool in_ = gy >= 0 && gy < P1 && cx >= 0 && cx < P2;
+              const bool h_ = in_ && (gy < 1 || gy >= P1 - 1 || cx < 1 || cx >= P2 - 1);
+              in_xy1 |= (in_ ? 1u : 0u) << (2 * y + e);
+              hal_xy1 |= (h_ ? 1u : 0u) << (2 * y + e);
+            }
         }
 #pragma unroll
         for (int y = 0; y < 2; ++y) {
@@ -418,7 +453,11 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
         const bool fast1 = xy_in[0] && p - 1 >= 1 && p - 1 < P0 - 1;
         double hv[2][2];
         unsigned hm = 0;
+#if RDG3F_HALO_Z
+        if (K == 2 && !fast1) hm = halo_fetch_z(p - 1, P0, int64_t(P1) * P2, P2, in_xy1, hal_xy1, base1, in, hv);
+#else
         if (K == 2 && !fast1) hm = halo_fetch<K, 1>(w, lane, Y0, X0, p - 1, P0, P1, P2, in, hv);
+#endif
         double x[4][4];
         load_rows(st + (2 * w) * F_BW, F_BW, lane, x);
         planes2<SG, I, 0>(x, prm, acc[0]);

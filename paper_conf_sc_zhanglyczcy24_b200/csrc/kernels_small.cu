@@ -10,6 +10,11 @@
 //   halo is staged from `in` (no exchange at all); longer runs exchange the first / last kR own rows
 //   through a global buffer after each block, each CTA waiting only for its two neighbours' step
 //   counters (release / acquire at gpu scope).
+// * 2D tiles (default for short runs, small2d_tile_kernel): independent CTAs, each owning a TY x TX
+//   tile and staging it with a T R-deep halo on all four sides from `in`; all T steps run on a
+//   region that shrinks by R per step, with no exchange and no co-residency requirement.  Against
+//   row slabs with the same T R-deep halo (below) the redundant halo work falls from about 5.5x to
+//   2x for Heat-2D 256^2 x 10 (16 x 32 tiles), which is what bounded the slab form (issue-bound).
 // * thread-block cluster (fallback, small2d_star_kernel): the same slab / block scheme with the whole
 //   grid in the shared memory of one cluster of <= 16 CTAs and the exchange through the neighbours'
 //   DSMEM mailboxes (st.shared::cluster via cluster.map_shared_rank), one cluster barrier per block.
@@ -331,6 +336,121 @@ small2d_grid_kernel(const double* __restrict__ in, double* __restrict__ out, dou
   strace(60);
 }
 
+// 2D-tile variant.  CTA (bx, by) owns interior rows [y0, y0 + TY) and columns [x0, x0 + TX) (padded
+// coordinates, y0 = R + by TY, x0 = R + bx TX) and stages rows [y0 - H, y0 + TY + H) x columns
+// [x0 - H, x0 + TX + H), H = T R, into both shared buffers (zero outside the padded array; array-halo
+// cells hold the fixed Dirichlet values and are never written).  Step s computes the interior points
+// within (T - s) R of the own tile; after T steps the own tile is exact.  Per-point arithmetic: the
+// scalar loop of the other variants, i.e. the streaming kernel's SIG_STAR order (bitwise equal).
+#ifndef SMALL_TILE_STRIPS
+#define SMALL_TILE_STRIPS 1   // threads walk row strips with a register window (0: one point per iteration)
+#endif
+#ifndef SMALL_TILE_TY
+#define SMALL_TILE_TY 8   // 512 threads (Heat-2D 256^2 x 10: 11.7 us back to back vs 14.0 with 4, 13.4 with 2)
+#endif
+constexpr int TL_TX = 64, TL_TY = SMALL_TILE_TY;   // threads: 64 columns x TL_TY row groups
+template <int R>
+__global__ void __launch_bounds__(TL_TX * TL_TY)
+small2d_tile_kernel(const double* __restrict__ in, double* __restrict__ out, int N0, int N1, int TY, int TX, int T,
+                    const __grid_constant__ StarArms w) {
+  extern __shared__ __align__(16) double sm[];
+  const int P0 = N0 + 2 * R, P1 = N1 + 2 * R, H = T * R;
+  const int y0 = R + blockIdx.y * TY, x0 = R + blockIdx.x * TX;
+  const int ty1 = min(TY, N0 - (y0 - R)), tx1 = min(TX, N1 - (x0 - R));   // own extent (edge tiles are partial)
+  const int SY = ty1 + 2 * H, SX = tx1 + 2 * H;                           // staged region
+  const int gy0 = y0 - H, gx0 = x0 - H;                                   // padded origin of buffer cell (0, 0)
+  double* const buf0 = sm;
+  double* const buf1 = sm + size_t(SY) * SX;
+  const int tid = threadIdx.y * TL_TX + threadIdx.x;
+  constexpr int NT = TL_TX * TL_TY;
+  {  // staging: all of a thread's loads first (one HBM / L2 latency instead of one per element)
+    constexpr int U = 8;
+    for (int i0 = tid; i0 < SY * SX; i0 += NT * U) {
+      double v[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int i = i0 + u * NT, r = i / SX, c = i - r * SX;
+        const int gy = gy0 + r, gx = gx0 + c;
+        v[u] = (i < SY * SX && gy >= 0 && gy < P0 && gx >= 0 && gx < P1) ? __ldg(in + int64_t(gy) * P1 + gx) : 0.0;
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int i = i0 + u * NT;
+        if (i < SY * SX) { buf0[i] = v[u]; buf1[i] = v[u]; }
+      }
+    }
+  }
+  __syncthreads();
+  // buffer rows / columns of interior (updatable) points
+  const int ilo_r = max(0, R - gy0), ihi_r = min(SY, R + N0 - gy0);
+  const int ilo_c = max(0, R - gx0), ihi_c = min(SX, R + N1 - gx0);
+  int cur = 0;
+  for (int st = 1; st <= T; ++st) {
+    const double* src = cur ? buf1 : buf0;
+    double* dst = cur ? buf0 : buf1;
+    const int m = (T - st) * R;   // distance from the own tile still computed at this step
+    const int r0 = max(ilo_r, H - m), r1 = min(ihi_r, H + ty1 + m);
+    const int c0 = max(ilo_c, H - m), c1 = min(ihi_c, H + tx1 + m);
+#if SMALL_TILE_STRIPS
+    // each thread walks a strip of consecutive rows of one column with the 2R + 1 rows of the
+    // vertical arm in a register window (one new shared load per row for it)
+    const int nr = r1 - r0, per = (nr + TL_TY - 1) / TL_TY;
+    const int ra = r0 + (int)threadIdx.y * per, rb = min(r1, ra + per);
+    for (int c = c0 + (int)threadIdx.x; c < c1 && ra < rb; c += TL_TX) {
+      const double* cp = src + size_t(ra) * SX + c;
+      double* op = dst + size_t(ra) * SX + c;
+      double win[2 * R + 1];
+#pragma unroll
+      for (int a = 0; a < 2 * R; ++a) win[a] = cp[(a - R) * SX];
+#pragma unroll 2
+      for (int r = ra; r < rb; ++r, cp += SX, op += SX) {
+        win[2 * R] = cp[R * SX];
+        double th = 0.0;
+#pragma unroll
+        for (int b = -R; b <= R; ++b) th = fma(w.h[R + b], b == 0 ? win[R] : cp[b], th);
+        double acc = 0.0;
+#pragma unroll
+        for (int a = -R; a <= R; ++a) {
+          if (a == 0) acc += th;
+          acc = fma(w.v[R + a], win[R + a], acc);
+        }
+        *op = acc;
+#pragma unroll
+        for (int a = 0; a < 2 * R; ++a) win[a] = win[a + 1];
+      }
+    }
+#else
+    for (int r = r0 + (int)threadIdx.y; r < r1; r += TL_TY) {
+      for (int c = c0 + (int)threadIdx.x; c < c1; c += TL_TX) {
+        const double* cx = src + size_t(r) * SX + c;
+        double th = 0.0;
+#pragma unroll
+        for (int b = -R; b <= R; ++b) th = fma(w.h[R + b], cx[b], th);
+        double acc = 0.0;
+#pragma unroll
+        for (int a = -R; a <= R; ++a) {
+          if (a == 0) acc += th;
+          acc = fma(w.v[R + a], cx[a * SX], acc);
+        }
+        dst[size_t(r) * SX + c] = acc;
+      }
+    }
+#endif
+    cur ^= 1;
+    __syncthreads();
+  }
+  // write back the own tile, extended by R into the array halo where the tile touches the array
+  // edge (those cells hold the input's Dirichlet values in both buffers)
+  const double* res = cur ? buf1 : buf0;
+  const int wr0 = H - (blockIdx.y == 0 ? R : 0), wr1 = H + ty1 + (y0 - R + ty1 == N0 ? R : 0);
+  const int wc0 = H - (blockIdx.x == 0 ? R : 0), wc1 = H + tx1 + (x0 - R + tx1 == N1 ? R : 0);
+  const int nwc = wc1 - wc0;
+  for (int i = tid; i < (wr1 - wr0) * nwc; i += NT) {
+    const int r = wr0 + i / nwc, c = wc0 + i % nwc;
+    out[int64_t(gy0 + r) * P1 + gx0 + c] = res[size_t(r) * SX + c];
+  }
+}
+
 // The two-arm star signature of the streaming engine (kernels_rdg.cu signature(), SIG_STAR).
 bool star_arms(const Plan& p, StarArms& w) {
   const int R = p.R, n = 2 * R + 1;
@@ -495,7 +615,7 @@ cudaError_t grid_launch(const Plan& p, const double* in, double* out, double* xc
 
 cudaError_t launch_grid_variant(Plan& p, const double* in, double* out, int64_t T, cudaStream_t s,
                                 const StarArms& w) {
-  if (p.small_cluster_only) return cudaErrorNotSupported;
+  if (p.small_mode == 1) return cudaErrorNotSupported;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
@@ -545,6 +665,72 @@ cudaError_t launch_grid_variant(Plan& p, const double* in, double* out, int64_t 
   }
   return cudaErrorNotSupported;
 }
+
+// Tile shape for the 2D-tile variant: the (TY, TX) in {8, 16, 32, 64}^2 with the least work per SM
+// (CTA rounds over the SMs x the CTA's trapezoid of points over the T steps); 0 if the halo'd tile
+// does not fit the shared memory.
+bool tile_shape(const Plan& p, int64_t T, int sms, int& TY, int& TX, size_t& smem) {
+  const int64_t H = T * p.R;
+  double best = 0.0;
+  TY = TX = 0;
+  for (int ty : {8, 16, 32, 64})
+    for (int tx : {8, 16, 32, 64}) {
+      const int ey = (int)std::min<int64_t>(ty, p.N[0]), ex = (int)std::min<int64_t>(tx, p.N[1]);
+      const size_t sb = 2 * size_t(ey + 2 * H) * size_t(ex + 2 * H) * sizeof(double);
+      if (sb > kMaxSmem) continue;
+      const int64_t G = ((p.N[0] + ty - 1) / ty) * ((p.N[1] + tx - 1) / tx);
+      double work = 0.0;
+      for (int64_t s = 1; s <= T; ++s) {
+        const int64_t m = (T - s) * p.R;
+        work += double(std::min<int64_t>(ey + 2 * m, p.N[0])) * double(std::min<int64_t>(ex + 2 * m, p.N[1]));
+      }
+      const double cost = double((G + sms - 1) / sms) * work;   // CTAs on the busiest SM x points per CTA
+      if (TY == 0 || cost < best) { best = cost; TY = ty; TX = tx; smem = sb; }
+    }
+  return TY > 0;
+}
+
+cudaError_t launch_tile_variant(const Plan& p, const double* in, double* out, int64_t T, cudaStream_t s,
+                                const StarArms& w) {
+  if (p.small_mode != 0 || T * p.R > SMALL_ONE_BLOCK_MAX_HALO) return cudaErrorNotSupported;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  int TY = 0, TX = 0;
+  size_t smem = 0;
+  if (!tile_shape(p, T, sms, TY, TX, smem)) return cudaErrorNotSupported;
+  const void* k = nullptr;
+  switch (p.R) {
+    case 1: k = (const void*)small2d_tile_kernel<1>; break;
+    case 2: k = (const void*)small2d_tile_kernel<2>; break;
+    case 3: k = (const void*)small2d_tile_kernel<3>; break;
+    case 4: k = (const void*)small2d_tile_kernel<4>; break;
+    default: return cudaErrorNotSupported;
+  }
+  {  // the dynamic shared memory attribute, once per (kernel, device)
+    static std::mutex mu;
+    static std::map<std::pair<const void*, int>, bool> done;
+    std::lock_guard<std::mutex> lock(mu);
+    bool& d = done[{k, dev}];
+    if (!d) {
+      if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem) != cudaSuccess) {
+        cudaGetLastError();
+        return cudaErrorNotSupported;
+      }
+      d = true;
+    }
+  }
+  const dim3 grid((unsigned)((p.N[1] + TX - 1) / TX), (unsigned)((p.N[0] + TY - 1) / TY), 1);
+  const dim3 block(TL_TX, TL_TY, 1);
+  const int N0 = (int)p.N[0], N1 = (int)p.N[1], Ti = (int)T;
+  switch (p.R) {
+    case 1: small2d_tile_kernel<1><<<grid, block, smem, s>>>(in, out, N0, N1, TY, TX, Ti, w); break;
+    case 2: small2d_tile_kernel<2><<<grid, block, smem, s>>>(in, out, N0, N1, TY, TX, Ti, w); break;
+    case 3: small2d_tile_kernel<3><<<grid, block, smem, s>>>(in, out, N0, N1, TY, TX, Ti, w); break;
+    case 4: small2d_tile_kernel<4><<<grid, block, smem, s>>>(in, out, N0, N1, TY, TX, Ti, w); break;
+  }
+  return cudaGetLastError();
+}
 }  // namespace
 
 #ifdef SMALL_TRACE
@@ -555,6 +741,8 @@ cudaError_t launch_small2d(Plan& p, const double* in, double* out, int64_t T, cu
   if (!star_arms(p, w) || T < 1) return cudaErrorInvalidValue;
   if (T > (int64_t(1) << 30)) return cudaErrorNotSupported;   // (int step counts) the per-step path runs it
   {
+    const cudaError_t et = launch_tile_variant(p, in, out, T, s, w);
+    if (et != cudaErrorNotSupported) return et;
     const cudaError_t eg = launch_grid_variant(p, in, out, T, s, w);
     if (eg != cudaErrorNotSupported) return eg;
   }

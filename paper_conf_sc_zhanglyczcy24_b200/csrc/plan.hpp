@@ -42,7 +42,8 @@ struct Plan {
   int force_no_tma = 0;   // LORA_NO_TMA=1: use the LDGSTS staging path (tests both loaders)
   int tc_no_bvs = 0;
   int no_small = 0;       // LORA_NO_SMALL=1: no single-launch path for small 2D grids (tests)
-  int small_cluster_only = 0;   // LORA_SMALL_MODE=cluster: the cluster variant of that path (tests)
+  int small_mode = 0;     // LORA_SMALL_MODE: 0 2D tiles for short runs, else the grid variant; 1 ("cluster")
+                          // the DSMEM cluster variant; 2 ("grid") the cooperative-grid variant (tests)
   int small_rp = 2;       // LORA_SMALL_RP: rows per CTA of its cooperative-grid variant (experiments)      // LORA_TC_NO_BVS=1: the Fig. 9 ablation (shuffle-based stage 2) in the TC engine
   int n_planes_point = 0;
   // CUDA-core engine, 2D, radius >= 3, W reflection-symmetric in both axes with a nonzero centre

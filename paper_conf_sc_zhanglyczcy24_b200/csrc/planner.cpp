@@ -423,8 +423,8 @@ int plan_build(Plan& p, const double* weights, int ndim, int radius, const int64
     p.tc_no_bvs = (b && b[0] == '1') ? 1 : 0;
     const char* sm = std::getenv("LORA_NO_SMALL");
     p.no_small = (sm && sm[0] == '1') ? 1 : 0;
-    const char* smode = std::getenv("LORA_SMALL_MODE");   // tests: "cluster" = the DSMEM cluster variant
-    p.small_cluster_only = (smode && std::strcmp(smode, "cluster") == 0) ? 1 : 0;
+    const char* smode = std::getenv("LORA_SMALL_MODE");   // tests: "cluster" / "grid" variants
+    p.small_mode = !smode ? 0 : (std::strcmp(smode, "cluster") == 0 ? 1 : (std::strcmp(smode, "grid") == 0 ? 2 : 0));
     const char* srp = std::getenv("LORA_SMALL_RP");       // experiments: rows per CTA of the grid variant
     p.small_rp = srp ? std::max(1, std::atoi(srp)) : 2;   // Heat-2D 256^2 x 10: 2 -> 14.8 us, 4 -> 15.8, 8 -> 18.1
   }

@@ -433,14 +433,17 @@ def test_zero_centre_tap_fallback_3d():
 @pytest.mark.parametrize("kind,h", [("heat2d", 1), ("star", 1), ("star", 2), ("star", 3), ("star", 4)])
 @pytest.mark.parametrize("shape", [(256, 256), (64, 100), (48, 33), (32, 258)])
 def test_small_cluster_path_bitwise(kind, h, shape, monkeypatch):
-    """Small 2D star grids run all T steps in one thread-block-cluster launch (kernels_small.cu,
-    DSMEM halo exchange): bitwise equal to the streaming engine's per-step launches
-    (LORA_NO_SMALL=1) and within 1e-12 of the oracle, for T on both sides of the fusion depth."""
+    """Small 2D star grids run all T steps in one launch (kernels_small.cu): the 2D-tile variant
+    (default for T R <= 16), the cooperative-grid variant and the thread-block-cluster (DSMEM)
+    variant are each bitwise equal to the streaming engine's per-step launches (LORA_NO_SMALL=1)
+    and within 1e-12 of the oracle, for T on both sides of the fusion depth."""
     W = synth.preset("heat2d") if kind == "heat2d" else synth.star_weights(2, h, 11 + h)
     g = synth.grid(tuple(n + 2 * h for n in shape), 20240101 + h)
-    for T in (1, 2, 5, 10):
-        out, info = run_gpu(W, g, T)                      # cooperative-grid variant (default)
+    for T in (1, 2, 5, 10, 17):
+        out, info = run_gpu(W, g, T)                      # default: tiles (T R <= 16), else the grid variant
         assert info["single_launch"] == 1, info
+        monkeypatch.setenv("LORA_SMALL_MODE", "grid")     # the cooperative-grid variant
+        out_gr, _ = run_gpu(W, g, T)
         monkeypatch.setenv("LORA_SMALL_MODE", "cluster")  # the thread-block-cluster (DSMEM) variant
         out_cl, _ = run_gpu(W, g, T)
         monkeypatch.delenv("LORA_SMALL_MODE")
@@ -450,4 +453,5 @@ def test_small_cluster_path_bitwise(kind, h, shape, monkeypatch):
         assert info2["single_launch"] == 0
         assert np.array_equal(out, ref_stream), (T, float(np.max(np.abs(out - ref_stream))))
         assert np.array_equal(out_cl, ref_stream), (T, float(np.max(np.abs(out_cl - ref_stream))))
+        assert np.array_equal(out_gr, ref_stream), (T, float(np.max(np.abs(out_gr - ref_stream))))
         assert rel_err(out, oracle.run(W, g, T)) <= 1e-12
