@@ -3,6 +3,8 @@
 #pragma once
 #include <cuda_runtime.h>
 
+#include <cstdlib>
+
 #include "plan.hpp"
 
 namespace lora {
@@ -18,6 +20,26 @@ inline bool pma1_unit_centre(const double* u, const double* v, double* uo, doubl
   for (int i = 0; i < 3; ++i) { uo[i] = u[i] * c; vo[i] = v[i] / c; }
   vo[1] = 1.0;
   return true;
+}
+
+// Radius-1 3D planes with the full symmetry of a radially symmetric stencil:
+// plane a0 of W is [a b a; b c b; a b a].  When planes 0 and 1 both have it and plane 2 mirrors
+// plane 0 (Box-3D27P), the 3D CUDA-core kernels evaluate the two plane operators JOINTLY on the
+// symmetric class sums they share (mode PM_SYM3, reading Q18): with px = x_l + x_r per
+// row, s1 = x_u + x_d, pc = px_u + px_d (corners), e = px + s1 (edges),
+//   d_k = a_k pc + (b_k e + c_k x)        (k = plane 0, 1)
+// 11 FP64 ops per point for both operators instead of 16 for the two PMA chains.  Both kernels
+// (unfused and fused) use the same formula in the same order, so they stay bitwise equal.
+// LORA_NO_SYM3=1 keeps the PMA form (A/B).  Returns false unless the plane has the symmetry.
+inline bool sym3_plane(const double* W, int a0, double& c, double& b, double& a) {
+  const double* q = W + 9 * a0;
+  a = q[0]; b = q[1]; c = q[4];
+  return q[2] == a && q[6] == a && q[8] == a && q[3] == b && q[5] == b && q[7] == b;
+}
+
+inline bool sym3_enabled() {
+  const char* e = std::getenv("LORA_NO_SYM3");
+  return !(e && e[0] == '1');
 }
 
 // Device-initiated halo exchange (csrc/dist_p2p.cu): the slab's boundary work items

@@ -32,7 +32,7 @@ template <int R> constexpr int BY = (R == 1 ? 4 : 2);
 constexpr int R3_ZC = 64;
 constexpr int R3_MAXK = 5;   // rank-1 terms per plane (<= 2R+1 for R <= 2)
 
-enum { PM_NONE = 0, PM_POINT = 1, PM_CHAINS = 2, PM_STAR = 3, PM_PMA1 = 4, PM_DIRECT = 5 };
+enum { PM_NONE = 0, PM_POINT = 1, PM_CHAINS = 2, PM_STAR = 3, PM_PMA1 = 4, PM_DIRECT = 5, PM_SYM3 = 6 };
 
 struct R3Params {
   int mode[5];               // per plane a0
@@ -41,6 +41,7 @@ struct R3Params {
   double w[5];               // PM_POINT weight (centre) / PM_PMA1 scalar C_{h+1}
   double u[5][R3_MAXK][5];   // plane, term, tap (centred, length 2R+1)
   double v[5][R3_MAXK][5];
+  double sym[2][3];          // PM_SYM3 (planes 0 and 1 jointly, R = 1): centre c, edge b, corner a
 };
 
 template <int R>
@@ -172,10 +173,42 @@ __device__ __forceinline__ void apply_plane(const double (&x)[BY<R> + 2 * R][2 *
   }
 }
 
+// PM_SYM3 (R = 1, planes 0 and 1 jointly, plane 2 = mirror of plane 0; kernels.hpp sym3_plane):
+// d0 (plane 0) goes to output planes z = p and p - 2, d1 (plane 1) to z = p - 1, in the order of the
+// per-plane path (plane 0 then its mirror, then plane 1).
+template <int I>
+__device__ __forceinline__ void apply_sym3(const double (&x)[BY<1> + 2][4], double (&acc)[3][BY<1>][2],
+                                           const R3Params& P) {
+  double px[BY<1> + 2][2];
+#pragma unroll
+  for (int r = 0; r < BY<1> + 2; ++r) {
+    px[r][0] = x[r][0] + x[r][2];
+    px[r][1] = x[r][1] + x[r][3];
+  }
+  constexpr int s0 = pm(I, 3), s2 = pm(I - 2, 3), s1 = pm(I - 1, 3);
+#pragma unroll
+  for (int y = 0; y < BY<1>; ++y)
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {
+      const double xc = x[y + 1][1 + e];
+      const double sv = x[y][1 + e] + x[y + 2][1 + e];
+      const double pc = px[y][e] + px[y + 2][e];
+      const double ed = px[y + 1][e] + sv;
+      const double d0 = fma(P.sym[0][2], pc, fma(P.sym[0][1], ed, P.sym[0][0] * xc));
+      const double d1 = fma(P.sym[1][2], pc, fma(P.sym[1][1], ed, P.sym[1][0] * xc));
+      acc[s0][y][e] += d0;
+      acc[s2][y][e] += d0;
+      acc[s1][y][e] += d1;
+    }
+}
+
 template <int R, class SG, int A0, int I>
 __device__ __forceinline__ void apply_all(const double (&x)[BY<R> + 2 * R][2 * R + 2],
                                           double (&acc)[2 * R + 1][BY<R>][2], const R3Params& P) {
-  if constexpr (A0 < 2 * R + 1) {
+  if constexpr (R == 1 && SG::m0 == PM_SYM3) {
+    static_assert(SG::m1 == PM_SYM3 && SG::mir == 1, "PM_SYM3 signature");
+    if constexpr (A0 == 0) apply_sym3<I>(x, acc, P);
+  } else if constexpr (A0 < 2 * R + 1) {
     // specialised modes exist for R = 1 only (plane 0, plane 1, plane 2 == mirror of plane 0)
     constexpr int MODE = R != 1 ? -1 : (A0 == 0 ? SG::m0 : (A0 == 1 ? SG::m1 : (SG::mir == 1 ? SG::m0 : -1)));
     constexpr int MIR = R != 1 ? -1 : SG::mir;
@@ -426,6 +459,14 @@ bool make_params3(const Plan& p, R3Params& prm, bool direct = false) {
       if (p.W[size_t(a0) * n * n + e] != p.W[size_t(n - 1 - a0) * n * n + e]) { same = false; break; }
     prm.mirror[a0] = same ? 1 : 0;
   }
+  if (R == 1 && prm.mode[0] == PM_PMA1 && prm.mode[1] == PM_PMA1 && prm.mirror[0] && sym3_enabled()) {
+    double c0, b0, a0_, c1, b1, a1;
+    if (sym3_plane(p.W.data(), 0, c0, b0, a0_) && sym3_plane(p.W.data(), 1, c1, b1, a1)) {
+      prm.mode[0] = prm.mode[1] = PM_SYM3;
+      prm.sym[0][0] = c0; prm.sym[0][1] = b0; prm.sym[0][2] = a0_;
+      prm.sym[1][0] = c1; prm.sym[1][1] = b1; prm.sym[1][2] = a1;
+    }
+  }
   return true;
 }
 
@@ -487,6 +528,9 @@ cudaError_t rdg3d_r(const Plan& p, const double* src, double* dst, cudaStream_t 
   const bool tma = !p.force_no_tma && encode_tmap(&map, src, 3, padded, box);
   if (!tma) std::memset(&map, 0, sizeof(map));
   if constexpr (R == 1) {  // Box-3D27P-like and Heat-3D-like plane signatures
+    if (prm.mode[0] == PM_SYM3)
+      return tma ? rdg3d_launch<R, Sig3<PM_SYM3, PM_SYM3, 1>, true>(p, src, dst, s, map, prm, d)
+                 : rdg3d_launch<R, Sig3<PM_SYM3, PM_SYM3, 1>, false>(p, src, dst, s, map, prm, d);
     if (prm.mode[0] == PM_PMA1 && prm.mode[1] == PM_PMA1 && prm.mirror[0])
       return tma ? rdg3d_launch<R, Sig3<PM_PMA1, PM_PMA1, 1>, true>(p, src, dst, s, map, prm, d)
                  : rdg3d_launch<R, Sig3<PM_PMA1, PM_PMA1, 1>, false>(p, src, dst, s, map, prm, d);

@@ -50,13 +50,14 @@ constexpr int F_BW = 66;             // staged columns (64 + 2R)
 constexpr int F_S1W = 72;            // step-1 plane buffer row pitch (doubles): data at [1, 65)
 constexpr int F_ZC = 64;
 
-enum { PM_NONE = 0, PM_POINT = 1, PM_CHAINS = 2, PM_STAR = 3, PM_PMA1 = 4 };
+enum { PM_NONE = 0, PM_POINT = 1, PM_CHAINS = 2, PM_STAR = 3, PM_PMA1 = 4, PM_SYM3 = 6 };   // (values as in kernels_rdg3d.cu)
 constexpr int F_MAXK = 3;
 
 struct FParams {
   int mode[3], K[3], mirror[3];
   double w[3];
   double u[3][F_MAXK][3], v[3][F_MAXK][3];
+  double sym[2][3];   // PM_SYM3 (planes 0 and 1 jointly): centre c, edge b, corner a (kernels.hpp sym3_plane)
 };
 
 __host__ __device__ constexpr int pm3(int a) { return ((a % 3) + 3) % 3; }
@@ -144,9 +145,36 @@ struct Sig3 {
 };
 
 // All plane operators of one input plane (ring position I) into a z-ring of 3 planes x 2 rows.
+// PM_SYM3: both operators jointly on the shared class sums, in the order of kernels_rdg3d.cu's
+// apply_sym3 (plane 0 assigned to its slot, added to the mirror slot; plane 1 added).
 template <class SG, int I, int A0>
 __device__ __forceinline__ void planes2(const double (&x)[4][4], const FParams& P, double (&acc)[3][2][2]) {
-  if constexpr (A0 < 3) {
+  if constexpr (SG::m0 == PM_SYM3) {
+    static_assert(SG::m1 == PM_SYM3 && SG::mir == 1 && SG::assign0, "PM_SYM3 signature");
+    if constexpr (A0 == 0) {
+      double px[4][2];
+#pragma unroll
+      for (int r = 0; r < 4; ++r) {
+        px[r][0] = x[r][0] + x[r][2];
+        px[r][1] = x[r][1] + x[r][3];
+      }
+      constexpr int s0 = pm3(I), s2 = pm3(I - 2), s1 = pm3(I - 1);
+#pragma unroll
+      for (int y = 0; y < 2; ++y)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const double xc = x[y + 1][1 + e];
+          const double sv = x[y][1 + e] + x[y + 2][1 + e];
+          const double pc = px[y][e] + px[y + 2][e];
+          const double ed = px[y + 1][e] + sv;
+          const double d0 = fma(P.sym[0][2], pc, fma(P.sym[0][1], ed, P.sym[0][0] * xc));
+          const double d1 = fma(P.sym[1][2], pc, fma(P.sym[1][1], ed, P.sym[1][0] * xc));
+          acc[s0][y][e] = d0;
+          acc[s2][y][e] += d0;
+          acc[s1][y][e] += d1;
+        }
+    }
+  } else if constexpr (A0 < 3) {
     const bool mirror = SG::mir >= 0 ? SG::mir == 1 : P.mirror[0] != 0;
     constexpr int MODE = A0 == 0 ? SG::m0 : (A0 == 1 ? SG::m1 : (SG::mir == 1 ? SG::m0 : -1));
     if (!(A0 == 2 && mirror)) {
@@ -589,6 +617,14 @@ bool make_fparams(const Plan& p, FParams& prm) {
   for (int e = 0; e < n * n; ++e)
     if (p.W[e] != p.W[size_t(2) * n * n + e]) { same = false; break; }
   prm.mirror[0] = same ? 1 : 0;
+  if (prm.mode[0] == PM_PMA1 && prm.mode[1] == PM_PMA1 && prm.mirror[0] && sym3_enabled()) {
+    double c0, b0, a0, c1, b1, a1;
+    if (sym3_plane(p.W.data(), 0, c0, b0, a0) && sym3_plane(p.W.data(), 1, c1, b1, a1)) {
+      prm.mode[0] = prm.mode[1] = PM_SYM3;
+      prm.sym[0][0] = c0; prm.sym[0][1] = b0; prm.sym[0][2] = a0;
+      prm.sym[1][0] = c1; prm.sym[1][1] = b1; prm.sym[1][2] = a1;
+    }
+  }
   return true;
 }
 
@@ -647,7 +683,11 @@ cudaError_t launch_fk(const Plan& p, const double* src, double* dst, cudaStream_
   const int box[3] = {1, F_IN, F_BW};
   const bool tma = !p.force_no_tma && encode_tmap(&map, src, 3, padded, box);
   if (!tma) std::memset(&map, 0, sizeof(map));
-  // specialisations: Box-3D27P-like (PMA planes, z-mirrored) and Heat-3D-like (point / star, mirrored)
+  // specialisations: Box-3D27P-like (symmetric class sums or PMA planes, z-mirrored) and Heat-3D-like
+  // (point / star, mirrored)
+  if (prm.mode[0] == PM_SYM3)
+    return tma ? launch_f<Sig3<PM_SYM3, PM_SYM3, 1>, K, true, P2P>(p, src, dst, s, map, prm, d)
+               : launch_f<Sig3<PM_SYM3, PM_SYM3, 1>, K, false, P2P>(p, src, dst, s, map, prm, d);
   if (prm.mode[0] == PM_PMA1 && prm.mode[1] == PM_PMA1 && prm.mirror[0])
     return tma ? launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, K, true, P2P>(p, src, dst, s, map, prm, d)
                : launch_f<Sig3<PM_PMA1, PM_PMA1, 1>, K, false, P2P>(p, src, dst, s, map, prm, d);

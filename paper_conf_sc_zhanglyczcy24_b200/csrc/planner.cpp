@@ -218,6 +218,22 @@ double cuda_fma_per_point(const Plan& p) {
     }
     return plane_cost(0);
   }
+  if (p.ndim == 3 && p.R == 1 && sym3_enabled()) {
+    // PM_SYM3 (kernels.hpp sym3_plane; chosen by the 3D kernels when planes 0 and 1 are PMA planes
+    // with the full [a b a; b c b; a b a] symmetry and plane 2 mirrors plane 0): px 1.5 (6 rows per 4
+    // outputs), 3 shared class sums, 3 per plane operator, 3 accumulating adds
+    auto pma1 = [&](int q) {
+      int cnt = 0, chain = 0, point = 0;
+      for (const Term& t : p.terms)
+        if (t.plane == q) { ++cnt; chain += t.kind == kChain && t.r == 1; point += t.kind == kPoint; }
+      return cnt == 2 && chain == 1 && point == 1;
+    };
+    bool mir = true;
+    for (int e = 0; e < 9; ++e) mir = mir && p.W[size_t(18) + e] == p.W[size_t(e)];
+    double c, b, a;
+    if (mir && pma1(0) && pma1(1) && sym3_plane(p.W.data(), 0, c, b, a) && sym3_plane(p.W.data(), 1, c, b, a))
+      return 1.5 + 3.0 + 2 * 3.0 + 3.0;
+  }
   double f = 0;
   for (int q = 0; q < n; ++q) {
     bool mirrored = false;
