@@ -37,6 +37,9 @@ namespace {
 #endif                // CTA barrier at the end of the iteration, the stages of an iteration independent).
                       // Measured slower (r02m, same box): Box-3D27P k = 2 393 -> 379 GS/s, Heat-3D 449 -> 416
 constexpr int F_LAG = RDG3F_LAG;
+#ifndef RDG3F_DECOUPLE
+#define RDG3F_DECOUPLE 0   // 1 (K = 2, TMA): mbarrier hand-offs between the stages instead of one CTA barrier
+#endif                     // per plane.  Measured slower (r02ze, same box): Box-3D27P 447 -> 428, Heat-3D 483 -> 448
 #ifndef RDG3F_HALO_Z
 #define RDG3F_HALO_Z 1   // stage-1 Dirichlet fetch with the x/y masks precomputed per item (halo_fetch_z)
 #endif
@@ -330,13 +333,29 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
   uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw);
   unsigned char* ring = smem_raw + 128;
   double* sbuf = reinterpret_cast<double*>(smem_raw + 128 + F_NS * STAGE);  // [K-1][2][F_S1][F_S1W]
-  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  // the warp index through a shuffle: ptxas then knows it is warp-uniform (warp-0-only branches stay
+  // uniform, and the weights keep their uniform registers)
+  const int tid = threadIdx.x, lane = tid & 31, w = __shfl_sync(0xffffffffu, tid >> 5, 0);
   const int P0 = (int)(N0 + 2), P1 = (int)(N1 + 2), P2 = (int)(N2 + 2);
   for (int i = tid; i < 2 * (K - 1) * S1B; i += blockDim.x) sbuf[i] = 0.0;   // margins stay zero
   const int my_items = blockIdx.x < nitems ? (nitems - 1 - blockIdx.x) / gridDim.x + 1 : 0;
   const int nstages = my_items * SI;
+  // DEC (K = 2, TMA): the stages hand planes over through mbarriers instead of a CTA barrier per plane
+  // (ncu: 16 % of the warps' stall samples sat at that barrier; warp 7 has no stage-2 rows and the
+  // stage-2 warps waited for each other): slot_free[s] — every warp has read input slot s (warp 0 then
+  // refills it); pub[par] — every warp has published its stage-1 rows of the plane buffer of parity
+  // par; cons[par] — the stage-2 warps have read that buffer (stage 1 may overwrite it two planes later)
+  constexpr bool DEC = RDG3F_DECOUPLE && K == 2 && TMA && !F_LAG;
+  static_assert(!DEC || 3 * F_NS + 4 <= 16, "mbarrier area");
+  uint64_t* slot_free = bar + F_NS;
+  uint64_t* pub = bar + 2 * F_NS;
+  uint64_t* cons = pub + 2;
   if (TMA && tid == 0) {
     for (int s = 0; s < F_NS; ++s) mbar_init(&bar[s], 1);
+    if constexpr (DEC) {
+      for (int s = 0; s < F_NS; ++s) mbar_init(&slot_free[s], F_WARPS);
+      for (int b = 0; b < 2; ++b) { mbar_init(&pub[b], F_WARPS); mbar_init(&cons[b], F_S1 / 2 - 1); }
+    }
     fence_barrier_init();
   }
   __syncthreads();
@@ -488,14 +507,30 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
 #endif
         double x[4][4];
         load_rows(st + (2 * w) * F_BW, F_BW, lane, x);
+        if constexpr (DEC) {   // this warp is done with the input slot
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&slot_free[slot]);
+        }
         planes2<SG, I, 0>(x, prm, acc[0]);
+        if constexpr (DEC) {   // the stage-2 warps have read this parity's buffer two planes ago
+          if (q >= 2) mbar_wait(&cons[par], ((q >> 1) + 1) & 1);
+        }
         if constexpr (K == 2)
           publish<K, 1, (I + 1) % 3, !SG::assign0>(acc, sbuf + (0 * 2 + par) * S1B, w, lane, hm, hv);
         else
           publish_ip<K, 1, (I + 1) % 3, !SG::assign0>(acc, sbuf + (0 * 2 + par) * S1B, w, lane, Y0, X0, p - 1, P0, P1, P2, in,
                                                       fast1);
       }
-      if constexpr (!F_LAG) {
+      if constexpr (DEC) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&pub[par]);   // my stage-1 rows of this plane are in the buffer
+        if (w == 0 && q + F_NS - 1 < nstages) {  // refill the slot of plane q - 1 once every warp read it
+          const int ps = (slot + F_NS - 1) % F_NS;
+          if (q >= 1) mbar_wait(&slot_free[ps], ((q - 1) / F_NS) & 1);
+          issue_next(ps);
+        }
+        mbar_wait(&pub[par], (q >> 1) & 1);      // every warp's stage-1 rows of this plane
+      } else if constexpr (!F_LAG) {
         __syncthreads();  // stage-1 plane visible; every warp is done with the input slot
         if (q + F_NS - 1 < nstages) issue_next((slot + F_NS - 1) % F_NS);
       }
@@ -511,7 +546,13 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
           const double* Sb = sbuf + ((S - 2) * 2 + rpar) * S1B;
           double x[4][4];
           load_rows(Sb + (2 * w) * F_S1W, F_S1W, lane, x);
+          if constexpr (DEC) {   // done reading the plane buffer
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&cons[par]);
+          }
           planes2<SG, IS, 0>(x, prm, acc[S - 1]);
+        } else if constexpr (DEC) {
+          if (w < F_S1 / 2 - (S - 1) && lane == 0) mbar_arrive(&cons[par]);   // a stage-2 warp without work
         }
         if constexpr (S < K) {
           // (S < K only for K = 3: in-place Dirichlet loads)
