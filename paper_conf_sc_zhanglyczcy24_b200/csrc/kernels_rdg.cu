@@ -42,6 +42,9 @@ constexpr int kRowUnroll = RDG_LOOP_UNROLL;   // (#pragma arguments are not macr
 #define RDG_WARPS_PER_CTA 4   // (Box-2D49P k=2: 2 warps 351, 4 warps 350, 8 warps 270 GS/s; Box-2D9P k=3: 654 / 692)
 #endif
 constexpr int RDG_WARPS = RDG_WARPS_PER_CTA;   // warps per CTA (independent streams)
+#ifndef RDG_PF_HALVES
+#define RDG_PF_HALVES 2   // 64-column halves of the next row prefetched (RDG_PF, loop form)
+#endif
 #ifndef RDG_NS_STAGES
 #define RDG_NS_STAGES 3
 #endif
@@ -388,7 +391,7 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
   if constexpr (LOOP) {
 #pragma unroll
     for (int h = 0; h < NH; ++h) {
-      if constexpr (PRE) {
+      if (PRE && h < RDG_PF_HALVES) {   // (RDG_PF_HALVES: only the first halves are prefetched)
         row_shift<R, SIG>(xq[h], acc[S - 1][h], P);
       } else {
         double x[2 * R + 2];
@@ -569,7 +572,7 @@ __device__ __forceinline__ void fused_rows_loop(const double* __restrict__ st, i
   constexpr bool PF = RDG_PF > 0 && R >= RDG_PF;
   if constexpr (PF) {
 #pragma unroll
-    for (int h = 0; h < NH; ++h) load_x<R>(st + 64 * h, p, xq[h]);
+    for (int h = 0; h < NH && h < RDG_PF_HALVES; ++h) load_x<R>(st + 64 * h, p, xq[h]);
   }
   double* orow = out + sc.ooff;   // output row of the final stage for I = 0 (only dereferenced when stored)
 #pragma unroll kRowUnroll
@@ -580,7 +583,7 @@ __device__ __forceinline__ void fused_rows_loop(const double* __restrict__ st, i
                                                               orow);
       if (I + 1 < SROWS) {
 #pragma unroll
-        for (int h = 0; h < NH; ++h) load_x<R>(st + (I + 1) * BW + 64 * h, p, xq[h]);
+        for (int h = 0; h < NH && h < RDG_PF_HALVES; ++h) load_x<R>(st + (I + 1) * BW + 64 * h, p, xq[h]);
       }
       fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 2, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
                                                                orow);
@@ -603,6 +606,9 @@ __device__ __forceinline__ void fused_rows_loop(const double* __restrict__ st, i
 // the fused kernels do not (see rdg_full).  0: never, 1: always (experiments).
 #define RDG_FULL 2
 #endif
+#ifndef RDG_NH_MINR
+#define RDG_NH_MINR 1   // smallest radius with NH = 2 in the fused kernels (r02zf: Box-2D9P k = 3 730 -> 747 GS/s with 1)
+#endif
 #ifndef RDG_NH_FUSED
 #define RDG_NH_FUSED 2   // 64-column halves per warp in the fused (K >= 2) kernels
 #endif
@@ -620,9 +626,9 @@ constexpr int rdg_cta_smem(int nh) {   // must match rdg_launch
 }
 // NH = 2 where two CTAs of it still fit the 228 KB of shared memory per SM (R = 3, 4)
 template <int R, int SIG, int K>
-// (radius 1 stays at NH = 1: Box-2D9P k = 3 641 vs 630 GS/s; radius 3 k = 2 gains 7 %)
+// (radius 1: Box-2D9P k = 3 641 vs 630 GS/s with vector-register weights, 747 vs 730 with uniform ones)
 constexpr int rdg_nh() {
-  return (K >= 2 && R >= 2 && RDG_NH_FUSED == 2 && 2 * (rdg_cta_smem<R, K>(2) + 1024) <= 228 * 1024) ? 2 : 1;
+  return (K >= 2 && R >= RDG_NH_MINR && RDG_NH_FUSED == 2 && 2 * (rdg_cta_smem<R, K>(2) + 1024) <= 228 * 1024) ? 2 : 1;
 }
 
 template <int R, int SIG, int K>
