@@ -229,6 +229,20 @@ def test_cuda_core_rank1_forms(L, monkeypatch):
     assert L.Stencil(W, (64, 64), engine="rdg_cuda").info()["fma_per_point_issued"] == 25
 
 
+def test_3d_joint_symmetric_planes(L, monkeypatch):
+    """3D CUDA-core engine (reading Q18): a radius-1 W whose planes 0 and 1 are
+    [a b a; b c b; a b a] with plane 2 = plane 0 (Box-3D27P) is evaluated on the shared class sums
+    (13.5 FP64 ops per point in the planner's count, against 15 for the two PMA planes); a plane
+    without the transposition symmetry, or LORA_NO_SYM3=1, keeps the PMA planes."""
+    W = synth.rsym_weights(3, 1, 7)
+    assert L.Stencil(W, (16, 16, 16), engine="rdg_cuda").info()["fma_per_point_issued"] == 13.5
+    Wa = W.copy()
+    Wa[1, 0, 1] = Wa[1, 2, 1] = W[1, 0, 1] * 1.5   # plane 1: b_vertical != b_horizontal (still PMA)
+    assert L.Stencil(Wa, (16, 16, 16), engine="rdg_cuda").info()["fma_per_point_issued"] == 15
+    monkeypatch.setenv("LORA_NO_SYM3", "1")
+    assert L.Stencil(W, (16, 16, 16), engine="rdg_cuda").info()["fma_per_point_issued"] == 15
+
+
 def test_plan_query_fields(L):
     W = synth.rsym_weights(2, 3, 4)
     info = L.Stencil(W, (100, 200), engine="tc").info()
