@@ -51,7 +51,10 @@ constexpr int F_S1 = 2 * F_WARPS;    // stage-1 rows per CTA column (2 per warp)
 constexpr int F_IN = F_S1 + 2;       // staged input rows
 constexpr int F_BW = 66;             // staged columns (64 + 2R)
 constexpr int F_S1W = 72;            // step-1 plane buffer row pitch (doubles): data at [1, 65)
-constexpr int F_ZC = 64;
+#ifndef RDG3F_ZC
+#define RDG3F_ZC 64   // z-chunk length (final planes per work item; balanced per grid)
+#endif
+constexpr int F_ZC = RDG3F_ZC;
 
 enum { PM_NONE = 0, PM_POINT = 1, PM_CHAINS = 2, PM_STAR = 3, PM_PMA1 = 4, PM_SYM3 = 6 };   // (values as in kernels_rdg3d.cu)
 constexpr int F_MAXK = 3;
@@ -140,7 +143,8 @@ struct Sig3 {
   static constexpr int m0 = M0, m1 = M1, mir = MIR;
   // TMA ring stages: 4 for the light point + star (Heat-3D) kernel (420 -> 430 GS/s), 3 otherwise
   // (Box-3D27P: 392 with 3, 388 with 4; tools/gpu_variants.sh, same box)
-  static constexpr int ns = RDG3F_NS > 0 ? RDG3F_NS : ((M0 == 1 && M1 == 3) ? 4 : 3);
+  // and the joint symmetric planes (Box-3D27P: 447 with 3, 456 with 4; r02zh)
+  static constexpr int ns = RDG3F_NS > 0 ? RDG3F_NS : (((M0 == 1 && M1 == 3) || M0 == PM_SYM3) ? 4 : 3);
   // plane 0 statically non-empty and its result an FMA chain: its contribution assigns (a bare
   // product, PM_POINT, would let nvcc contract it with the next addition into one FMA, which the
   // unfused kernel's 0 + w x does not: results would differ from two single steps in the last bit)
