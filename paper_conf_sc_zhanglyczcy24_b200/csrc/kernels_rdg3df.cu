@@ -3,16 +3,17 @@
 //
 // A CTA (8 warps) owns a column of the domain: 64 lane columns x 16 step-1 rows (14 final rows),
 // streaming along z through a chunk of ZC final planes.  For every input plane p (TMA 3D box
-// 18 x 66, 3-stage ring; zero fill outside the array):
+// 18 x 66, 3- or 4-stage ring; zero fill outside the array):
 //   stage 1: warp w applies the plane operators (Alg. 2: PMA / star / point-wise / general rank-1
-//            chains per plane) to produce step-1 rows 2w, 2w+1 and scatters them into a register
+//            chains per plane; the two symmetric planes of Box-3D27P jointly on shared class sums,
+//            PM_SYM3, Q18) to produce step-1 rows 2w, 2w+1 and scatters them into a register
 //            z-ring of 3 step-1 planes; the completed step-1 plane p-1 gets the fixed Dirichlet halo
 //            re-imposed and is written to a shared plane buffer (double-buffered);
 //   one __syncthreads;
 //   stage 2: warps 0..6 apply the same operators to that step-1 plane (final rows 2w, 2w+1) into a
 //            second z-ring; the completed final plane p-2 is stored.
 // Every point goes through the same arithmetic as two unfused steps of kernels_rdg3d.cu's mode
-// code, so the result equals two separate steps to rounding; halo handling makes it exact
+// code (bitwise equal to two unfused steps), so the result equals two steps to rounding; halo handling makes it exact
 // temporal blocking (reading Q5).  The lane columns lose one valid column per side per
 // fused step: x bands overlap with stride 60 (even TMA origin).
 #include <cuda_runtime.h>
