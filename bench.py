@@ -332,19 +332,21 @@ def main():
     stream = torch.cuda.current_stream(dev)
     sptr = stream.cuda_stream
 
-    zero_copy = ep is not None and info["fuse_k"] == 1
+    zero_copy = ep is not None
     if zero_copy:
-        # zero-copy use of the exchange buffers (unfused launches keep the caller's layout): the slab
-        # lives in buffer 0, the result lands in buffer T % 2 (T even: buffer 0 again, so each timed
-        # step continues the evolution).  Fused launches use deep halos: copy-in / copy-out instead.
-        b0 = L.lora_stencil_p2p_buffer(ep, 0)
+        # zero-copy use of the exchange buffers: the slab lives in the caller-layout view of buffer 0
+        # (lora_stencil_p2p_view: inside the deep-halo buffer for fused launches), the result lands in
+        # view n_launch % 2 (n_launch = ceil(T / k) even: view 0 again, so each timed step continues
+        # the evolution) — no copy-in / copy-out per step
+        n_launch = -(-T // max(1, info["fuse_k"]))
+        b0 = L.lora_stencil_p2p_view(ep, 0)
 
         class _Dev:
             __cuda_array_interface__ = {"shape": tuple(x.shape), "typestr": "<f8", "data": (int(b0), False),
                                         "version": 3, "strides": None}
         torch.as_tensor(_Dev(), device=dev).copy_(x)
         torch.cuda.synchronize(dev)
-        bT = L.lora_stencil_p2p_buffer(ep, T % 2)
+        bT = L.lora_stencil_p2p_view(ep, n_launch % 2)
 
     def step():
         if ep is not None:

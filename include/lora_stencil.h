@@ -219,10 +219,11 @@ int lora_stencil_dist_exchange_plan_ex(const lora_plan* p, int rank, int nranks,
  *
  * Exchange buffers: the communicator owns two padded slabs (the ping-pong pair the neighbours
  * write into; rows = lower halo depth + n0 + upper halo depth) plus the flag words, allocated with
- * cudaMalloc on the current device (IPC-exportable).  lora_stencil_p2p_buffer exposes them: for an
- * unfused endpoint (k = 1) they have the caller's layout, and a caller that fills buffer 0 directly
- * and passes it as `in_local` (and buffer L%2 as `out_local`, L = the number of launches = T for
- * k = 1) avoids the copy-in / copy-out.
+ * cudaMalloc on the current device (IPC-exportable).  lora_stencil_p2p_buffer exposes them, and
+ * lora_stencil_p2p_view the caller-layout array inside each (the padded local slab with R-deep halos,
+ * same row pitch, starting at buffer row hl - R; the buffer itself for an unfused endpoint): a caller
+ * that fills view 0 directly and passes it as `in_local` (and view L%2 as `out_local`, L = the
+ * number of launches, ceil(T / k)) avoids the copy-in / copy-out, fused or not.
  *
  * A spin-wait that sees no progress for 20 s (a neighbour that never runs) gives up instead of
  * hanging the GPU and sets a device error word: lora_stencil_p2p_status reports it. */
@@ -243,6 +244,9 @@ int lora_stencil_p2p_connect(lora_p2p* c, const void* lo_handle, const void* hi_
 int lora_stencil_p2p_connect_local(lora_p2p* c, const lora_p2p* lo, const lora_p2p* hi);
 /* Device pointer of exchange buffer i (0 or 1), or NULL. */
 double* lora_stencil_p2p_buffer(const lora_p2p* c, int i);
+/* Device pointer of the caller-layout view of exchange buffer i (0 or 1; see above), or NULL.
+ * Owned by the endpoint; valid until lora_stencil_p2p_destroy. */
+double* lora_stencil_p2p_view(const lora_p2p* c, int i);
 /* Collective over the connected ranks (every rank calls with the same timesteps), ordered on
  * `stream`: copy-in (skipped if in_local is buffer 0), T steps with the in-kernel exchange, a
  * final wait for the neighbours' last rows, copy-out (skipped if out_local is buffer T%2). */

@@ -87,6 +87,7 @@ _sig = {
     "lora_stencil_p2p_connect": (ctypes.c_int, [_P, _P, _P]),
     "lora_stencil_p2p_connect_local": (ctypes.c_int, [_P, _P, _P]),
     "lora_stencil_p2p_buffer": (_P, [_P, ctypes.c_int]),
+    "lora_stencil_p2p_view": (_P, [_P, ctypes.c_int]),
     "lora_stencil_run_dist_p2p": (ctypes.c_int, [_P, _P, _P, _P, ctypes.c_int64, _P]),
     "lora_stencil_p2p_status": (ctypes.c_int, [_P]),
     "lora_stencil_p2p_destroy": (None, [_P]),
@@ -265,6 +266,12 @@ def lora_stencil_p2p_connect_local(c, lo, hi) -> None:
 
 def lora_stencil_p2p_buffer(c, i: int) -> int:
     return int(_lib.lora_stencil_p2p_buffer(c, int(i)) or 0)
+
+
+def lora_stencil_p2p_view(c, i: int) -> int:
+    """Caller-layout view (padded local slab, R-deep halos) inside exchange buffer i: pass view 0 as
+    `in` and view (launches % 2) as `out` of lora_stencil_run_dist_p2p to skip the copies."""
+    return int(_lib.lora_stencil_p2p_view(c, int(i)) or 0)
 
 
 def lora_stencil_run_dist_p2p(plan, c, in_ptr: int, out_ptr: int, timesteps: int, stream: int = 0) -> None:

@@ -307,6 +307,11 @@ double* lora_stencil_p2p_buffer(const lora_p2p* c, int i) {
   return c->buf[i];
 }
 
+double* lora_stencil_p2p_view(const lora_p2p* c, int i) {
+  if (!c || i < 0 || i > 1) return nullptr;
+  return c->buf[i] + int64_t(c->hl - c->R) * c->row;   // caller row 0 = buffer row hl - R
+}
+
 int lora_stencil_run_dist_p2p(lora_plan* p, lora_p2p* c, const double* in_local, double* out_local,
                               int64_t timesteps, void* stream) {
   using namespace lora;
@@ -329,10 +334,11 @@ int lora_stencil_run_dist_p2p(lora_plan* p, lora_p2p* c, const double* in_local,
     done += st;
   }
   const int64_t L = (int64_t)steps.size();
-  const bool same_layout = c->hl == R && c->hh == R;
-  // zero-copy use of the exchange buffers (caller layout only): in = buffer 0 and out = buffer L%2
-  // may coincide (L even): `in` is fully consumed by the first launch and its halo is buffer 0's own
-  const bool zero_copy = same_layout && in_local == c->buf[0] && out_local == c->buf[L % 2];
+  // zero-copy use of the exchange buffers: in = the caller-layout view of buffer 0 and out = that of
+  // buffer L%2 (lora_stencil_p2p_view; the buffers themselves for R-deep halos) may coincide (L even):
+  // `in` is fully consumed by the first launch and its halo is buffer 0's own
+  const int64_t vshift = int64_t(c->hl - R) * c->row;
+  const bool zero_copy = in_local == c->buf[0] + vshift && out_local == c->buf[L % 2] + vshift;
   const char* a = reinterpret_cast<const char*>(in_local);
   const char* b = reinterpret_cast<const char*>(out_local);
   if (!zero_copy && a < b + bytes && b < a + bytes) return fail(LORA_ERR_ALIAS, "in and out overlap");

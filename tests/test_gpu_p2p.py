@@ -54,19 +54,20 @@ def _run_local(W, g, h, shape, T, engine, counts, zero_copy=False, repeat=1, fus
     for r in range(P):
         L.lora_stencil_p2p_connect_local(eps[r], eps[r - 1] if r > 0 else None, eps[r + 1] if r < P - 1 else None)
     torch.cuda.synchronize()
+    nl = -(-T // max(1, sts[0].info()["fuse_k"])) if engine == "rdg_cuda" else T   # launches per run
     for _ in range(repeat):
         if zero_copy:
-            # fill every rank's buffer 0 through a tensor view of the library buffer BEFORE any run is
-            # enqueued: a device-wide synchronize between the ranks' enqueues would wait on a kernel
-            # that spins for a neighbour whose run is not enqueued yet
+            # fill every rank's view 0 (the caller layout inside exchange buffer 0; with deep halos it
+            # starts H - h rows in) BEFORE any run is enqueued: a device-wide synchronize between the
+            # ranks' enqueues would wait on a kernel that spins for a neighbour whose run is not enqueued yet
             for r in range(P):
-                torch.as_tensor(_DevBuf(L.lora_stencil_p2p_buffer(eps[r], 0), xs[r].shape), device="cuda").copy_(xs[r])
+                torch.as_tensor(_DevBuf(L.lora_stencil_p2p_view(eps[r], 0), xs[r].shape), device="cuda").copy_(xs[r])
             torch.cuda.synchronize()
         for r in range(P):
             inp, outp = xs[r].data_ptr(), ys[r].data_ptr()
             if zero_copy:
-                inp = L.lora_stencil_p2p_buffer(eps[r], 0)
-                outp = L.lora_stencil_p2p_buffer(eps[r], T % 2)
+                inp = L.lora_stencil_p2p_view(eps[r], 0)
+                outp = L.lora_stencil_p2p_view(eps[r], nl % 2)
             L.lora_stencil_run_dist_p2p(sts[r].plan, eps[r], inp, outp, T, streams[r].cuda_stream)
         torch.cuda.synchronize()
     for r in range(P):
@@ -74,7 +75,7 @@ def _run_local(W, g, h, shape, T, engine, counts, zero_copy=False, repeat=1, fus
     out = g.copy()
     for r, (s0, c) in enumerate(slabs):
         if zero_copy:
-            res = torch.as_tensor(_DevBuf(L.lora_stencil_p2p_buffer(eps[r], T % 2), xs[r].shape), device="cuda")
+            res = torch.as_tensor(_DevBuf(L.lora_stencil_p2p_view(eps[r], nl % 2), xs[r].shape), device="cuda")
             res = res.cpu().numpy()
         else:
             res = ys[r].cpu().numpy()
@@ -161,6 +162,10 @@ def test_p2p_fused_deep_halo_bitwise(case):
         assert np.array_equal(out, ref), (T, float(np.nanmax(np.abs(out - ref))))
     out = _run_local(W, g, h, shape, 5, "rdg_cuda", counts, fuse_k=k, repeat=2)
     assert np.array_equal(out, _global(W, g, 5, "rdg_cuda"))
+    # zero-copy through the caller-layout views of the deep-halo buffers (lora_stencil_p2p_view)
+    for T in (2 * k, 2 * k + 1):
+        out = _run_local(W, g, h, shape, T, "rdg_cuda", counts, fuse_k=k, zero_copy=True)
+        assert np.array_equal(out, _global(W, g, T, "rdg_cuda")), T
 
 
 FUSED3D = [
