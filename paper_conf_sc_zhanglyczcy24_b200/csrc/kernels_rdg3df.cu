@@ -389,22 +389,22 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
   auto issue_next = [&](int slot) {
     double* dst = reinterpret_cast<double*>(ring + slot * STAGE);
     const int x = pX - 1, y = pY - K, z = pZ - K + pj;
-    if (act && pj == 0 && tid == 0) {   // this column's halo planes come from a neighbour
-      bool lo, hi;
+    if (act && pj == 0 && w == 0) {   // this column's halo planes come from a neighbour (warp 0,
+      bool lo, hi;                     // warp-uniform wait: kernels.hpp / p2p.cuh p2p_wait_units_warp)
       touches(pZ, lo, hi);
       if (lo || hi) {
         if (dp.wait_units > 0) {   // the neighbour's previous launch had another geometry: every unit
-          if (lo) p2p_wait_units(dp.wait_lo, 0, dp.wait_units - 1, dp.wait_val, dp.err);
-          if (hi) p2p_wait_units(dp.wait_hi, 0, dp.wait_units - 1, dp.wait_val, dp.err);
+          if (lo) p2p_wait_units_warp(dp.wait_lo, 0, dp.wait_units - 1, dp.wait_val, dp.err);
+          if (hi) p2p_wait_units_warp(dp.wait_hi, 0, dp.wait_units - 1, dp.wait_val, dp.err);
         } else {
           const int u = pitem % (nbx * nby), ux = u % nbx, uy = u / nbx;
           for (int yy = max(uy - 1, 0); yy <= min(uy + 1, nby - 1); ++yy) {
             const int u0 = yy * nbx + max(ux - 1, 0), u1 = yy * nbx + min(ux + 1, nbx - 1);
-            if (lo) p2p_wait_units(dp.wait_lo, u0, u1, dp.wait_val, dp.err);
-            if (hi) p2p_wait_units(dp.wait_hi, u0, u1, dp.wait_val, dp.err);
+            if (lo) p2p_wait_units_warp(dp.wait_lo, u0, u1, dp.wait_val, dp.err);
+            if (hi) p2p_wait_units_warp(dp.wait_hi, u0, u1, dp.wait_val, dp.err);
           }
         }
-        fence_proxy_async_global();
+        if (lane == 0) fence_proxy_async_global();
       }
     }
     // warp 0 reconverges here: lane 0 may have spun above, and the CTA barriers that follow are
@@ -573,15 +573,17 @@ __global__ void __launch_bounds__(F_WARPS * 32, RDG3F_MINB) rdg3df_kernel(const 
             // the plane goes to this slab and, for the first / last H own planes of a slab with a
             // neighbour there, into that neighbour's halo as well (peer memory)
             const int64_t e0 = (int64_t(zf) * P1 + Y0 + 2 * w) * P2 + X0 + c0;
-            const bool rlo = t_lo && zf < dp.lo_end, rhi = t_hi && zf >= dp.hi_begin;
-            const int nd = 1 + (rlo ? 1 : 0) + (rhi ? 1 : 0);
-            for (int d = 0; d < nd; ++d) {
-              double* o = d == 0 ? out + e0 : ((rlo && d == 1) ? dp.dst_lo + (e0 + dp.off_lo) : dp.dst_hi + (e0 + dp.off_hi));
+            auto store_to = [&](double* o) {
 #pragma unroll
               for (int y = 0; y < 2; ++y)
 #pragma unroll
                 for (int e = 0; e < 2; ++e)
                   if (st_ok[y][e]) o[y * P2 + e] = acc[K - 1][s][y][e];
+            };
+            store_to(out + e0);
+            if (act) {   // (uniform per CTA; rare: the slab's first / last H planes)
+              if (t_lo && zf < dp.lo_end) store_to(dp.dst_lo + (e0 + dp.off_lo));
+              if (t_hi && zf >= dp.hi_begin) store_to(dp.dst_hi + (e0 + dp.off_hi));
             }
           }
           if constexpr (!SG::assign0) {
