@@ -373,7 +373,8 @@ __device__ __forceinline__ void store_pairs(double* o, const double (&v)[NH][2],
 // PRE: stage S's input row is already in xq (the prefetched stage-1 row); stages S down to SMIN run.
 // LOOP: runtime row loop (row index Ir, shift-register row update row_shift) instead of the ring
 // form unrolled over the 2R + 1 ring positions (template row index I, ring position I0).
-template <int R, int SIG, int K, int NH, bool FULL, int I0, int I_, int S, bool PRE = false, int SMIN = 1, bool LOOP = false>
+template <int R, int SIG, int K, int NH, bool FULL, int I0, int I_, int S, bool PRE = false, int SMIN = 1, bool LOOP = false,
+          bool REM = true>
 __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, int p,
                                            double (&acc)[K][NH][2 * R + 1][2], const RdgParams& P,
                                            double* __restrict__ bufs, int par, const double* __restrict__ in,
@@ -458,7 +459,7 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
         // LOOP: orow is this row's output pointer, advanced by the loop (no 64-bit index per row)
         double* o = LOOP ? orow : out + (sc.ooff + int64_t(I) * P1);
         store_pairs<NH, (R & 1) != 0>(o, v, lc);
-        if (I < sc.rem_lo || I >= sc.rem_hi) {   // warp-uniform, rare
+        if (REM && (I < sc.rem_lo || I >= sc.rem_hi)) {   // warp-uniform, rare (REM: the stage has such rows)
           const int64_t e = sc.ooff + int64_t(I) * P1;
           if (I < sc.rem_lo) store_pairs<NH>(dp.dst_lo + (e + dp.off_lo), v, lc);
           if (I >= sc.rem_hi) store_pairs<NH>(dp.dst_hi + (e + dp.off_hi), v, lc);
@@ -486,7 +487,7 @@ __device__ __forceinline__ void fused_iter(const double* __restrict__ st_row, in
     }
   }
   if constexpr (S > SMIN)
-    fused_iter<R, SIG, K, NH, FULL, I0, I_, S - 1, false, SMIN, LOOP>(st_row, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, Ir,
+    fused_iter<R, SIG, K, NH, FULL, I0, I_, S - 1, false, SMIN, LOOP, REM>(st_row, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, Ir,
                                                                       orow);
 }
 
@@ -562,7 +563,7 @@ constexpr bool rdg_loop() {
 }
 
 // The rows of one staged tile as a runtime loop (one copy of the K x NH row code; see row_shift).
-template <int R, int SIG, int K, int NH, bool FULL>
+template <int R, int SIG, int K, int NH, bool FULL, bool REM = true>
 __device__ __forceinline__ void fused_rows_loop(const double* __restrict__ st, int p, double (&acc)[K][NH][2 * R + 1][2],
                                                 const RdgParams& P, double* __restrict__ bufs,
                                                 const double* __restrict__ in, double* __restrict__ out, int64_t P1,
@@ -579,16 +580,16 @@ __device__ __forceinline__ void fused_rows_loop(const double* __restrict__ st, i
   for (int I = 0; I < SROWS; ++I, orow += P1) {
     const int par = (par0 + I) & 1;
     if constexpr (PF) {
-      fused_iter<R, SIG, K, NH, FULL, 0, 0, 1, true, 1, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, 1, true, 1, true, REM>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
                                                               orow);
       if (I + 1 < SROWS) {
 #pragma unroll
         for (int h = 0; h < NH && h < RDG_PF_HALVES; ++h) load_x<R>(st + (I + 1) * BW + 64 * h, p, xq[h]);
       }
-      fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 2, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 2, true, REM>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
                                                                orow);
     } else {
-      fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 1, true>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 1, true, REM>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
                                                                orow);
     }
     __syncwarp();
@@ -813,8 +814,12 @@ __global__ void __launch_bounds__(RDG_WARPS * 32, (rdg_minb<R, SIG, K>())) rdg2d
     for (int S = 1; S < K; ++S) full = full && sc.hlo[S - 1] <= 0 && sc.hhi[S - 1] >= G::SROWS;
     double xq[NH][2 * R + 2];   // prefetched stage-1 input row (RDG_PF)
     if constexpr (rdg_loop<R, SIG, K>()) {
+      // P2P: only the stages holding one of the slab's first / last H rows take the row code with
+      // the peer stores (the others run the single-GPU row code: 931 vs 997 us per launch)
+      const bool rem = P2P && (sc.rem_lo > 0 || sc.rem_hi < G::SROWS);
       if (rdg_full<R, SIG, K>() && full) fused_rows_loop<R, SIG, K, NH, true>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
-      else fused_rows_loop<R, SIG, K, NH, false>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
+      else if (rem) fused_rows_loop<R, SIG, K, NH, false, true>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
+      else fused_rows_loop<R, SIG, K, NH, false, false>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
     } else {
       if (rdg_full<R, SIG, K>() && full) fused_rows<R, SIG, K, NH, true, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
       else fused_rows<R, SIG, K, NH, false, 0>(st, lane, acc, prm, bufs, in, out, P1, sc, lc, yb & 1, dp, xq);
