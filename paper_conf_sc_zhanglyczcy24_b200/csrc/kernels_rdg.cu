@@ -42,6 +42,9 @@ constexpr int kRowUnroll = RDG_LOOP_UNROLL;   // (#pragma arguments are not macr
 #define RDG_WARPS_PER_CTA 4   // (Box-2D49P k=2: 2 warps 351, 4 warps 350, 8 warps 270 GS/s; Box-2D9P k=3: 654 / 692)
 #endif
 constexpr int RDG_WARPS = RDG_WARPS_PER_CTA;   // warps per CTA (independent streams)
+#ifndef RDG_S1FIRST
+#define RDG_S1FIRST 0   // 1: stage 1 before stages K .. 2 in each row iteration (r02zr: Box-2D49P 448 -> 426)
+#endif
 #ifndef RDG_PF_HALVES
 #define RDG_PF_HALVES 2   // 64-column halves of the next row prefetched (RDG_PF, loop form)
 #endif
@@ -588,6 +591,11 @@ __device__ __forceinline__ void fused_rows_loop(const double* __restrict__ st, i
       }
       fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 2, true, REM>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
                                                                orow);
+    } else if constexpr (RDG_S1FIRST) {   // stage 1, then stages K .. 2 (the stages of an iteration are independent)
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, 1, false, 1, true, REM>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
+                                                                    orow);
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 2, true, REM>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
+                                                                    orow);
     } else {
       fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 1, true, REM>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
                                                                orow);
