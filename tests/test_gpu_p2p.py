@@ -164,7 +164,7 @@ def test_p2p_fused_deep_halo_bitwise(case):
     assert np.array_equal(out, _global(W, g, 5, "rdg_cuda"))
     # zero-copy through the caller-layout views of the deep-halo buffers (lora_stencil_p2p_view)
     for T in (2 * k, 2 * k + 1):
-        out = _run_local(W, g, h, shape, T, "rdg_cuda", counts, fuse_k=k, zero_copy=True)
+        out = _run_local(W, g, h, shape, T, "rdg_cuda", counts, fuse_k=k, zero_copy=True, repeat=2)
         assert np.array_equal(out, _global(W, g, T, "rdg_cuda")), T
 
 
