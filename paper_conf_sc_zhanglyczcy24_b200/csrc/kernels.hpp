@@ -27,8 +27,8 @@ inline bool pma1_unit_centre(const double* u, const double* v, double* uo, doubl
 // plane 0 (Box-3D27P), the 3D CUDA-core kernels evaluate the two plane operators JOINTLY on the
 // symmetric class sums they share (mode PM_SYM3, reading Q18): with px = x_l + x_r per
 // row, s1 = x_u + x_d, pc = px_u + px_d (corners), e = px + s1 (edges),
-//   d_k = a_k pc + (b_k e + c_k x)        (k = plane 0, 1)
-// 11 FP64 ops per point for both operators instead of 16 for the two PMA chains.  Both kernels
+//   d_0 = a_0 pc + (b_0 e + c_0 x); plane 1 straight into its accumulator: acc = a_1 pc + (b_1 e + (c_1 x + acc))
+// 12 FP64 ops per point for both operators (incl. accumulation) instead of 16 for the two PMA chains.  Both kernels
 // (unfused and fused) use the same formula in the same order, so they stay bitwise equal.
 // LORA_NO_SYM3=1 keeps the PMA form (A/B).  Returns false unless the plane has the symmetry.
 inline bool sym3_plane(const double* W, int a0, double& c, double& b, double& a) {

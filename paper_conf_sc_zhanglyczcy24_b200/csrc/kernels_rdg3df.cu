@@ -176,10 +176,9 @@ __device__ __forceinline__ void planes2(const double (&x)[4][4], const FParams& 
           const double pc = px[y][e] + px[y + 2][e];
           const double ed = px[y + 1][e] + sv;
           const double d0 = fma(P.sym[0][2], pc, fma(P.sym[0][1], ed, P.sym[0][0] * xc));
-          const double d1 = fma(P.sym[1][2], pc, fma(P.sym[1][1], ed, P.sym[1][0] * xc));
           acc[s0][y][e] = d0;
           acc[s2][y][e] += d0;
-          acc[s1][y][e] += d1;
+          acc[s1][y][e] = fma(P.sym[1][2], pc, fma(P.sym[1][1], ed, fma(P.sym[1][0], xc, acc[s1][y][e])));   // plane 1 into its slot
         }
     }
   } else if constexpr (A0 < 3) {

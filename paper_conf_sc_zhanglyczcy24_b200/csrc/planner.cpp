@@ -221,7 +221,8 @@ double cuda_fma_per_point(const Plan& p) {
   if (p.ndim == 3 && p.R == 1 && sym3_enabled()) {
     // PM_SYM3 (kernels.hpp sym3_plane; chosen by the 3D kernels when planes 0 and 1 are PMA planes
     // with the full [a b a; b c b; a b a] symmetry and plane 2 mirrors plane 0): px 1.5 (6 rows per 4
-    // outputs), 3 shared class sums, 3 per plane operator, 3 accumulating adds
+    // outputs), 3 shared class sums, 3 per plane operator, 2 accumulating adds (plane 1's operator
+    // accumulates through its FMAs)
     auto pma1 = [&](int q) {
       int cnt = 0, chain = 0, point = 0;
       for (const Term& t : p.terms)
@@ -232,7 +233,7 @@ double cuda_fma_per_point(const Plan& p) {
     for (int e = 0; e < 9; ++e) mir = mir && p.W[size_t(18) + e] == p.W[size_t(e)];
     double c, b, a;
     if (mir && pma1(0) && pma1(1) && sym3_plane(p.W.data(), 0, c, b, a) && sym3_plane(p.W.data(), 1, c, b, a))
-      return 1.5 + 3.0 + 2 * 3.0 + 3.0;
+      return 1.5 + 3.0 + 2 * 3.0 + 2.0;
   }
   double f = 0;
   for (int q = 0; q < n; ++q) {

@@ -232,10 +232,10 @@ def test_cuda_core_rank1_forms(L, monkeypatch):
 def test_3d_joint_symmetric_planes(L, monkeypatch):
     """3D CUDA-core engine (reading Q18): a radius-1 W whose planes 0 and 1 are
     [a b a; b c b; a b a] with plane 2 = plane 0 (Box-3D27P) is evaluated on the shared class sums
-    (13.5 FP64 ops per point in the planner's count, against 15 for the two PMA planes); a plane
+    (12.5 FP64 ops per point in the planner's count, against 15 for the two PMA planes); a plane
     without the transposition symmetry, or LORA_NO_SYM3=1, keeps the PMA planes."""
     W = synth.rsym_weights(3, 1, 7)
-    assert L.Stencil(W, (16, 16, 16), engine="rdg_cuda").info()["fma_per_point_issued"] == 13.5
+    assert L.Stencil(W, (16, 16, 16), engine="rdg_cuda").info()["fma_per_point_issued"] == 12.5
     Wa = W.copy()
     Wa[1, 0, 1] = Wa[1, 2, 1] = W[1, 0, 1] * 1.5   # plane 1: b_vertical != b_horizontal (still PMA)
     assert L.Stencil(Wa, (16, 16, 16), engine="rdg_cuda").info()["fma_per_point_issued"] == 15
