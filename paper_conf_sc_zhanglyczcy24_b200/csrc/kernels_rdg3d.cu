@@ -201,10 +201,34 @@ __device__ __forceinline__ void apply_sym3(const double (&x)[BY<1> + 2][4], doub
     }
 }
 
+// Heat-3D signature (R = 1: point planes 0 / 2 mirrored, star plane 1): every contribution goes
+// straight into its accumulator through FMAs (8 FP64 ops per point instead of 10 with the products
+// and sums formed first); the same formula and order as kernels_rdg3df.cu's planes2.
+template <int I>
+__device__ __forceinline__ void apply_heat(const double (&x)[BY<1> + 2][4], double (&acc)[3][BY<1>][2],
+                                           const R3Params& P) {
+  constexpr int s0 = pm(I, 3), s2 = pm(I - 2, 3), s1 = pm(I - 1, 3);
+#pragma unroll
+  for (int y = 0; y < BY<1>; ++y)
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {
+      acc[s0][y][e] = fma(P.w[0], x[y + 1][1 + e], acc[s0][y][e]);
+      acc[s2][y][e] = fma(P.w[0], x[y + 1][1 + e], acc[s2][y][e]);
+      double t = acc[s1][y][e];
+#pragma unroll
+      for (int b = -1; b <= 1; ++b) t = fma(P.v[1][0][1 + b], x[y + 1][1 + e + b], t);
+#pragma unroll
+      for (int a = -1; a <= 1; ++a) t = fma(P.u[1][1][1 + a], x[y + 1 + a][1 + e], t);
+      acc[s1][y][e] = t;
+    }
+}
+
 template <int R, class SG, int A0, int I>
 __device__ __forceinline__ void apply_all(const double (&x)[BY<R> + 2 * R][2 * R + 2],
                                           double (&acc)[2 * R + 1][BY<R>][2], const R3Params& P) {
-  if constexpr (R == 1 && SG::m0 == PM_SYM3) {
+  if constexpr (R == 1 && SG::m0 == PM_POINT && SG::m1 == PM_STAR && SG::mir == 1) {
+    if constexpr (A0 == 0) apply_heat<I>(x, acc, P);
+  } else if constexpr (R == 1 && SG::m0 == PM_SYM3) {
     static_assert(SG::m1 == PM_SYM3 && SG::mir == 1, "PM_SYM3 signature");
     if constexpr (A0 == 0) apply_sym3<I>(x, acc, P);
   } else if constexpr (A0 < 2 * R + 1) {

@@ -157,7 +157,25 @@ struct Sig3 {
 // apply_sym3 (plane 0 assigned to its slot, added to the mirror slot; plane 1 added).
 template <class SG, int I, int A0>
 __device__ __forceinline__ void planes2(const double (&x)[4][4], const FParams& P, double (&acc)[3][2][2]) {
-  if constexpr (SG::m0 == PM_SYM3) {
+  if constexpr (SG::m0 == PM_POINT && SG::m1 == PM_STAR && SG::mir == 1) {
+    // Heat-3D: every contribution straight into its accumulator (kernels_rdg3d.cu apply_heat)
+    if constexpr (A0 == 0) {
+      constexpr int s0 = pm3(I), s2 = pm3(I - 2), s1 = pm3(I - 1);
+#pragma unroll
+      for (int y = 0; y < 2; ++y)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          acc[s0][y][e] = fma(P.w[0], x[y + 1][1 + e], acc[s0][y][e]);
+          acc[s2][y][e] = fma(P.w[0], x[y + 1][1 + e], acc[s2][y][e]);
+          double t = acc[s1][y][e];
+#pragma unroll
+          for (int b = -1; b <= 1; ++b) t = fma(P.v[1][0][1 + b], x[y + 1][1 + e + b], t);
+#pragma unroll
+          for (int a = -1; a <= 1; ++a) t = fma(P.u[1][1][1 + a], x[y + 1 + a][1 + e], t);
+          acc[s1][y][e] = t;
+        }
+    }
+  } else if constexpr (SG::m0 == PM_SYM3) {
     static_assert(SG::m1 == PM_SYM3 && SG::mir == 1 && SG::assign0, "PM_SYM3 signature");
     if constexpr (A0 == 0) {
       double px[4][2];
