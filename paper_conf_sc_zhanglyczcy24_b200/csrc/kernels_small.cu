@@ -345,6 +345,9 @@ small2d_grid_kernel(const double* __restrict__ in, double* __restrict__ out, dou
 #ifndef SMALL_TILE_STRIPS
 #define SMALL_TILE_STRIPS 1   // threads walk row strips with a register window (0: one point per iteration)
 #endif
+#ifndef SMALL_TILE_FULL
+#define SMALL_TILE_FULL 1     // every step over the whole staged interior (fixed bounds; 0: the shrinking cone)
+#endif
 #ifndef SMALL_TILE_TY
 #define SMALL_TILE_TY 8   // 512 threads (Heat-2D 256^2 x 10: 11.7 us back to back vs 14.0 with 4, 13.4 with 2)
 #endif
@@ -363,20 +366,24 @@ small2d_tile_kernel(const double* __restrict__ in, double* __restrict__ out, int
   double* const buf1 = sm + size_t(SY) * SX;
   const int tid = threadIdx.y * TL_TX + threadIdx.x;
   constexpr int NT = TL_TX * TL_TY;
-  {  // staging: all of a thread's loads first (one HBM / L2 latency instead of one per element)
+  {  // staging: thread (x, y) takes columns x, x + 64, ... of rows y, y + TL_TY, ...; all of a thread's
+     // loads of a column first (one HBM / L2 latency instead of one per element), no divisions
     constexpr int U = 8;
-    for (int i0 = tid; i0 < SY * SX; i0 += NT * U) {
-      double v[U];
+    for (int c = (int)threadIdx.x; c < SX; c += TL_TX) {
+      const int gx = gx0 + c;
+      const bool cin = gx >= 0 && gx < P1;
+      for (int r0 = (int)threadIdx.y; r0 < SY; r0 += TL_TY * U) {
+        double v[U];
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const int i = i0 + u * NT, r = i / SX, c = i - r * SX;
-        const int gy = gy0 + r, gx = gx0 + c;
-        v[u] = (i < SY * SX && gy >= 0 && gy < P0 && gx >= 0 && gx < P1) ? __ldg(in + int64_t(gy) * P1 + gx) : 0.0;
-      }
+        for (int u = 0; u < U; ++u) {
+          const int r = r0 + u * TL_TY, gy = gy0 + r;
+          v[u] = (r < SY && cin && gy >= 0 && gy < P0) ? __ldg(in + int64_t(gy) * P1 + gx) : 0.0;
+        }
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const int i = i0 + u * NT;
-        if (i < SY * SX) { buf0[i] = v[u]; buf1[i] = v[u]; }
+        for (int u = 0; u < U; ++u) {
+          const int r = r0 + u * TL_TY;
+          if (r < SY) { buf0[r * SX + c] = v[u]; buf1[r * SX + c] = v[u]; }
+        }
       }
     }
   }
@@ -385,13 +392,47 @@ small2d_tile_kernel(const double* __restrict__ in, double* __restrict__ out, int
   const int ilo_r = max(0, R - gy0), ihi_r = min(SY, R + N0 - gy0);
   const int ilo_c = max(0, R - gx0), ihi_c = min(SX, R + N1 - gx0);
   int cur = 0;
+#if SMALL_TILE_FULL
+  // every step computes the whole staged interior except its outer R ring (fixed bounds, no per-step
+  // set-up): cells within s R of the staged edge are stale after step s, and s R <= T R = H never
+  // reaches the own tile, whose values are exactly those of the per-step path
+  const int r0 = max(ilo_r, R), r1 = min(ihi_r, SY - R), c0 = max(ilo_c, R), c1 = min(ihi_c, SX - R);
+  const int per = (r1 - r0 + TL_TY - 1) / TL_TY;
+  const int ra = r0 + (int)threadIdx.y * per, rb = min(r1, ra + per);
+#endif
   for (int st = 1; st <= T; ++st) {
     const double* src = cur ? buf1 : buf0;
     double* dst = cur ? buf0 : buf1;
+#if !SMALL_TILE_FULL
     const int m = (T - st) * R;   // distance from the own tile still computed at this step
     const int r0 = max(ilo_r, H - m), r1 = min(ihi_r, H + ty1 + m);
     const int c0 = max(ilo_c, H - m), c1 = min(ihi_c, H + tx1 + m);
-#if SMALL_TILE_STRIPS
+#endif
+#if SMALL_TILE_FULL
+    for (int c = c0 + (int)threadIdx.x; c < c1 && ra < rb; c += TL_TX) {
+      const double* cp = src + size_t(ra) * SX + c;
+      double* op = dst + size_t(ra) * SX + c;
+      double win[2 * R + 1];
+#pragma unroll
+      for (int a = 0; a < 2 * R; ++a) win[a] = cp[(a - R) * SX];
+#pragma unroll 2
+      for (int r = ra; r < rb; ++r, cp += SX, op += SX) {
+        win[2 * R] = cp[R * SX];
+        double th = 0.0;
+#pragma unroll
+        for (int b = -R; b <= R; ++b) th = fma(w.h[R + b], b == 0 ? win[R] : cp[b], th);
+        double acc = 0.0;
+#pragma unroll
+        for (int a = -R; a <= R; ++a) {
+          if (a == 0) acc += th;
+          acc = fma(w.v[R + a], win[R + a], acc);
+        }
+        *op = acc;
+#pragma unroll
+        for (int a = 0; a < 2 * R; ++a) win[a] = win[a + 1];
+      }
+    }
+#elif SMALL_TILE_STRIPS
     // each thread walks a strip of consecutive rows of one column with the 2R + 1 rows of the
     // vertical arm in a register window (one new shared load per row for it)
     const int nr = r1 - r0, per = (nr + TL_TY - 1) / TL_TY;
@@ -667,7 +708,7 @@ cudaError_t launch_grid_variant(Plan& p, const double* in, double* out, int64_t 
 }
 
 // Tile shape for the 2D-tile variant: the (TY, TX) in {8, 16, 32, 64}^2 with the least work per SM
-// (CTA rounds over the SMs x the CTA's trapezoid of points over the T steps); 0 if the halo'd tile
+// (CTA rounds over the SMs x the CTA's points over the T steps); 0 if the halo'd tile
 // does not fit the shared memory.
 bool tile_shape(const Plan& p, int64_t T, int sms, int& TY, int& TX, size_t& smem) {
   const int64_t H = T * p.R;
@@ -680,8 +721,8 @@ bool tile_shape(const Plan& p, int64_t T, int sms, int& TY, int& TX, size_t& sme
       if (sb > kMaxSmem) continue;
       const int64_t G = ((p.N[0] + ty - 1) / ty) * ((p.N[1] + tx - 1) / tx);
       double work = 0.0;
-      for (int64_t s = 1; s <= T; ++s) {
-        const int64_t m = (T - s) * p.R;
+      for (int64_t s = 1; s <= T; ++s) {   // points computed per step (SMALL_TILE_FULL: the staged interior)
+        const int64_t m = SMALL_TILE_FULL ? H - p.R : (T - s) * p.R;
         work += double(std::min<int64_t>(ey + 2 * m, p.N[0])) * double(std::min<int64_t>(ex + 2 * m, p.N[1]));
       }
       const double cost = double((G + sms - 1) / sms) * work;   // CTAs on the busiest SM x points per CTA
