@@ -345,6 +345,10 @@ small2d_grid_kernel(const double* __restrict__ in, double* __restrict__ out, dou
 #ifndef SMALL_TILE_STRIPS
 #define SMALL_TILE_STRIPS 1   // threads walk row strips with a register window (0: one point per iteration)
 #endif
+#ifndef SMALL_TILE_UNROLL
+#define SMALL_TILE_UNROLL 2   // row-strip unroll of the 2D-tile kernel
+#endif
+constexpr int kTileUnroll = SMALL_TILE_UNROLL;   // (#pragma arguments are not macro-expanded)
 #ifndef SMALL_TILE_FULL
 #define SMALL_TILE_FULL 1     // every step over the whole staged interior (fixed bounds; 0: the shrinking cone)
 #endif
@@ -415,7 +419,7 @@ small2d_tile_kernel(const double* __restrict__ in, double* __restrict__ out, int
       double win[2 * R + 1];
 #pragma unroll
       for (int a = 0; a < 2 * R; ++a) win[a] = cp[(a - R) * SX];
-#pragma unroll 2
+#pragma unroll kTileUnroll
       for (int r = ra; r < rb; ++r, cp += SX, op += SX) {
         win[2 * R] = cp[R * SX];
         double th = 0.0;
