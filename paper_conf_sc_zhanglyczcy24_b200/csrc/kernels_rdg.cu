@@ -42,6 +42,9 @@ constexpr int kRowUnroll = RDG_LOOP_UNROLL;   // (#pragma arguments are not macr
 #define RDG_WARPS_PER_CTA 4   // (Box-2D49P k=2: 2 warps 351, 4 warps 350, 8 warps 270 GS/s; Box-2D9P k=3: 654 / 692)
 #endif
 constexpr int RDG_WARPS = RDG_WARPS_PER_CTA;   // warps per CTA (independent streams)
+#ifndef RDG_S1LOAD
+#define RDG_S1LOAD 0   // 1: load stage 1's row before stages K .. 2 run (r02zzb: Box-2D49P 450 -> 447)
+#endif
 #ifndef RDG_S1FIRST
 #define RDG_S1FIRST 0   // 1: stage 1 before stages K .. 2 in each row iteration (r02zr: Box-2D49P 448 -> 426)
 #endif
@@ -591,6 +594,14 @@ __device__ __forceinline__ void fused_rows_loop(const double* __restrict__ st, i
       }
       fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 2, true, REM>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
                                                                orow);
+    } else if constexpr (RDG_S1LOAD) {   // stage 1's input row loaded first, stages K .. 2, then stage 1
+      double x1[NH][2 * R + 2];
+#pragma unroll
+      for (int h = 0; h < NH; ++h) load_x<R>(st + I * BW + 64 * h, p, x1[h]);
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, K, false, 2, true, REM>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
+                                                                    orow);
+      fused_iter<R, SIG, K, NH, FULL, 0, 0, 1, true, 1, true, REM>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, x1, I,
+                                                                   orow);
     } else if constexpr (RDG_S1FIRST) {   // stage 1, then stages K .. 2 (the stages of an iteration are independent)
       fused_iter<R, SIG, K, NH, FULL, 0, 0, 1, false, 1, true, REM>(st + I * BW, p, acc, P, bufs, par, in, out, P1, sc, lc, dp, xq, I,
                                                                     orow);
