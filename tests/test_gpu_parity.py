@@ -455,3 +455,44 @@ def test_small_cluster_path_bitwise(kind, h, shape, monkeypatch):
         assert np.array_equal(out_cl, ref_stream), (T, float(np.max(np.abs(out_cl - ref_stream))))
         assert np.array_equal(out_gr, ref_stream), (T, float(np.max(np.abs(out_gr - ref_stream))))
         assert rel_err(out, oracle.run(W, g, T)) <= 1e-12
+
+
+@pytest.mark.parametrize("kind", ["rsym", "heat3d"])
+@pytest.mark.parametrize("shape", [(40, 37, 70), (9, 130, 66)])
+def test_3d_symmetric_plane_forms(kind, shape, monkeypatch):
+    """3D CUDA-core engine, reading Q18: the joint evaluation of the symmetric planes
+    (Box-3D27P, PM_SYM3) and the FMA-accumulated Heat-3D form agree with the oracle to 1e-12 and with
+    the PMA / per-plane form (LORA_NO_SYM3=1) to rounding; fused (k = 2) and unfused runs of the
+    same form are bitwise equal."""
+    W = synth.rsym_weights(3, 1, 31) if kind == "rsym" else synth.preset("heat3d")
+    g = synth.grid(tuple(n + 2 for n in shape), 20240131)
+    T = 5
+    ref = oracle.run(W, g, T)
+    fused, info = run_gpu(W, g, T, engine="rdg_cuda", fuse_k=2)
+    unfused, _ = run_gpu(W, g, T, engine="rdg_cuda", fuse_k=1)
+    assert info["fuse_k"] == 2
+    assert np.array_equal(fused, unfused)
+    assert rel_err(fused, ref) <= 1e-12
+    monkeypatch.setenv("LORA_NO_SYM3", "1")
+    pma, info_p = run_gpu(W, g, T, engine="rdg_cuda", fuse_k=2)
+    monkeypatch.delenv("LORA_NO_SYM3")
+    assert rel_err(pma, ref) <= 1e-12
+    if kind == "rsym":
+        assert info["fma_per_point_issued"] == 12.5 and info_p["fma_per_point_issued"] == 15
+
+
+def test_p2p_view_pointers():
+    """lora_stencil_p2p_view: the caller-layout view of an exchange buffer (R-deep halos, same row pitch)
+    starts hl - R rows into the buffer; out-of-range indices give NULL."""
+    import paper_conf_sc_zhanglyczcy24_b200 as L
+    W = synth.rsym_weights(2, 3, 4)
+    st = L.Stencil(W, (64, 100), engine="rdg_cuda", fuse_k=2)
+    for nranks, rank in ((1, 0), (2, 0), (2, 1), (3, 1)):
+        ep = L.lora_stencil_p2p_create(st.plan, nranks, rank)
+        row = (100 + 6) * 8
+        hl = 6 if rank > 0 else 3                      # H = k R = 6 deep towards a lower neighbour
+        for i in (0, 1):
+            assert L.lora_stencil_p2p_view(ep, i) - L.lora_stencil_p2p_buffer(ep, i) == (hl - 3) * row
+        assert L.lora_stencil_p2p_view(ep, 2) == 0 and L.lora_stencil_p2p_view(ep, -1) == 0
+        L.lora_stencil_p2p_destroy(ep)
+    st.close()
