@@ -52,9 +52,9 @@ constexpr int RDG_WARPS = RDG_WARPS_PER_CTA;   // warps per CTA (independent str
 #define RDG_PF_HALVES 2   // 64-column halves of the next row prefetched (RDG_PF, loop form)
 #endif
 #ifndef RDG_NS_STAGES
-#define RDG_NS_STAGES 3
+#define RDG_NS_STAGES 2   // r02zzg/h: Box-2D49P 449 -> 454, Box-2D9P 716 -> 748, Star-2D13P 476 -> 499 GS/s vs 3 stages
 #endif
-constexpr int RDG_NS = RDG_NS_STAGES;   // ring stages per warp (3 keeps 4 CTAs = 16 warps per SM)
+constexpr int RDG_NS = RDG_NS_STAGES;   // TMA ring stages per warp
 
 enum { SIG_PMA = 0, SIG_STAR = 1, SIG_FULL = 2, SIG_DIRECT = 3, SIG_ROWS = 4 };   // DIRECT: W itself in u[][] (K11)
 
